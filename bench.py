@@ -1,0 +1,370 @@
+#!/usr/bin/env python
+"""Benchmark of the TileSpGEMM hot path: fp64 C = A^2 GFLOPS (2 x products / time) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl tsg|reference]
+
+One step = one tsg_spgemm call (steps 1-3 of Section 3.3 plus all allocation, the paper's timed
+region P:2969-2986), inputs resident in HBM, timed with CUDA events on the launching stream,
+max over ranks.  The default workload is C2 stencil27-128 (BASELINE.json configs[1]); its
+inputs (A: ~0.7 GB in tile form) are larger than the 126 MB L2, so no flush is needed; smaller
+configs flush L2 with a 512 MB write between timed steps (outside the events).
+
+Prints ONE JSON line (rank 0).  ``--impl reference`` times the CPU oracle (the reference arm of
+this tier) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "fp64 C=A^2 GFLOPS (2×products/time) at 1/2/4/8 B200; % HBM roofline"
+UNIT = "GFLOPS"
+L2_BYTES = 126 * 2 ** 20
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def tile_bytes(tm, ntiles, nnz):
+    """S(M) = 8(tm+1) + 60*tiles + 9*nnz."""
+    return 8 * (tm + 1) + 60 * ntiles + 9 * nnz
+
+
+class ClockSampler:
+    """nvidia-smi sampled every 200 ms while the timed region runs (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        time.sleep(0.3)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def oracle_baseline(A, budget_s: float = 12.0, max_rows=None):
+    """The oracle as it stands (single thread) on a bounded row sample of A*A."""
+    import oracle
+
+    oracle.build()
+    m = A.m
+    # calibrate on a small row block, then size the sample to ~budget_s seconds
+    probe = np.arange(0, min(m, 256), dtype=np.int64)
+    t0 = time.perf_counter()
+    oracle.spgemm(A, A, rows=probe)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    rows_per_s = len(probe) / dt
+    R = int(min(m, max(len(probe), rows_per_s * budget_s)))
+    if max_rows:
+        R = min(R, max_rows)
+    rows = np.arange(0, R, dtype=np.int64)
+    sub = gen_row_block(A, R)
+    prods = oracle.products(sub, A)
+    t0 = time.perf_counter()
+    C = oracle.spgemm(A, A, rows=rows)
+    el = time.perf_counter() - t0
+    return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
+                      f"(oracle/tsg_oracle.c), {el:.2f} s", "seconds": el, "products": int(prods)}
+
+
+def gen_row_block(A, R):
+    from workloads import gen
+
+    return gen.row_block(A, 0, R)
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle timed as it stands on bounded samples of the workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    from workloads import gen
+
+    A = gen.config(args.config)
+    for _ in range(args.warmup):
+        oracle_baseline(A, budget_s=2.0)
+    vals, secs, prods = [], 0.0, 0
+    last = None
+    for _ in range(args.steps):
+        last = oracle_baseline(A, budget_s=args.ref_step_s)
+        vals.append(last["value"])
+        secs += last["seconds"]
+        prods += last["products"]
+    value = 2.0 * prods / secs / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}", "n": A.m, "nnz_a": A.nnz},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": last["sample"]},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--impl", default="tsg", choices=["tsg", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget-s", type=float, default=12.0)
+    ap.add_argument("--ref-step-s", type=float, default=6.0)
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
+    args = ap.parse_args()
+    if args.warmup < 3 and not args.profile:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+
+    import paper_conf_ppopp_niuljs0022_b200 as tsg
+    from workloads import gen
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=dev)
+
+    A = gen.config(args.config)
+    stream = torch.cuda.current_stream()
+    T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.col).to(dev),
+                         torch.from_numpy(A.val).to(dev), (A.m, A.n))
+    # shard C tile rows across ranks (strong scaling of one matrix)
+    if world > 1:
+        from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
+
+        cuts = tdist.partition_tile_rows(A, A, world)
+        I0, I1 = int(cuts[rank]), int(cuts[rank + 1])
+        Ashard = tsg.slice_rows(T, I0, I1)
+    else:
+        I0, I1 = 0, T.tile_m
+        Ashard = T
+    # one instrumented call for the exact counts (products are a property of the input)
+    C0 = tsg.spgemm(Ashard, T, stats=True, products=True)
+    st0 = C0.stats
+    del C0
+    small_inputs = tile_bytes(T.tile_m, T.num_tiles, T.nnz) < 2 * L2_BYTES
+    flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev) if small_inputs else None
+
+    def one_step(timing=True):
+        return tsg.spgemm(Ashard, T, stats=True, timing=timing)
+
+    for _ in range(args.warmup):
+        C = one_step()
+        del C
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    launches0 = tsg.kernel_launch_count()
+    step_ms, s3_ms, s2_ms, s1_ms = [], [], [], []
+    stats_last = None
+    with ClockSampler(local) if not args.profile else _Null() as clk:
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        for _ in range(args.steps):
+            if flush is not None:
+                flush.fill_(1)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            C = one_step()
+            e1.record(stream)
+            e1.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+            st = C.stats
+            s1_ms.append(st["ms_step1"] + st["ms_index"])
+            s2_ms.append(st["ms_step2"])
+            s3_ms.append(st["ms_step3"])
+            stats_last = st
+            del C
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+    launches = tsg.kernel_launch_count() - launches0
+    local_ms = float(np.mean(step_ms))
+    ms = local_ms
+    prods_local = st0["products"]
+    prods = prods_local
+    if dist:
+        t = torch.tensor([local_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        p = torch.tensor([prods_local], dtype=torch.int64, device=dev)
+        dist.all_reduce(p)
+        prods = int(p.item())
+    value = 2.0 * prods / (ms / 1e3) / 1e9
+
+    # roofline of the dominant kernel (step 3 numeric unless another step is longer)
+    bw, bw_src = peaks()
+    nnzC, ntC = stats_last["nnz_c"], stats_last["tiles_c"]
+    steps_ms = {"step1": float(np.mean(s1_ms)), "step2": float(np.mean(s2_ms)), "step3": float(np.mean(s3_ms))}
+    alg = {  # algorithmic bytes per launch of each step's kernels
+        "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + 6 * T.num_tiles + 8 * (T.tile_m + 1) + 12 * ntC,
+        "step2": 32 * (Ashard.num_tiles + T.num_tiles) + 60 * ntC,
+        "step3": 9 * (Ashard.nnz + T.nnz + nnzC) + 48 * (Ashard.num_tiles + T.num_tiles) + 56 * ntC,
+    }
+    dom = max(steps_ms, key=steps_ms.get)
+    achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + tile_bytes(T.tile_m, T.num_tiles, T.nnz) + \
+        tile_bytes(Ashard.tile_m, ntC, nnzC)
+    roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",
+            "frac": achieved / bw, "traffic": traffic, "algorithmic_bytes": alg[dom], "peak_source": bw_src,
+            "kernel_ms": steps_ms[dom]}
+
+    # end to end through the public API with host buffers (H2D of A's CSR, D2H of C's tiles)
+    e2e = None
+    if not args.profile and args.e2e_steps > 0:
+        h_rp = torch.from_numpy(A.rowptr).pin_memory()
+        h_ci = torch.from_numpy(A.col).pin_memory()
+        h_v = torch.from_numpy(A.val).pin_memory()
+        Cx = one_step(timing=False)
+        bufs = {k: torch.empty(v.numel(), dtype=_host_dtype(v), pin_memory=True) for k, v in Cx.arrays().items()}
+        bo = sum(b.numel() * b.element_size() for b in bufs.values())
+        bi = h_rp.numel() * 8 + h_ci.numel() * 4 + h_v.numel() * 8
+        del Cx
+        torch.cuda.synchronize()
+        e2e_ms = []
+        for _ in range(args.e2e_steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            Th = tsg.csr_to_tiles(h_rp, h_ci, h_v, (A.m, A.n))
+            Ah = tsg.slice_rows(Th, I0, I1) if world > 1 else Th
+            Cx = tsg.spgemm(Ah, Th)
+            Cx.copy_to_host(bufs)
+            e1.record(stream)
+            e1.synchronize()
+            e2e_ms.append(e0.elapsed_time(e1))
+            del Cx, Ah, Th
+        em = float(np.mean(e2e_ms))
+        if dist:
+            t = torch.tensor([em], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            em = float(t.item())
+        e2e = {"value": 2.0 * prods / (em / 1e3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": int(bi),
+               "d2h_bytes_per_step": int(bo), "ms_per_step": em,
+               "includes": "H2D of A's CSR + tsg_csr_to_tiles + tsg_spgemm + D2H of C's tile arrays"}
+
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return 0
+    cpu = None
+    if not args.no_cpu_baseline and not args.profile and world == 1:
+        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s)
+        cpu.pop("seconds", None)
+        cpu.pop("products", None)
+    clocks = clk.summary() if not args.profile else None
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}", "n": A.m, "nnz_a": A.nnz,
+                   "products": prods, "nnz_c": nnzC if world == 1 else None, "tiles_c": ntC if world == 1 else None,
+                   "parallelism": f"tile-row shards x{world}" if world > 1 else "single GPU",
+                   "l2": ("512 MB flush between timed steps" if flush is not None else
+                          f"inputs larger than L2 (A tiles {tile_bytes(T.tile_m, T.num_tiles, T.nnz) / 1e6:.0f} MB > 126 MB)"),
+                   "step_ms": {k: round(v, 4) for k, v in steps_ms.items()},
+                   "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw},
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "clocks": clocks,
+    }
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+    return 0
+
+
+def _host_dtype(t):
+    import torch
+
+    return torch.int16 if t.dtype == torch.uint16 else t.dtype
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,263 @@
+"""B200-native TileSpGEMM hot path (Niu et al., PPoPP'22) -- Python binding.
+
+Argument marshalling only: every step of the path runs in libtsg.so's sm_100a kernels behind
+the C ABI of ``include/tsg.h``.  PyTorch provides device memory (input tensors), the current
+stream and process groups; results alias library-owned device memory as torch tensors.
+
+    import paper_conf_ppopp_niuljs0022_b200 as tsg
+    A = tsg.csr_to_tiles(rowptr, col, val, (m, n))        # torch CUDA tensors (int64/int32/float64)
+    C = tsg.spgemm(A, A)                                 # C = A^2 in the sparse-tile format
+    rp, ci, v = tsg.tiles_to_csr(C)                      # back to CSR (torch CUDA tensors)
+
+Names follow the paper: tile_ptr / tile_col / tile_nnz / row_ptr / mask / idx / val (Section 3.2,
+PAPER.md P:795-878).
+"""
+from __future__ import annotations
+
+import ctypes as C
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _lib
+from ._lib import TILE, DENSE_NNZ, TsgError  # noqa: F401
+
+__all__ = ["Tiles", "csr_to_tiles", "spgemm", "tiles_to_csr", "slice_rows", "wrap", "TsgError",
+           "kernel_launch_count"]
+
+_DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8)}
+
+
+class _DeviceArray:
+    """__cuda_array_interface__ over library memory; keeps the owning handle alive."""
+
+    def __init__(self, ptr: int, count: int, dtype: str, owner):
+        self._owner = owner
+        self.__cuda_array_interface__ = {"shape": (int(count),), "typestr": _DT[dtype][0],
+                                         "data": (int(ptr or 0) if count else 0, False), "version": 3,
+                                         "strides": None, "stream": None}
+
+
+def _torch():
+    import torch
+
+    return torch
+
+
+def _stream_ptr(stream=None) -> int:
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+class _Handle:
+    """Owns one tsg_tiles*; destroys it when the last reference (incl. tensor views) goes."""
+
+    def __init__(self, ptr: int):
+        self.ptr = ptr
+
+    def __del__(self):
+        if self.ptr:
+            try:
+                _lib.load().tsg_tiles_destroy(C.c_void_p(self.ptr), None)
+            except Exception:
+                pass
+            self.ptr = 0
+
+
+@dataclass
+class Tiles:
+    """A device-resident matrix in sparse-tile form (tensors alias the library's arrays)."""
+
+    handle: _Handle
+    m: int
+    n: int
+    tile_m: int
+    tile_n: int
+    num_tiles: int
+    nnz: int
+    tile_ptr: object
+    tile_col: object
+    tile_nnz: object
+    row_ptr: object
+    mask: object
+    idx: object
+    val: object
+    stats: dict | None = None
+
+    @property
+    def ptr(self) -> C.c_void_p:
+        return C.c_void_p(self.handle.ptr)
+
+    @property
+    def shape(self):
+        return (self.m, self.n)
+
+    def arrays(self) -> dict:
+        return {k: getattr(self, k) for k in ("tile_ptr", "tile_col", "tile_nnz", "row_ptr", "mask", "idx", "val")}
+
+    def copy_to_host(self, out: dict | None = None, stream=None) -> dict:
+        """Copy the seven arrays into host buffers (numpy or pinned torch CPU tensors) via the C ABI."""
+        sizes = {"tile_ptr": (self.tile_m + 1, np.int64), "tile_col": (self.num_tiles, np.int32),
+                 "tile_nnz": (self.num_tiles + 1, np.int64), "row_ptr": (16 * self.num_tiles, np.uint8),
+                 "mask": (16 * self.num_tiles, np.uint16), "idx": (self.nnz, np.uint8), "val": (self.nnz, np.float64)}
+        if out is None:
+            out = {k: np.empty(n, dt) for k, (n, dt) in sizes.items()}
+        ptrs = []
+        for k in sizes:
+            a = out[k]
+            ptrs.append(C.c_void_p(a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data))
+        _lib.check(_lib.load().tsg_tiles_copy_to_host(self.ptr, C.c_void_p(_stream_ptr(stream)), *ptrs))
+        return out
+
+
+def _from_handle(ptr: int, stats=None) -> Tiles:
+    L = _lib.load()
+    h = _Handle(ptr)
+    v = _lib.TilesView()
+    _lib.check(L.tsg_tiles_get_view(C.c_void_p(ptr), C.byref(v)))
+    torch = _torch()
+
+    def t(p, count, dt):
+        if count == 0:
+            return torch.empty(0, dtype=getattr(torch, dt), device="cuda")
+        return torch.as_tensor(_DeviceArray(p, count, dt, h), device="cuda")
+
+    return Tiles(h, v.m, v.n, v.tile_m, v.tile_n, v.num_tiles, v.nnz,
+                 t(v.tile_ptr, v.tile_m + 1, "int64"), t(v.tile_col, v.num_tiles, "int32"),
+                 t(v.tile_nnz, v.num_tiles + 1, "int64"), t(v.row_ptr, 16 * v.num_tiles, "uint8"),
+                 t(v.mask, 16 * v.num_tiles, "uint16"), t(v.idx, v.nnz, "uint8"), t(v.val, v.nnz, "float64"),
+                 stats)
+
+
+def _dptr(x, dtype) -> C.c_void_p:
+    torch = _torch()
+    if not isinstance(x, torch.Tensor) or not x.is_cuda:
+        raise TypeError("expected a CUDA torch tensor")
+    if x.dtype != dtype or not x.is_contiguous():
+        raise TypeError(f"expected a contiguous {dtype} tensor, got {x.dtype}")
+    return C.c_void_p(x.data_ptr() if x.numel() else 0)
+
+
+def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=None) -> Tiles:
+    """CSR -> sparse tiles on the GPU (tsg_csr_to_tiles).
+
+    Device input: torch CUDA tensors (int64 row_ptr, int32 col_idx, float64 val).
+    Host input: numpy arrays or CPU torch tensors (pinned for speed) -- copied in by the library.
+    """
+    torch = _torch()
+    m, n = int(shape[0]), int(shape[1])
+    L = _lib.load()
+    out = C.c_void_p()
+    flags = _lib.VALIDATE if validate else 0
+    host = not (isinstance(row_ptr, torch.Tensor) and row_ptr.is_cuda)
+    if host:
+        flags |= _lib.INPUT_HOST
+        arrs = []
+        for a, dt in ((row_ptr, np.int64), (col_idx, np.int32), (val, np.float64)):
+            if isinstance(a, torch.Tensor):
+                a = a.contiguous()
+                arrs.append((a, C.c_void_p(a.data_ptr() if a.numel() else 0)))
+            else:
+                a = np.ascontiguousarray(a, dtype=dt)
+                arrs.append((a, C.c_void_p(a.ctypes.data if a.size else 0)))
+        nnz = int(arrs[0][0][-1]) if m >= 0 and len(arrs[0][0]) else 0
+        rc = L.tsg_csr_to_tiles(m, n, nnz, arrs[0][1], arrs[1][1], arrs[2][1], flags, None,
+                                C.c_void_p(_stream_ptr(stream)), C.byref(out))
+    else:
+        nnz = int(col_idx.numel())
+        rc = L.tsg_csr_to_tiles(m, n, nnz, _dptr(row_ptr, torch.int64), _dptr(col_idx, torch.int32),
+                                _dptr(val, torch.float64), flags, None, C.c_void_p(_stream_ptr(stream)),
+                                C.byref(out))
+    _lib.check(rc)
+    return _from_handle(out.value)
+
+
+def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, products: bool = False,
+           scan_only: bool = False, list_always: bool = False, dense_threshold: int | None = None,
+           stream=None) -> Tiles:
+    """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3)."""
+    L = _lib.load()
+    flags = 0
+    if timing:
+        flags |= _lib.STATS_TIMING
+    if products:
+        flags |= _lib.STATS_PRODUCTS
+    if scan_only:
+        flags |= _lib.STEP1_SCAN_ONLY
+    if list_always:
+        flags |= _lib.STEP1_LIST_ALWAYS
+    if dense_threshold is not None:
+        if not 1 <= dense_threshold <= 257:
+            raise ValueError("dense_threshold must be in [1, 257]")
+        flags |= dense_threshold << _lib.DENSE_THRESHOLD_SHIFT
+    st = _lib.Stats() if (stats or timing or products) else None
+    out = C.c_void_p()
+    rc = L.tsg_spgemm(A.ptr, B.ptr, flags, None, C.c_void_p(_stream_ptr(stream)), C.byref(out),
+                      C.byref(st) if st is not None else None)
+    _lib.check(rc)
+    return _from_handle(out.value, st.as_dict() if st is not None else None)
+
+
+def tiles_to_csr(T: Tiles, stream=None):
+    """Sparse tiles -> CSR on the GPU; returns (row_ptr int64, col_idx int32, val float64) tensors."""
+    L = _lib.load()
+    torch = _torch()
+    rp, ci, v = C.c_void_p(), C.c_void_p(), C.c_void_p()
+    nnz = C.c_int64()
+    _lib.check(L.tsg_tiles_to_csr(T.ptr, None, C.c_void_p(_stream_ptr(stream)), C.byref(rp), C.byref(ci),
+                                  C.byref(v), C.byref(nnz)))
+    owner = _CsrOwner([rp.value, ci.value, v.value])
+
+    def t(p, count, dt):
+        if count == 0:
+            return torch.empty(0, dtype=getattr(torch, dt), device="cuda")
+        return torch.as_tensor(_DeviceArray(p, count, dt, owner), device="cuda")
+
+    return t(rp.value, T.m + 1, "int64"), t(ci.value, nnz.value, "int32"), t(v.value, nnz.value, "float64")
+
+
+class _CsrOwner:
+    def __init__(self, ptrs):
+        self.ptrs = ptrs
+
+    def __del__(self):
+        try:
+            L = _lib.load()
+            for p in self.ptrs:
+                if p:
+                    L.tsg_free(C.c_void_p(p), 0, None, None)
+        except Exception:
+            pass
+
+
+def slice_rows(T: Tiles, tile_row_begin: int, tile_row_end: int, stream=None) -> Tiles:
+    """Zero-copy view of tile rows [begin, end) (tsg_tiles_slice_rows).  Keeps T alive."""
+    out = C.c_void_p()
+    _lib.check(_lib.load().tsg_tiles_slice_rows(T.ptr, int(tile_row_begin), int(tile_row_end),
+                                                C.c_void_p(_stream_ptr(stream)), C.byref(out)))
+    V = _from_handle(out.value)
+    V.handle.parent = T.handle  # the view borrows T's arrays
+    return V
+
+
+def wrap(m: int, n: int, arrays: dict, keepalive=None) -> Tiles:
+    """Borrowing handle over seven torch CUDA tensors laid out as Section 3.2 (tsg_tiles_wrap)."""
+    torch = _torch()
+    v = _lib.TilesView()
+    v.m, v.n = int(m), int(n)
+    v.tile_m, v.tile_n = (m + TILE - 1) // TILE, (n + TILE - 1) // TILE
+    v.num_tiles = int(arrays["tile_col"].numel())
+    v.nnz = int(arrays["val"].numel())
+    for k, dt in (("tile_ptr", torch.int64), ("tile_col", torch.int32), ("tile_nnz", torch.int64),
+                  ("row_ptr", torch.uint8), ("mask", torch.uint16), ("idx", torch.uint8), ("val", torch.float64)):
+        setattr(v, k, _dptr(arrays[k], dt).value)
+    out = C.c_void_p()
+    _lib.check(_lib.load().tsg_tiles_wrap(C.byref(v), None, C.byref(out)))
+    T = _from_handle(out.value)
+    T.handle.keep = (arrays, keepalive)
+    return T
+
+
+def kernel_launch_count() -> int:
+    return int(_lib.load().tsg_kernel_launch_count())

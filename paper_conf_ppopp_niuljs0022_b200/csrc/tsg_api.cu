@@ -1,0 +1,324 @@
+// tsg_api.cu -- the extern "C" boundary of libtsg (include/tsg.h): argument validation, handle
+// lifetime, allocation policy, error translation.  Every compute step lives in the kernels of
+// tsg_convert.cu / tsg_spgemm.cu; this file launches nothing but two tiny rebase kernels.
+#include <cstring>
+
+#include "tsg_internal.cuh"
+
+namespace tsg {
+
+std::atomic<int64_t> g_launches{0};
+static thread_local std::string t_last_error;
+static thread_local int64_t t_call_launches = 0;
+
+void set_last_error(const std::string &msg) { t_last_error = msg; }
+void note_launch() { t_call_launches++; }
+void reset_call_launches() { t_call_launches = 0; }
+int64_t call_launches() { return t_call_launches; }
+
+static void ensure_pool_cached() {
+    // keep freed blocks in the device's default pool (a caching allocator, reading A15)
+    static std::atomic<int> done{-1};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return;
+    if (done.load() == dev) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    done.store(dev);
+}
+
+void *Allocator::alloc(size_t bytes, cudaStream_t s) const {
+    if (custom) return hook.alloc(bytes, (void *)s, hook.ctx);
+    ensure_pool_cached();
+    void *p = nullptr;
+    cudaError_t e = cudaMallocAsync(&p, bytes, s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();  // clear the sticky-free error state of a failed allocation
+        return nullptr;
+    }
+    return p;
+}
+
+void Allocator::free(void *p, size_t bytes, cudaStream_t s) const {
+    if (!p) return;
+    if (custom)
+        hook.free(p, bytes, (void *)s, hook.ctx);
+    else
+        cudaFreeAsync(p, s);
+}
+
+int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {
+    int64_t v = 0;
+    TSG_CUDA(cudaMemcpyAsync(&v, dptr, sizeof(v), cudaMemcpyDeviceToHost, s));
+    TSG_CUDA(cudaStreamSynchronize(s));
+    return v;
+}
+
+namespace {
+__global__ void k_rebase(const int64_t *__restrict__ src, int64_t *__restrict__ dst, int64_t count) {
+    int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < count) dst[i] = src[i] - src[0];
+}
+}  // namespace
+
+void launch_rebase(const int64_t *src, int64_t *dst, int64_t count, cudaStream_t s) {
+    TSG_LAUNCH(k_rebase, grid_for(count, 256), 256, 0, s, src, dst, count);
+}
+
+static void destroy_handle(tsg_tiles *T, cudaStream_t s) {
+    if (!T) return;
+    for (int i = 0; i < 7; i++)
+        if (T->owns[i]) T->al.free(T->array(i), T->bytes[i], s);
+    delete T;
+}
+
+template <typename F>
+static tsg_status guarded(F &&f) {
+    try {
+        f();
+        return TSG_OK;
+    } catch (const Error &e) {
+        set_last_error(e.msg);
+        return e.status;
+    } catch (const std::bad_alloc &) {
+        set_last_error("host allocation failed");
+        return TSG_ERR_OOM;
+    } catch (...) {
+        set_last_error("unknown internal error");
+        return TSG_ERR_INTERNAL;
+    }
+}
+
+}  // namespace tsg
+
+using namespace tsg;
+
+extern "C" {
+
+const char *tsg_status_string(tsg_status s) {
+    switch (s) {
+        case TSG_OK: return "TSG_OK";
+        case TSG_ERR_INVALID_ARG: return "TSG_ERR_INVALID_ARG";
+        case TSG_ERR_SHAPE: return "TSG_ERR_SHAPE";
+        case TSG_ERR_UNSORTED: return "TSG_ERR_UNSORTED";
+        case TSG_ERR_OVERFLOW: return "TSG_ERR_OVERFLOW";
+        case TSG_ERR_OOM: return "TSG_ERR_OOM";
+        case TSG_ERR_CUDA: return "TSG_ERR_CUDA";
+        case TSG_ERR_INTERNAL: return "TSG_ERR_INTERNAL";
+    }
+    return "TSG_ERR_UNKNOWN";
+}
+
+const char *tsg_last_error(void) { return t_last_error.c_str(); }
+int tsg_abi_version(void) { return TSG_ABI_VERSION; }
+int64_t tsg_kernel_launch_count(void) { return g_launches.load(); }
+
+tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *row_ptr,
+                            const int32_t *col_idx, const double *val, uint32_t flags,
+                            const tsg_allocator *al, void *stream, tsg_tiles **out) {
+    if (out) *out = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(out, TSG_ERR_INVALID_ARG, "out is NULL");
+        TSG_REQUIRE(m >= 0 && n >= 0 && nnz >= 0, TSG_ERR_INVALID_ARG, "negative size");
+        TSG_REQUIRE(row_ptr, TSG_ERR_INVALID_ARG, "row_ptr is NULL");
+        TSG_REQUIRE(nnz == 0 || (col_idx && val), TSG_ERR_INVALID_ARG, "col_idx/val NULL with nnz > 0");
+        TSG_REQUIRE((flags & ~(uint32_t)(TSG_INPUT_HOST | TSG_VALIDATE)) == 0, TSG_ERR_INVALID_ARG, "unknown flag");
+        TSG_REQUIRE(n < ((int64_t)1 << 31) && m < ((int64_t)1 << 35), TSG_ERR_OVERFLOW, "dimension too large");
+        cudaStream_t s = (cudaStream_t)stream;
+        Allocator A = Allocator::from(al);
+        tsg_tiles *T = new tsg_tiles();
+        T->al = A;
+        try {
+            if (flags & TSG_INPUT_HOST) {
+                Buffers staging(A, s);
+                int64_t *drp = staging.get<int64_t>(m + 1);
+                int32_t *dci = staging.get<int32_t>(nnz);
+                double *dv = staging.get<double>(nnz);
+                TSG_CUDA(cudaMemcpyAsync(drp, row_ptr, sizeof(int64_t) * (m + 1), cudaMemcpyHostToDevice, s));
+                if (nnz) {
+                    TSG_CUDA(cudaMemcpyAsync(dci, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, s));
+                    TSG_CUDA(cudaMemcpyAsync(dv, val, sizeof(double) * nnz, cudaMemcpyHostToDevice, s));
+                }
+                launch_csr_to_tiles(m, n, nnz, drp, dci, dv, flags & TSG_VALIDATE, A, s, T);
+            } else {
+                launch_csr_to_tiles(m, n, nnz, row_ptr, col_idx, val, flags & TSG_VALIDATE, A, s, T);
+            }
+        } catch (...) {
+            destroy_handle(T, s);
+            throw;
+        }
+        *out = T;
+    });
+}
+
+tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const tsg_allocator *al,
+                      void *stream, tsg_tiles **C, tsg_stats *stats) {
+    if (C) *C = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(A && B && C, TSG_ERR_INVALID_ARG, "NULL handle");
+        TSG_REQUIRE(A->n == B->m, TSG_ERR_SHAPE, "A.n != B.m");
+        cudaStream_t s = (cudaStream_t)stream;
+        Allocator al_ = Allocator::from(al);
+        tsg_tiles *T = new tsg_tiles();
+        T->al = al_;
+        try {
+            run_spgemm(A, B, flags, al_, s, T, stats);
+        } catch (...) {
+            destroy_handle(T, s);
+            throw;
+        }
+        *C = T;
+    });
+}
+
+tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *stream, int64_t **row_ptr,
+                            int32_t **col_idx, double **val, int64_t *nnz) {
+    if (row_ptr) *row_ptr = nullptr;
+    if (col_idx) *col_idx = nullptr;
+    if (val) *val = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(T && row_ptr && col_idx && val, TSG_ERR_INVALID_ARG, "NULL argument");
+        cudaStream_t s = (cudaStream_t)stream;
+        Allocator A = Allocator::from(al);
+        Buffers out(A, s);
+        int64_t *rp = out.get<int64_t>(T->m + 1);
+        int32_t *ci = out.get<int32_t>(T->nnz);
+        double *v = out.get<double>(T->nnz);
+        launch_tiles_to_csr(T, rp, ci, v, s);
+        out.take(rp);
+        out.take(ci);
+        out.take(v);
+        *row_ptr = rp;
+        *col_idx = ci;
+        *val = v;
+        if (nnz) *nnz = T->nnz;
+    });
+}
+
+tsg_status tsg_tiles_get_view(const tsg_tiles *T, tsg_tiles_view *o) {
+    return guarded([&] {
+        TSG_REQUIRE(T && o, TSG_ERR_INVALID_ARG, "NULL argument");
+        o->m = T->m;
+        o->n = T->n;
+        o->tile_m = T->tm;
+        o->tile_n = T->tn;
+        o->num_tiles = T->nt;
+        o->nnz = T->nnz;
+        o->tile_ptr = T->tile_ptr;
+        o->tile_col = T->tile_col;
+        o->tile_nnz = T->tile_nnz;
+        o->row_ptr = T->row_ptr;
+        o->mask = T->mask;
+        o->idx = T->idx;
+        o->val = T->val;
+    });
+}
+
+tsg_status tsg_tiles_wrap(const tsg_tiles_view *v, const tsg_allocator *owner, tsg_tiles **out) {
+    if (out) *out = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(v && out, TSG_ERR_INVALID_ARG, "NULL argument");
+        TSG_REQUIRE(v->m >= 0 && v->n >= 0 && v->num_tiles >= 0 && v->nnz >= 0, TSG_ERR_INVALID_ARG, "negative size");
+        TSG_REQUIRE(v->tile_m == ceil_div(v->m, TILE) && v->tile_n == ceil_div(v->n, TILE), TSG_ERR_INVALID_ARG,
+                    "tile_m/tile_n inconsistent with m/n");
+        TSG_REQUIRE(v->tile_ptr && v->tile_nnz, TSG_ERR_INVALID_ARG, "tile_ptr/tile_nnz NULL");
+        tsg_tiles *T = new tsg_tiles();
+        T->m = v->m;
+        T->n = v->n;
+        T->tm = v->tile_m;
+        T->tn = v->tile_n;
+        T->nt = v->num_tiles;
+        T->nnz = v->nnz;
+        T->tile_ptr = const_cast<int64_t *>(v->tile_ptr);
+        T->tile_col = const_cast<int32_t *>(v->tile_col);
+        T->tile_nnz = const_cast<int64_t *>(v->tile_nnz);
+        T->row_ptr = const_cast<uint8_t *>(v->row_ptr);
+        T->mask = const_cast<uint16_t *>(v->mask);
+        T->idx = const_cast<uint8_t *>(v->idx);
+        T->val = const_cast<double *>(v->val);
+        if (owner) {
+            T->al = Allocator::from(owner);
+            TSG_REQUIRE(T->al.custom, TSG_ERR_INVALID_ARG, "owner allocator needs alloc and free");
+            size_t b[7] = {sizeof(int64_t) * (size_t)(T->tm + 1), sizeof(int32_t) * (size_t)T->nt,
+                           sizeof(int64_t) * (size_t)(T->nt + 1), (size_t)(16 * T->nt),
+                           sizeof(uint16_t) * (size_t)(16 * T->nt), (size_t)T->nnz, sizeof(double) * (size_t)T->nnz};
+            for (int i = 0; i < 7; i++) {
+                T->owns[i] = true;
+                T->bytes[i] = b[i];
+            }
+        }
+        *out = T;
+    });
+}
+
+tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t b, int64_t e, void *stream, tsg_tiles **view) {
+    if (view) *view = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(T && view, TSG_ERR_INVALID_ARG, "NULL argument");
+        TSG_REQUIRE(0 <= b && b <= e && e <= T->tm, TSG_ERR_INVALID_ARG, "tile row range out of bounds");
+        cudaStream_t s = (cudaStream_t)stream;
+        int64_t t0 = 0, t1 = 0, z0 = 0, z1 = 0;
+        TSG_CUDA(cudaMemcpyAsync(&t0, T->tile_ptr + b, 8, cudaMemcpyDeviceToHost, s));
+        TSG_CUDA(cudaMemcpyAsync(&t1, T->tile_ptr + e, 8, cudaMemcpyDeviceToHost, s));
+        TSG_CUDA(cudaStreamSynchronize(s));
+        TSG_CUDA(cudaMemcpyAsync(&z0, T->tile_nnz + t0, 8, cudaMemcpyDeviceToHost, s));
+        TSG_CUDA(cudaMemcpyAsync(&z1, T->tile_nnz + t1, 8, cudaMemcpyDeviceToHost, s));
+        TSG_CUDA(cudaStreamSynchronize(s));
+        Allocator A;  // default pool for the two rebased offset arrays
+        Buffers buf(A, s);
+        int64_t *tp = buf.get<int64_t>(e - b + 1);
+        int64_t *tz = buf.get<int64_t>(t1 - t0 + 1);
+        launch_rebase(T->tile_ptr + b, tp, e - b + 1, s);
+        launch_rebase(T->tile_nnz + t0, tz, t1 - t0 + 1, s);
+        tsg_tiles *V = new tsg_tiles();
+        V->m = std::min<int64_t>(TILE * (e - b), T->m - TILE * b);
+        if (V->m < 0) V->m = 0;
+        V->n = T->n;
+        V->tm = e - b;
+        V->tn = T->tn;
+        V->nt = t1 - t0;
+        V->nnz = z1 - z0;
+        V->tile_ptr = tp;
+        V->tile_col = T->tile_col + t0;
+        V->tile_nnz = tz;
+        V->row_ptr = T->row_ptr + 16 * t0;
+        V->mask = T->mask + 16 * t0;
+        V->idx = T->idx + z0;
+        V->val = T->val + z0;
+        V->al = A;
+        V->owns[0] = V->owns[2] = true;
+        V->bytes[0] = buf.take(tp);
+        V->bytes[2] = buf.take(tz);
+        *view = V;
+    });
+}
+
+tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
+                                  int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, double *val) {
+    return guarded([&] {
+        TSG_REQUIRE(T, TSG_ERR_INVALID_ARG, "NULL handle");
+        cudaStream_t s = (cudaStream_t)stream;
+        auto cp = [&](void *dst, const void *src, size_t bytes) {
+            if (dst && bytes) TSG_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, s));
+        };
+        cp(tile_ptr, T->tile_ptr, sizeof(int64_t) * (T->tm + 1));
+        cp(tile_col, T->tile_col, sizeof(int32_t) * T->nt);
+        cp(tile_nnz, T->tile_nnz, sizeof(int64_t) * (T->nt + 1));
+        cp(row_ptr, T->row_ptr, 16 * T->nt);
+        cp(mask, T->mask, sizeof(uint16_t) * 16 * T->nt);
+        cp(idx, T->idx, T->nnz);
+        cp(val, T->val, sizeof(double) * T->nnz);
+        TSG_CUDA(cudaStreamSynchronize(s));
+    });
+}
+
+void tsg_tiles_destroy(tsg_tiles *T, void *stream) { destroy_handle(T, (cudaStream_t)stream); }
+
+void tsg_free(void *ptr, size_t bytes, const tsg_allocator *al, void *stream) {
+    Allocator::from(al).free(ptr, bytes, (cudaStream_t)stream);
+}
+
+}  // extern "C"

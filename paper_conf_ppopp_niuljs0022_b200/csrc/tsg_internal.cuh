@@ -1,0 +1,173 @@
+// tsg_internal.cuh -- shared internals of libtsg (handle layout, allocation, errors, launches).
+// Nothing here is visible through the C ABI (include/tsg.h).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <string>
+#include <vector>
+
+#include "../../include/tsg.h"
+
+namespace tsg {
+
+constexpr int TILE = TSG_TILE;
+
+// ------------------------------------------------------------------------------------------
+// errors: thrown inside the library, converted to tsg_status at the ABI boundary
+// ------------------------------------------------------------------------------------------
+struct Error {
+    tsg_status status;
+    std::string msg;
+};
+
+void set_last_error(const std::string &msg);
+
+[[noreturn]] inline void fail(tsg_status s, const std::string &msg) { throw Error{s, msg}; }
+
+#define TSG_CUDA(call)                                                                          \
+    do {                                                                                        \
+        cudaError_t e_ = (call);                                                                \
+        if (e_ != cudaSuccess)                                                                  \
+            ::tsg::fail(e_ == cudaErrorMemoryAllocation ? TSG_ERR_OOM : TSG_ERR_CUDA,           \
+                        std::string(#call) + ": " + cudaGetErrorString(e_) + " @" __FILE__ ":" + \
+                            std::to_string(__LINE__));                                          \
+    } while (0)
+
+#define TSG_REQUIRE(cond, status, msg)                    \
+    do {                                                  \
+        if (!(cond)) ::tsg::fail((status), (msg));        \
+    } while (0)
+
+// launch bookkeeping: every kernel goes through TSG_LAUNCH so the evidence counter is exact
+extern std::atomic<int64_t> g_launches;
+
+#define TSG_LAUNCH(kernel, grid, block, smem, stream, ...)                                     \
+    do {                                                                                        \
+        if ((grid) > 0) {                                                                       \
+            kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);                         \
+            ::tsg::g_launches.fetch_add(1, std::memory_order_relaxed);                          \
+            ::tsg::note_launch();                                                               \
+            TSG_CUDA(cudaGetLastError());                                                       \
+        }                                                                                       \
+    } while (0)
+
+void note_launch();  // per-call counter (thread-local)
+
+// ------------------------------------------------------------------------------------------
+// allocation: either the user's stream-ordered hook or cudaMallocAsync on the default pool
+// ------------------------------------------------------------------------------------------
+struct Allocator {
+    tsg_allocator hook{};
+    bool custom = false;
+    static Allocator from(const tsg_allocator *al) {
+        Allocator a;
+        if (al && al->alloc && al->free) {
+            a.hook = *al;
+            a.custom = true;
+        }
+        return a;
+    }
+    void *alloc(size_t bytes, cudaStream_t s) const;
+    void free(void *p, size_t bytes, cudaStream_t s) const;
+};
+
+// RAII list of device buffers; frees (stream-ordered) whatever is still owned at scope exit.
+class Buffers {
+   public:
+    Buffers(const Allocator &al, cudaStream_t s) : al_(al), s_(s) {}
+    ~Buffers() { release_all(); }
+    template <typename T>
+    T *get(int64_t count) {
+        size_t bytes = sizeof(T) * (size_t)(count > 0 ? count : 0);
+        if (bytes < 256) bytes = 256;  // never hand out NULL; keep 256-byte alignment
+        void *p = al_.alloc(bytes, s_);
+        if (!p) fail(TSG_ERR_OOM, "device allocation of " + std::to_string(bytes) + " bytes failed");
+        items_.push_back({p, bytes});
+        return static_cast<T *>(p);
+    }
+    // detach a buffer from the list (ownership moves to a handle); returns its byte size
+    size_t take(void *p) {
+        for (size_t i = 0; i < items_.size(); i++)
+            if (items_[i].p == p) {
+                size_t b = items_[i].bytes;
+                items_[i] = items_.back();
+                items_.pop_back();
+                return b;
+            }
+        fail(TSG_ERR_INTERNAL, "take() of an unknown buffer");
+    }
+    void release_all() {
+        for (auto &it : items_) al_.free(it.p, it.bytes, s_);
+        items_.clear();
+    }
+
+   private:
+    struct Item {
+        void *p;
+        size_t bytes;
+    };
+    Allocator al_;
+    cudaStream_t s_;
+    std::vector<Item> items_;
+};
+
+}  // namespace tsg
+
+// ------------------------------------------------------------------------------------------
+// the handle (opaque in the ABI)
+// ------------------------------------------------------------------------------------------
+struct tsg_tiles {
+    int64_t m = 0, n = 0, tm = 0, tn = 0, nt = 0, nnz = 0;
+    int64_t *tile_ptr = nullptr;
+    int32_t *tile_col = nullptr;
+    int64_t *tile_nnz = nullptr;
+    uint8_t *row_ptr = nullptr;
+    uint16_t *mask = nullptr;
+    uint8_t *idx = nullptr;
+    double *val = nullptr;
+    // ownership: which arrays this handle frees, their byte sizes, and through what
+    tsg::Allocator al;
+    bool owns[7] = {false, false, false, false, false, false, false};
+    size_t bytes[7] = {0, 0, 0, 0, 0, 0, 0};
+    void *array(int i) const {
+        void *a[7] = {tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val};
+        return a[i];
+    }
+};
+
+namespace tsg {
+
+// ------------------------------------------------------------------------------------------
+// device scan: out[0] = 0, out[i+1] = out[i] + in[i]; out has n+1 entries; out may alias in
+// when Tin == int64_t.  Three-phase (reduce / scan sums / downsweep), recursive on the sums.
+// ------------------------------------------------------------------------------------------
+template <typename Tin>
+void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buffers &tmp);
+
+// read one int64 from device memory (blocking on stream s)
+int64_t read_scalar(const int64_t *dptr, cudaStream_t s);
+
+// per-call launch counter access (thread-local)
+void reset_call_launches();
+int64_t call_launches();
+
+// kernels shared by the API translation units
+void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,
+                         const double *v, bool validate, const Allocator &al, cudaStream_t s,
+                         tsg_tiles *out);
+void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, double *v, cudaStream_t s);
+void launch_rebase(const int64_t *src, int64_t *dst, int64_t count, cudaStream_t s);
+void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Allocator &al,
+                cudaStream_t s, tsg_tiles *C, tsg_stats *stats);
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline unsigned grid_for(int64_t work, int per_block, int64_t cap = 1 << 30) {
+    int64_t g = ceil_div(work, per_block);
+    if (g > cap) g = cap;
+    return (unsigned)(g > 0 ? g : 0);
+}
+
+}  // namespace tsg

@@ -1,0 +1,87 @@
+"""The C-ABI library loads and exports every entry point include/tsg.h declares (no GPU needed)."""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import re
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "tsg.h")
+LIB = os.path.join(ROOT, "paper_conf_ppopp_niuljs0022_b200", "libtsg.so")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    # build in-tree if needed (nvcc cross-compiles sm_100a without a GPU)
+    subprocess.check_call(["make", "-s", "-j8", "paper_conf_ppopp_niuljs0022_b200/libtsg.so"], cwd=ROOT)
+    return C.CDLL(LIB)
+
+
+def declared_symbols():
+    text = open(HEADER).read()
+    return sorted(set(re.findall(r"^TSG_API\s+[\w\s\*]*?\b(tsg_\w+)\s*\(", text, flags=re.M)))
+
+
+def test_header_declares_the_boundary():
+    syms = declared_symbols()
+    for name in ("tsg_csr_to_tiles", "tsg_spgemm", "tsg_tiles_to_csr"):
+        assert name in syms
+    assert len(syms) >= 13
+
+
+def test_library_exports_every_declared_symbol(lib):
+    out = subprocess.check_output(["nm", "-D", "--defined-only", LIB], text=True)
+    exported = set(re.findall(r"\sT\s+(tsg_\w+)", out))
+    missing = [s for s in declared_symbols() if s not in exported]
+    assert not missing, missing
+    for s in declared_symbols():
+        assert getattr(lib, s) is not None
+
+
+def test_binding_lists_every_symbol(lib):
+    from paper_conf_ppopp_niuljs0022_b200 import _lib
+
+    assert sorted(_lib.SYMBOLS) == declared_symbols()
+
+
+def test_non_compute_entry_points(lib):
+    lib.tsg_status_string.restype = C.c_char_p
+    assert lib.tsg_status_string(0) == b"TSG_OK"
+    assert lib.tsg_status_string(5) == b"TSG_ERR_OOM"
+    assert lib.tsg_abi_version() == 1
+    lib.tsg_last_error.restype = C.c_char_p
+    assert isinstance(lib.tsg_last_error(), bytes)
+
+
+def test_invalid_arguments_are_rejected_without_a_gpu(lib):
+    """Argument validation happens before any CUDA call: NULL/negative inputs return INVALID_ARG."""
+    out = C.c_void_p()
+    lib.tsg_csr_to_tiles.argtypes = [C.c_int64] * 3 + [C.c_void_p] * 3 + [C.c_uint32, C.c_void_p, C.c_void_p,
+                                                                           C.POINTER(C.c_void_p)]
+    assert lib.tsg_csr_to_tiles(-1, 4, 0, None, None, None, 0, None, None, C.byref(out)) == 1
+    assert lib.tsg_csr_to_tiles(4, 4, 0, None, None, None, 0, None, None, C.byref(out)) == 1
+    assert out.value is None
+    lib.tsg_spgemm.argtypes = [C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.POINTER(C.c_void_p),
+                               C.c_void_p]
+    assert lib.tsg_spgemm(None, None, 0, None, None, C.byref(out), None) == 1
+
+
+def test_product_path_fails_loudly_without_the_library(tmp_path):
+    code = ("import paper_conf_ppopp_niuljs0022_b200._lib as L\n"
+            "try:\n    L.load()\nexcept ImportError as e:\n    print('IMPORT-ERROR', e)\n")
+    env = dict(os.environ, TSG_LIBRARY=str(tmp_path / "missing.so"), PYTHONPATH=ROOT)
+    res = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, cwd=ROOT)
+    assert "IMPORT-ERROR" in res.stdout
+
+
+def test_product_package_never_imports_the_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_ppopp_niuljs0022_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                text = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in text and "from oracle" not in text and "tsg_oracle" not in text, f

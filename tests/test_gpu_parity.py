@@ -1,0 +1,301 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar (BASELINE.json north_star): structure bit-exact (tile_ptr, tile_col, tile_nnz, row_ptr, mask,
+idx, CSR row_ptr/col) and fp64 values within |c - c_ref| <= 1e-12 * sum|a*b| per entry.  The
+kernels sum in ascending k with FMA (reading A8/A16), so values are also compared bitwise
+against the oracle's fma mode (+0 == -0).
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+from tests.helpers import assert_values_close, bitwise_equal_values, csr_dense
+from workloads import gen
+
+pytestmark = pytest.mark.gpu
+
+ARRAYS = ("tile_ptr", "tile_col", "tile_nnz", "row_ptr", "mask", "idx", "val")
+
+
+@pytest.fixture(scope="module")
+def tsg(cuda_device):
+    import paper_conf_ppopp_niuljs0022_b200 as m
+
+    return m
+
+
+def to_dev(A):
+    import torch
+
+    return (torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.col).cuda(), torch.from_numpy(A.val).cuda())
+
+
+def tiles_of(tsg, A):
+    rp, ci, v = to_dev(A)
+    return tsg.csr_to_tiles(rp, ci, v, (A.m, A.n))
+
+
+def host(T) -> dict:
+    import torch
+
+    out = {}
+    for k in ARRAYS:
+        x = getattr(T, k)
+        if x.dtype == torch.uint16:
+            x = x.view(torch.int16)
+        a = x.cpu().numpy()
+        out[k] = a.view(np.uint16) if k == "mask" else a
+    return out
+
+
+def assert_tiles_equal(got: dict, ref, values="bitwise", absref=None):
+    for k in ARRAYS[:-1]:
+        exp = getattr(ref, k)
+        assert got[k].shape == exp.shape, (k, got[k].shape, exp.shape)
+        assert np.array_equal(got[k], exp), k
+    if values == "bitwise":
+        assert bitwise_equal_values(got["val"], ref.val)
+
+
+# ------------------------------------------------------------------------------------------
+# a5 / a6: conversion
+# ------------------------------------------------------------------------------------------
+CONVERT_CASES = [
+    lambda: gen.config("C1"),
+    lambda: gen.random_sparse(1, 1, 1.0, 1),
+    lambda: gen.random_sparse(15, 17, 0.3, 2),
+    lambda: gen.random_sparse(17, 100, 0.05, 3),
+    lambda: gen.random_sparse(1000, 1000, 0.003, 4, empty_rows=[0, 5, 999]),
+    lambda: gen.random_sparse(0, 5, 0.5, 5),
+    lambda: gen.random_sparse(40, 40, 0.0, 6),
+    lambda: gen.dense_block(48, 33),
+    lambda: gen.rmat(11),
+    lambda: gen.hub(700, hub_rows=(3,), hub_cols=(5,), density=0.002),
+]
+
+
+@pytest.mark.parametrize("case", range(len(CONVERT_CASES)))
+def test_csr_to_tiles_bitwise(tsg, case):
+    A = CONVERT_CASES[case]()
+    T = tiles_of(tsg, A)
+    ref = oracle.csr_to_tiles(A)
+    assert (T.m, T.n, T.num_tiles, T.nnz) == (A.m, A.n, ref.num_tiles, ref.nnz)
+    assert_tiles_equal(host(T), ref)
+    rp, ci, v = tsg.tiles_to_csr(T)
+    assert np.array_equal(rp.cpu().numpy(), A.rowptr)
+    assert np.array_equal(ci.cpu().numpy(), A.col)
+    assert np.array_equal(v.cpu().numpy(), A.val)
+
+
+def test_csr_to_tiles_host_input_and_validation(tsg):
+    A = gen.random_sparse(100, 90, 0.05, 7)
+    T = tsg.csr_to_tiles(A.rowptr, A.col, A.val, (A.m, A.n), validate=True)
+    assert_tiles_equal(host(T), oracle.csr_to_tiles(A))
+    bad = gen.CSR(2, 4, np.array([0, 2, 3]), np.array([2, 1, 0], np.int32), np.ones(3))
+    with pytest.raises(tsg.TsgError) as e:
+        tsg.csr_to_tiles(bad.rowptr, bad.col, bad.val, (2, 4), validate=True)
+    assert e.value.name == "TSG_ERR_UNSORTED"
+
+
+# ------------------------------------------------------------------------------------------
+# a0-a4: spgemm parity
+# ------------------------------------------------------------------------------------------
+def pair_cases():
+    c = []
+    A = gen.config("C1")
+    c.append(("C1", A, A))
+    c.append(("C1-pinned", gen.poisson2d(64, "pinned"), gen.poisson2d(64, "pinned")))
+    S = gen.stencil27(10)
+    c.append(("stencil27-10", S, S))
+    F = gen.strip_fem(8, 30, 6)
+    c.append(("strip-fem-8x30", F, F))  # dense-accumulator tiles
+    R = gen.rmat(12)
+    c.append(("rmat-12", R, R))
+    c.append(("rect", gen.random_sparse(37, 50, 0.08, 1), gen.random_sparse(50, 23, 0.1, 2)))
+    c.append(("ragged", gen.random_sparse(100, 115, 0.03, 3), gen.random_sparse(115, 81, 0.03, 4)))
+    c.append(("single", gen.from_coo(20, 20, [7], [11], [2.5]), gen.from_coo(20, 20, [11], [3], [-4.0])))
+    c.append(("empty-A", gen.random_sparse(64, 64, 0.0, 1), gen.random_sparse(64, 64, 0.1, 1)))
+    c.append(("no-products", gen.from_coo(32, 32, [0], [1], [1.0]), gen.from_coo(32, 32, [2], [3], [1.0])))
+    D = gen.dense_block(64, 64)
+    c.append(("dense-64", D, D))
+    c.append(("hub", gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004),
+              gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)))
+    c.append(("identity", gen.identity(300, 3.0), gen.random_sparse(300, 300, 0.02, 9)))
+    c.append(("perm", gen.permutation(257, 1), gen.permutation(257, 2)))
+    return c
+
+
+PAIRS = pair_cases()
+
+
+@pytest.mark.parametrize("name,A,B", PAIRS, ids=[p[0] for p in PAIRS])
+def test_spgemm_matches_oracle(tsg, name, A, B):
+    TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
+    C = tsg.spgemm(TA, TB, stats=True, products=True)
+    ref = oracle.expected_tiles(A, B)
+    ref_fma = oracle.expected_tiles(A, B, fma=True)
+    got = host(C)
+    assert_tiles_equal(got, ref, values=None)
+    absref = oracle.csr_to_tiles(_abs_csr(A, B)).val
+    assert_values_close(got["val"], ref.val, absref)
+    assert bitwise_equal_values(got["val"], ref_fma.val), "ascending-k FMA order must match the oracle bitwise"
+    d = oracle.diagnostics(A, B)
+    st = C.stats
+    assert st["tiles_c"] == d["tiles_c"] == C.num_tiles
+    assert st["nnz_c"] == d["nnz_c"]
+    assert st["pairs"] == d["pairs"]
+    assert st["products"] == d["products"]
+    assert st["tiles_dense"] == int((np.diff(ref.tile_nnz) >= 192).sum())
+    # CSR assembly of the result
+    rp, ci, v = tsg.tiles_to_csr(C)
+    O = oracle.spgemm(A, B, fma=True)
+    assert np.array_equal(rp.cpu().numpy(), O.rowptr) and np.array_equal(ci.cpu().numpy(), O.col)
+    assert bitwise_equal_values(v.cpu().numpy(), O.val)
+
+
+def _abs_csr(A, B):
+    O = oracle.spgemm(A, B)
+    return gen.CSR(O.m, O.n, O.rowptr, O.col, O.abs)
+
+
+@pytest.mark.parametrize("opts", [dict(scan_only=True), dict(list_always=True), dict(dense_threshold=1),
+                                  dict(dense_threshold=257), dict(dense_threshold=100)])
+def test_modes_give_identical_results(tsg, opts):
+    """Step-1 modes and the accumulator threshold change the work split, never the result."""
+    for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1")):
+        T = tiles_of(tsg, A)
+        base = host(tsg.spgemm(T, T))
+        alt = host(tsg.spgemm(T, T, **opts))
+        for k in ARRAYS[:-1]:
+            assert np.array_equal(base[k], alt[k]), (opts, k)
+        assert bitwise_equal_values(base["val"], alt["val"])
+
+
+def test_threshold_boundary_tiles(tsg):
+    """C tiles with nnz 191, 192, 193 straddle t_nnz = 192."""
+    rng = np.random.default_rng(0)
+    for target in (191, 192, 193):
+        # C = I16 * B where B is one 16x16 tile with `target` nonzeros -> C tile nnz = target
+        cells = rng.choice(256, target, replace=False)
+        B = gen.from_coo(16, 16, cells // 16, cells % 16, rng.uniform(-1, 1, target))
+        I = gen.identity(16, 1.5)
+        C = tsg.spgemm(tiles_of(tsg, I), tiles_of(tsg, B), stats=True)
+        assert C.stats["tiles_dense"] == (1 if target >= 192 else 0)
+        ref = oracle.expected_tiles(I, B, fma=True)
+        assert_tiles_equal(host(C), ref)
+
+
+def test_nonfinite_and_cancellation(tsg):
+    # dense tiles with an Inf and a NaN inside: the dense path must not turn Inf*0 into NaN
+    A = gen.dense_block(16, 16)
+    A.val[5] = np.inf
+    A.val[40] = np.nan
+    B = gen.random_sparse(16, 16, 0.5, 3)
+    for a, b in ((A, B), (B, A), (A, A)):
+        for th in (1, 257):
+            C = tsg.spgemm(tiles_of(tsg, a), tiles_of(tsg, b), dense_threshold=th)
+            ref = oracle.expected_tiles(a, b, fma=True)
+            assert_tiles_equal(host(C), ref)
+    # exact cancellation keeps the structural entry (reading A11)
+    X = gen.from_coo(16, 16, [0, 0], [0, 1], [1.0, 1.0])
+    Y = gen.from_coo(16, 16, [0, 1], [0, 0], [1.0, -1.0])
+    C = tsg.spgemm(tiles_of(tsg, X), tiles_of(tsg, Y))
+    assert C.nnz == 1 and host(C)["val"][0] == 0.0
+
+
+def test_determinism_and_symmetry(tsg):
+    R = gen.random_sparse(400, 400, 0.01, 4)
+    S = (R.to_scipy() + R.to_scipy().T).tocsr()
+    S.sort_indices()
+    A = gen.CSR(400, 400, S.indptr.astype(np.int64), S.indices.astype(np.int32), S.data.astype(np.float64))
+    T = tiles_of(tsg, A)
+    c1, c2 = host(tsg.spgemm(T, T)), host(tsg.spgemm(T, T))
+    for k in ARRAYS:
+        assert np.array_equal(c1[k], c2[k])
+    rp, ci, v = tsg.tiles_to_csr(tsg.spgemm(T, T))
+    D = csr_dense(400, 400, rp.cpu().numpy(), ci.cpu().numpy(), v.cpu().numpy())
+    assert bitwise_equal_values(D, D.T)
+
+
+def test_chained_output_as_input(tsg):
+    """A^3 = (A^2) A with the exported C tiles fed straight back."""
+    A = gen.stencil27(8)
+    T = tiles_of(tsg, A)
+    C2 = tsg.spgemm(T, T)
+    C3 = tsg.spgemm(C2, T)
+    A2 = oracle.spgemm(A, A, fma=True)
+    A2c = gen.CSR(A2.m, A2.n, A2.rowptr, A2.col, A2.val)
+    ref = oracle.expected_tiles(A2c, A, fma=True)
+    assert_tiles_equal(host(C3), ref)
+
+
+def test_slice_rows_and_wrap(tsg):
+    A = gen.rmat(11)
+    T = tiles_of(tsg, A)
+    full = oracle.spgemm(A, A, fma=True)
+    b, e = 17, 60
+    V = tsg.slice_rows(T, b, e)
+    CV = tsg.spgemm(V, T)
+    rows = np.arange(16 * b, 16 * e)
+    sub = oracle.spgemm(A, A, fma=True, rows=rows)
+    ref = oracle.csr_to_tiles(gen.CSR(len(rows), A.n, sub.rowptr, sub.col, sub.val))
+    assert_tiles_equal(host(CV), ref)
+    W = tsg.wrap(A.m, A.n, T.arrays(), keepalive=T)
+    CW = tsg.spgemm(W, W)
+    assert_tiles_equal(host(CW), oracle.csr_to_tiles(gen.CSR(full.m, full.n, full.rowptr, full.col, full.val)))
+
+
+def test_launch_counter_advances(tsg):
+    A = gen.config("C1")
+    T = tiles_of(tsg, A)
+    n0 = tsg.kernel_launch_count()
+    C = tsg.spgemm(T, T, stats=True)
+    assert tsg.kernel_launch_count() - n0 == C.stats["kernel_launches"] > 5
+    assert C.stats["host_syncs"] == 3
+
+
+# ------------------------------------------------------------------------------------------
+# full-size configurations, in the launch configuration bench.py times
+# ------------------------------------------------------------------------------------------
+CLOSED = {  # SURVEY §8(c) closed forms (structure and counts are value independent)
+    "C2": dict(nnz_c=254_840_104, products=1_489_355_288),
+    "C3": dict(nnz_c=28_850_976, products=562_529_664),
+}
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
+def test_full_size_sampled_rows(tsg, cfg):
+    import torch
+
+    A = gen.config(cfg)
+    T = tiles_of(tsg, A)
+    C = tsg.spgemm(T, T, stats=True, products=True)
+    st = C.stats
+    if cfg in CLOSED:
+        assert st["nnz_c"] == CLOSED[cfg]["nnz_c"] and st["products"] == CLOSED[cfg]["products"]
+    else:
+        assert st["products"] == oracle.products(A, A)
+    # properties at any size: sum of popcounts == nnz, row offsets consistent, tiles non-empty
+    mask = C.mask.view(torch.int16).to(torch.int32) & 0xFFFF
+    pop = torch.zeros_like(mask)
+    for b in range(16):
+        pop += (mask >> b) & 1
+    assert int(pop.sum()) == C.nnz
+    pop2 = pop.view(-1, 16)
+    rp = C.row_ptr.view(-1, 16).to(torch.int32)
+    assert torch.equal(rp, torch.cumsum(pop2, 1) - pop2)
+    assert bool((C.tile_nnz[1:] > C.tile_nnz[:-1]).all())
+    # sampled rows against the oracle, one by one
+    rng = np.random.default_rng(11)
+    rows = np.unique(np.concatenate([[0, A.m - 1], rng.integers(0, A.m, 300)]))
+    sub = oracle.spgemm(A, A, fma=True, rows=rows)
+    crp, cci, cv = tsg.tiles_to_csr(C)
+    crp_h = crp.cpu().numpy()
+    for t, i in enumerate(rows):
+        b, e = int(crp_h[i]), int(crp_h[i + 1])
+        s0, s1 = int(sub.rowptr[t]), int(sub.rowptr[t + 1])
+        assert np.array_equal(cci[b:e].cpu().numpy(), sub.col[s0:s1]), i
+        assert bitwise_equal_values(cv[b:e].cpu().numpy(), sub.val[s0:s1]), i
