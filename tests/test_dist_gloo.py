@@ -1,0 +1,111 @@
+"""Multi-rank host logic of the sharded path, on CPU with the gloo backend (world_size 2).
+
+The local per-rank compute is the oracle here (a test-injected stand-in for the GPU kernels);
+what is under test is paper_conf_ppopp_niuljs0022_b200.dist: the product-balanced tile-row
+partition, the broadcast of B's arrays, the uneven all-gather and the offset rebasing.
+"""
+from __future__ import annotations
+
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_partition_balances_products():
+    from workloads import gen
+
+    for A in (gen.rmat(11), gen.config("C1"), gen.strip_fem(4, 40, 6)):
+        w = tdist.tile_row_products(A, A)
+        import oracle
+
+        assert w.sum() == oracle.products(A, A)
+        for world in (1, 2, 3, 4, 8):
+            cuts = tdist.partition_tile_rows(A, A, world)
+            assert cuts[0] == 0 and cuts[-1] == w.size and np.all(np.diff(cuts) >= 0) and len(cuts) == world + 1
+            loads = [w[cuts[g]:cuts[g + 1]].sum() for g in range(world)]
+            # no shard exceeds its fair share by more than one tile row's weight
+            assert max(loads) <= w.sum() / world + w.max()
+
+
+def test_partition_more_ranks_than_rows():
+    from workloads import gen
+
+    A = gen.random_sparse(20, 20, 0.3, 1)  # 2 tile rows
+    cuts = tdist.partition_tile_rows(A, A, 8)
+    assert cuts[0] == 0 and cuts[-1] == 2 and len(cuts) == 9 and np.all(np.diff(cuts) >= 0)
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _to_torch(T):
+    return {"tile_ptr": torch.from_numpy(T.tile_ptr), "tile_col": torch.from_numpy(T.tile_col),
+            "tile_nnz": torch.from_numpy(T.tile_nnz), "row_ptr": torch.from_numpy(T.row_ptr),
+            "mask": torch.from_numpy(T.mask.view(np.int16)).view(torch.uint16), "idx": torch.from_numpy(T.idx),
+            "val": torch.from_numpy(T.val)}
+
+
+def _worker(rank, world, port, result_path):
+    import sys
+
+    sys.path.insert(0, ROOT)
+    import oracle
+    from workloads import gen
+
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        A = gen.rmat(10)
+        # 1) broadcast B's tile arrays from rank 0
+        TB = oracle.csr_to_tiles(A)
+        meta = (A.m, A.n, TB.num_tiles, TB.nnz) if rank == 0 else None
+        arrs = _to_torch(TB) if rank == 0 else None
+        meta_r, got = tdist.broadcast_tiles(arrs, meta, 0, torch.device("cpu"))
+        ref = _to_torch(TB)
+        ok_b = meta_r == (A.m, A.n, TB.num_tiles, TB.nnz) and all(
+            torch.equal(got[k].view(torch.int16) if k == "mask" else got[k],
+                        ref[k].view(torch.int16) if k == "mask" else ref[k]) for k in tdist.ARRAYS)
+        # 2) local shard of C tile rows (oracle stands in for the GPU kernels)
+        cuts = tdist.partition_tile_rows(A, A, world)
+        I0, I1 = int(cuts[rank]), int(cuts[rank + 1])
+        rows = np.arange(16 * I0, min(16 * I1, A.m), dtype=np.int64)
+        sub = oracle.spgemm(A, A, fma=True, rows=rows)
+        Cl = oracle.csr_to_tiles(gen.CSR(len(rows), A.n, sub.rowptr, sub.col, sub.val))
+        piece = dict(m=len(rows), n=A.n, **_to_torch(Cl))
+        # 3) uneven all-gather + rebasing
+        m, n, full = tdist.allgatherv_tiles(piece)
+        exp = oracle.expected_tiles(A, A, fma=True)
+        ok_c = (m, n) == (A.m, A.n)
+        for k in tdist.ARRAYS:
+            a = full[k].view(torch.int16).numpy().view(np.uint16) if k == "mask" else full[k].numpy()
+            ok_c &= bool(np.array_equal(a, getattr(exp, k)))
+        with open(f"{result_path}.{rank}", "w") as f:
+            f.write(f"{int(ok_b)} {int(ok_c)} {I0} {I1}")
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_broadcast_and_allgatherv_world2(tmp_path):
+    world = 2
+    port = _free_port()
+    mp.spawn(_worker, args=(world, port, str(tmp_path / "res")), nprocs=world, join=True)
+    spans = []
+    for r in range(world):
+        ok_b, ok_c, i0, i1 = open(tmp_path / f"res.{r}").read().split()
+        assert ok_b == "1", f"broadcast mismatch on rank {r}"
+        assert ok_c == "1", f"assembled C mismatch on rank {r}"
+        spans.append((int(i0), int(i1)))
+    assert spans[0][0] == 0 and spans[0][1] == spans[1][0]

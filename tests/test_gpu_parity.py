@@ -278,15 +278,22 @@ def test_full_size_sampled_rows(tsg, cfg):
         assert st["nnz_c"] == CLOSED[cfg]["nnz_c"] and st["products"] == CLOSED[cfg]["products"]
     else:
         assert st["products"] == oracle.products(A, A)
-    # properties at any size: sum of popcounts == nnz, row offsets consistent, tiles non-empty
-    mask = C.mask.view(torch.int16).to(torch.int32) & 0xFFFF
-    pop = torch.zeros_like(mask)
-    for b in range(16):
-        pop += (mask >> b) & 1
-    assert int(pop.sum()) == C.nnz
-    pop2 = pop.view(-1, 16)
-    rp = C.row_ptr.view(-1, 16).to(torch.int32)
-    assert torch.equal(rp, torch.cumsum(pop2, 1) - pop2)
+    # properties at any size (chunked to bound memory): sum of popcounts == nnz, row offsets
+    # consistent with the masks, every tile non-empty
+    total = 0
+    CH = 1 << 24
+    for t0 in range(0, C.num_tiles, CH):
+        t1 = min(C.num_tiles, t0 + CH)
+        mask = C.mask[16 * t0:16 * t1].view(torch.int16).to(torch.int32) & 0xFFFF
+        pop = torch.zeros_like(mask)
+        for b in range(16):
+            pop += (mask >> b) & 1
+        total += int(pop.sum())
+        pop2 = pop.view(-1, 16)
+        rp = C.row_ptr[16 * t0:16 * t1].view(-1, 16).to(torch.int32)
+        assert torch.equal(rp, torch.cumsum(pop2, 1) - pop2)
+        del mask, pop, pop2, rp
+    assert total == C.nnz
     assert bool((C.tile_nnz[1:] > C.tile_nnz[:-1]).all())
     # sampled rows against the oracle, one by one
     rng = np.random.default_rng(11)
