@@ -227,7 +227,7 @@ def main():
     if dist:
         dist.barrier()
     launches0 = tsg.kernel_launch_count()
-    step_ms, s3_ms, s2_ms, s1_ms = [], [], [], []
+    step_ms, s3_ms, s2_ms, s1_ms, sa_ms, host_ms = [], [], [], [], [], []
     stats_last = None
     with ClockSampler(local) if not args.profile else _Null() as clk:
         torch.cuda.synchronize()
@@ -246,6 +246,8 @@ def main():
             s1_ms.append(st["ms_step1"] + st["ms_index"])
             s2_ms.append(st["ms_step2"])
             s3_ms.append(st["ms_step3"])
+            sa_ms.append(st["ms_alloc"])
+            host_ms.append((st["ms_host_sync"], st["ms_host_alloc"]))
             stats_last = st
             del C
         torch.cuda.synchronize()
@@ -269,6 +271,7 @@ def main():
     bw, bw_src = peaks()
     nnzC, ntC = stats_last["nnz_c"], stats_last["tiles_c"]
     steps_ms = {"step1": float(np.mean(s1_ms)), "step2": float(np.mean(s2_ms)), "step3": float(np.mean(s3_ms))}
+    alloc_ms = float(np.mean(sa_ms))
     alg = {  # algorithmic bytes per launch of each step's kernels
         "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + 6 * T.num_tiles + 8 * (T.tile_m + 1) + 12 * ntC,
         "step2": 32 * (Ashard.num_tiles + T.num_tiles) + 60 * ntC,
@@ -338,7 +341,10 @@ def main():
                    "parallelism": f"tile-row shards x{world}" if world > 1 else "single GPU",
                    "l2": ("512 MB flush between timed steps" if flush is not None else
                           f"inputs larger than L2 (A tiles {tile_bytes(T.tile_m, T.num_tiles, T.nnz) / 1e6:.0f} MB > 126 MB)"),
-                   "step_ms": {k: round(v, 4) for k, v in steps_ms.items()},
+                   "step_ms": {k: round(v, 4) for k, v in steps_ms.items()}, "alloc_sync_ms": round(alloc_ms, 4),
+                   "step_ms_all": [round(x, 3) for x in step_ms],
+                   "host_sync_alloc_ms": [round(float(np.mean([h[0] for h in host_ms])), 3),
+                                          round(float(np.mean([h[1] for h in host_ms])), 3)],
                    "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw},
         "roofline": roof,
         "cpu_baseline": cpu,

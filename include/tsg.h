@@ -102,6 +102,7 @@ typedef struct {
     int32_t step1_list_tiles; /* A tiles that used the B-row-list expansion (mode ii) */
     int32_t host_syncs;       /* blocking device->host scalar reads performed */
     float ms_index, ms_step1, ms_step2, ms_alloc, ms_step3, ms_total; /* CUDA-event times */
+    float ms_host_sync, ms_host_alloc; /* host wall time blocked in scalar reads / allocation calls */
 } tsg_stats;
 
 /* flags for tsg_csr_to_tiles */

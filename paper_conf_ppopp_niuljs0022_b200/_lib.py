@@ -49,7 +49,8 @@ class Stats(C.Structure):
                 ("tiles_dense", C.c_int64), ("tiles_sparse", C.c_int64), ("kernel_launches", C.c_int64),
                 ("step1_list_tiles", C.c_int32), ("host_syncs", C.c_int32),
                 ("ms_index", C.c_float), ("ms_step1", C.c_float), ("ms_step2", C.c_float),
-                ("ms_alloc", C.c_float), ("ms_step3", C.c_float), ("ms_total", C.c_float)]
+                ("ms_alloc", C.c_float), ("ms_step3", C.c_float), ("ms_total", C.c_float),
+                ("ms_host_sync", C.c_float), ("ms_host_alloc", C.c_float)]
 
     def as_dict(self) -> dict:
         return {f[0]: getattr(self, f[0]) for f in self._fields_}

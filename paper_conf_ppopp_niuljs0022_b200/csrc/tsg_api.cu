@@ -1,6 +1,7 @@
 // tsg_api.cu -- the extern "C" boundary of libtsg (include/tsg.h): argument validation, handle
 // lifetime, allocation policy, error translation.  Every compute step lives in the kernels of
 // tsg_convert.cu / tsg_spgemm.cu; this file launches nothing but two tiny rebase kernels.
+#include <chrono>
 #include <cstring>
 
 #include "tsg_internal.cuh"
@@ -8,12 +9,20 @@
 namespace tsg {
 
 std::atomic<int64_t> g_launches{0};
+thread_local double t_host_alloc_ms = 0.0, t_host_sync_ms = 0.0;
+double now_ms() {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 static thread_local std::string t_last_error;
 static thread_local int64_t t_call_launches = 0;
 
 void set_last_error(const std::string &msg) { t_last_error = msg; }
 void note_launch() { t_call_launches++; }
-void reset_call_launches() { t_call_launches = 0; }
+void reset_call_launches() {
+    t_call_launches = 0;
+    t_host_alloc_ms = 0.0;
+    t_host_sync_ms = 0.0;
+}
 int64_t call_launches() { return t_call_launches; }
 
 static void ensure_pool_cached() {
@@ -53,7 +62,9 @@ void Allocator::free(void *p, size_t bytes, cudaStream_t s) const {
 int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {
     int64_t v = 0;
     TSG_CUDA(cudaMemcpyAsync(&v, dptr, sizeof(v), cudaMemcpyDeviceToHost, s));
+    const double t0 = now_ms();
     TSG_CUDA(cudaStreamSynchronize(s));
+    t_host_sync_ms += now_ms() - t0;
     return v;
 }
 

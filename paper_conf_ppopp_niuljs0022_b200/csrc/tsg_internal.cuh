@@ -56,6 +56,10 @@ extern std::atomic<int64_t> g_launches;
 
 void note_launch();  // per-call counter (thread-local)
 
+// host-time accounting of one call (thread-local): blocked in scalar reads / allocation calls
+extern thread_local double t_host_alloc_ms, t_host_sync_ms;
+double now_ms();
+
 // ------------------------------------------------------------------------------------------
 // allocation: either the user's stream-ordered hook or cudaMallocAsync on the default pool
 // ------------------------------------------------------------------------------------------
@@ -83,7 +87,9 @@ class Buffers {
     T *get(int64_t count) {
         size_t bytes = sizeof(T) * (size_t)(count > 0 ? count : 0);
         if (bytes < 256) bytes = 256;  // never hand out NULL; keep 256-byte alignment
+        const double t0 = now_ms();
         void *p = al_.alloc(bytes, s_);
+        t_host_alloc_ms += now_ms() - t0;
         if (!p) fail(TSG_ERR_OOM, "device allocation of " + std::to_string(bytes) + " bytes failed");
         items_.push_back({p, bytes});
         return static_cast<T *>(p);
@@ -150,7 +156,7 @@ void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buff
 // read one int64 from device memory (blocking on stream s)
 int64_t read_scalar(const int64_t *dptr, cudaStream_t s);
 
-// per-call launch counter access (thread-local)
+// per-call launch counter (thread-local)
 void reset_call_launches();
 int64_t call_launches();
 

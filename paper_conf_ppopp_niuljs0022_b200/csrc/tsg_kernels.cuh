@@ -1,0 +1,127 @@
+// tsg_kernels.cuh -- parameter blocks and host launchers shared by the step translation units
+// (tsg_step1.cu: a0/a1, tsg_step23.cu: a2/a4) and the orchestration in tsg_spgemm.cu.
+#pragma once
+
+#include "tsg_internal.cuh"
+
+namespace tsg {
+
+typedef unsigned long long u64c;
+
+// device-side counters of one tsg_spgemm call (zeroed at the start)
+struct DevCounters {
+    u64c max_u_small;  // largest candidate count among shared-memory rows
+    u64c nbig;         // rows sorted in global memory
+    u64c big_u;        // their total candidate count
+    u64c list_tiles;   // A tiles expanded through B row lists
+    u64c pairs;        // contributing pairs
+    u64c products;     // intermediate products (stats only)
+    u64c n2light;      // step-2 class sizes
+    u64c n2heavy;
+    u64c n3small;      // step-3 class sizes
+    u64c n3medium;
+    u64c n3dense;
+    u64c pad;
+};
+
+constexpr int ROW_T = 256;        // threads of a step-1 row CTA
+constexpr int ROW_NW = ROW_T / 32;
+constexpr int ROW_CAP = 4096;     // max candidates of a row sorted in shared memory
+constexpr int LIGHT_WORK = 16;    // step-2 thread-per-tile class: (pair, c) items of the tile
+constexpr int SMALL_NNZ = 16;     // step-3 thread-per-tile class: C tile nnz
+
+// ---------------- a1 row sort
+struct S1Params {
+    const int64_t *tpA;
+    const int64_t *tnzA;      // A tile_nnz (for the per-C-tile work estimate)
+    const uint16_t *colOccA;
+    const int64_t *costOff;
+    const int64_t *startA;
+    const int32_t *tcB;
+    const uint16_t *rowOccB;
+    const uint32_t *list;
+    const int32_t *rowJlo;
+    const int32_t *rowJhi;
+    const uint8_t *rowClass;
+    uint64_t *pairs;   // [Utot]  (posA << 32) | posB, at costOff[a0] + i
+    int32_t *tJ;       // [Utot]  C tile column of rank r, at costOff[a0] + r
+    uint32_t *tStart;  // [Utot]  first pair (row-relative)
+    uint32_t *tCnt;    // [Utot]  pair count
+    uint32_t *tWork;   // [Utot]  (pair, c) items: sum over pairs of popc(colOcc(A) & rowOcc(B))
+    int64_t *nC;       // [tm]    C tiles of the row
+    const int32_t *bigList;
+    const int64_t *bigOff;
+    uint64_t *bigKeysA, *bigKeysB;
+    uint32_t *bigPosB, *bigKpos;
+    DevCounters *cnt;
+};
+
+// ---------------- compaction of step-1 results into per-C-tile arrays + step-2 classes
+struct CompactParams {
+    int64_t tm;
+    const int64_t *tpA;
+    const int64_t *costOff;
+    const int64_t *tilePtrC;
+    const int32_t *tJ;
+    const uint32_t *tStart;
+    const uint32_t *tCnt;
+    const uint32_t *tWork;
+    int32_t *tile_col;
+    int64_t *pairBeg;
+    uint32_t *pairCnt;
+    uint32_t *work;   // (pair, c) items per C tile: the step-2 class split
+};
+
+// ---------------- a2 step 2 and a4 step 3: warps take groups of 32 consecutive C tiles
+struct StepParams {
+    int64_t ntC;
+    const int64_t *pairBeg;
+    const uint32_t *pairCnt;
+    const uint64_t *pairs;
+    // A
+    const int64_t *tnzA;
+    const uint8_t *rpA;
+    const uint16_t *mA;
+    const uint16_t *mTA;      // transposed masks
+    const uint16_t *colOccA;
+    const uint8_t *ixA;
+    const double *vA;
+    // B
+    const int64_t *tnzB;
+    const uint8_t *rpB;
+    const uint16_t *mB;
+    const uint16_t *rowOccB;
+    const uint8_t *ixB;
+    const double *vB;
+    // C
+    int64_t *tnzC;   // step 2: per-tile nnz; step 3: offsets
+    uint8_t *rpC;
+    uint16_t *mC;
+    uint8_t *ixC;
+    double *vC;
+    const uint32_t *work;  // step-2 class split
+    int dense_threshold;
+    DevCounters *cnt;
+};
+
+// launchers (tsg_step1.cu)
+void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s);
+void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
+                    uint32_t *list, cudaStream_t s);
+void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int64_t ntA, const int32_t *tcA,
+                     const uint16_t *maskA, int32_t *rnnz, DevCounters *cnt, cudaStream_t s);
+void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA, const int64_t *tpB,
+                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, bool scan_only, int64_t *cost,
+                       int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s);
+void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
+                     const int32_t *jhiA, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass, int64_t *nC,
+                     int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s);
+void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, cudaStream_t s);
+void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s);
+void launch_compact(const CompactParams &P, cudaStream_t s);
+
+// launchers (tsg_step23.cu)
+void launch_step2(const StepParams &P, cudaStream_t s);
+void launch_step3(const StepParams &P, cudaStream_t s);
+
+}  // namespace tsg

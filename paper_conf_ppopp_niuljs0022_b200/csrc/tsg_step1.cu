@@ -1,0 +1,480 @@
+// tsg_step1.cu -- SURVEY §8(a) rows a0 (helper indices) and a1 (step 1 of Section 3.3).
+//
+// Step 1 of the paper computes the tile layout of C by a structural SpGEMM C' = A'B'
+// and step 2 then intersects tile index sets per C tile (Alg 2 l.4-18).  Here both
+// come out of one exact per-tile-row pass: each A tile enumerates its candidate B
+// tiles (whole B tile row, or the B row list of its single column), a CTA per tile row sorts the
+// row's candidates by tile column J (stable, so pairs stay in ascending K), and the heads of
+// equal-J runs are the non-empty C tiles.  Pairs without products (colOcc(A)&rowOcc(B) == 0) are
+// dropped (reading B3), so C never stores an empty tile (reading A6).
+#include "tsg_kernels.cuh"
+
+namespace tsg {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+enum RowClass : uint8_t { ROW_EMPTY = 0, ROW_SMALL = 1, ROW_BIG = 2 };
+
+__device__ __forceinline__ int bits_for(uint64_t v) {  // bits needed to represent v (>= 1)
+    return v ? 64 - __clzll((long long)v) : 1;
+}
+
+// ------------------------------------------------------------------------------------------
+// a0: occupancy words.  rowOcc bit r = row r non-empty; colOcc = OR of the 16 row masks.
+// A pair (A_IK, B_KJ) has a product iff colOcc(A_IK) & rowOcc(B_KJ) != 0.
+// ------------------------------------------------------------------------------------------
+__global__ void k_occupancy(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ row_occ,
+                            uint16_t *__restrict__ col_occ) {
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= nt) return;
+    const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
+    uint4 a = __ldg(p), b = __ldg(p + 1);
+    uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    uint32_t ro = 0, co = 0;
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+        uint32_t lo = w[k] & 0xffffu, hi = w[k] >> 16;
+        ro |= (lo ? 1u : 0u) << (2 * k);
+        ro |= (hi ? 1u : 0u) << (2 * k + 1);
+        co |= lo | hi;
+    }
+    if (row_occ) row_occ[t] = (uint16_t)ro;
+    if (col_occ) col_occ[t] = (uint16_t)co;
+}
+
+// B row lists ("mode ii"): for each global row k of B, the B tiles of tile row k/16 whose row
+// k%16 is non-empty, ascending tile column.  One warp = two B tile rows, lane r = row r.
+__global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__restrict__ tpB,
+                                                 const uint16_t *__restrict__ maskB, const int64_t *__restrict__ lptr,
+                                                 int32_t *__restrict__ lcnt, uint32_t *__restrict__ list) {
+    const int lane = threadIdx.x & 31, r = lane & 15;
+    const int64_t K = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
+    if (K >= tmB) return;
+    const int64_t t0 = tpB[K], t1 = tpB[K + 1];
+    if (!list) {
+        int c = 0;
+        for (int64_t t = t0; t < t1; t++) c += maskB[t * TILE + r] != 0;
+        lcnt[K * TILE + r] = c;
+    } else {
+        int64_t pos = lptr[K * TILE + r];
+        for (int64_t t = t0; t < t1; t++)
+            if (maskB[t * TILE + r]) list[pos++] = (uint32_t)t;
+    }
+}
+
+// stats only: nnz of every global row of B, then products per A tile
+__global__ void __launch_bounds__(256) k_brow_nnz(int64_t tmB, const int64_t *__restrict__ tpB,
+                                                  const uint16_t *__restrict__ maskB, int32_t *__restrict__ rnnz) {
+    const int lane = threadIdx.x & 31, r = lane & 15;
+    const int64_t K = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
+    if (K >= tmB) return;
+    int c = 0;
+    for (int64_t t = tpB[K]; t < tpB[K + 1]; t++) c += __popc(maskB[t * TILE + r]);
+    rnnz[K * TILE + r] = c;
+}
+
+__global__ void k_products(int64_t ntA, const int32_t *__restrict__ tcA, const uint16_t *__restrict__ maskA,
+                           const int32_t *__restrict__ rnnz, DevCounters *cnt) {
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    u64c p = 0;
+    if (t < ntA) {
+        int64_t K = tcA[t];
+        for (int r = 0; r < TILE; r++) {
+            uint32_t m = maskA[t * TILE + r];
+            while (m) {
+                int c = __ffs(m) - 1;
+                m &= m - 1;
+                p += rnnz[K * TILE + c];
+            }
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(FULL, p, o);
+    if ((threadIdx.x & 31) == 0 && p) atomicAdd(&cnt->products, p);
+}
+
+// ------------------------------------------------------------------------------------------
+// a1 (plan): per A tile, how its candidate B tiles are enumerated.
+//   scan mode: every tile of B tile row K (filtered later by occupancy);
+//   list mode: when A_IK touches a single column c, exactly the B row list of k = 16K + c
+//              (all of them contribute, no filter, no duplicates).
+// cost = number of candidates; start encodes the mode (list: -(start+1)).
+// ------------------------------------------------------------------------------------------
+__global__ void k_atile_plan(int64_t ntA, const int32_t *__restrict__ tcA, const uint16_t *__restrict__ colOccA,
+                             const int64_t *__restrict__ tpB, const int32_t *__restrict__ tcB,
+                             const int64_t *__restrict__ lptr, const uint32_t *__restrict__ list, bool scan_only,
+                             int64_t *__restrict__ cost, int64_t *__restrict__ start, int32_t *__restrict__ jlo,
+                             int32_t *__restrict__ jhi, DevCounters *cnt) {
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    bool is_list = false;
+    if (t < ntA) {
+        const int64_t K = tcA[t];
+        const uint32_t co = colOccA[t];
+        int64_t b0 = tpB[K], len = tpB[K + 1] - b0, st = b0;
+        if (!scan_only && lptr && __popc(co) == 1) {
+            int64_t k = K * TILE + (__ffs(co) - 1);
+            int64_t l0 = lptr[k], ll = lptr[k + 1] - l0;
+            if (ll < len) {
+                is_list = true;
+                len = ll;
+                st = l0;
+            }
+        }
+        cost[t] = len;
+        start[t] = is_list ? -(st + 1) : st;
+        if (len > 0) {
+            int64_t f = is_list ? (int64_t)list[st] : st, l = is_list ? (int64_t)list[st + len - 1] : st + len - 1;
+            jlo[t] = tcB[f];
+            jhi[t] = tcB[l];
+        } else {
+            jlo[t] = 0x7fffffff;
+            jhi[t] = -1;
+        }
+    }
+    unsigned b = __ballot_sync(FULL, is_list);
+    if ((threadIdx.x & 31) == 0 && b) atomicAdd(&cnt->list_tiles, (u64c)__popc(b));
+}
+
+// a1 (row plan): candidate window and class of every tile row (one warp per row)
+__global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const int64_t *__restrict__ costOff,
+                           const int32_t *__restrict__ jloA, const int32_t *__restrict__ jhiA,
+                           int32_t *__restrict__ rowJlo, int32_t *__restrict__ rowJhi, uint8_t *__restrict__ rowClass,
+                           int64_t *__restrict__ nC, int32_t *__restrict__ bigList, int64_t *__restrict__ bigOff,
+                           DevCounters *cnt) {
+    const int lane = threadIdx.x & 31;
+    const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (I >= tmA) return;
+    const int64_t a0 = tpA[I], a1 = tpA[I + 1];
+    int lo = 0x7fffffff, hi = -1;
+    for (int64_t t = a0 + lane; t < a1; t += 32) {
+        lo = min(lo, jloA[t]);
+        hi = max(hi, jhiA[t]);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        lo = min(lo, __shfl_xor_sync(FULL, lo, o));
+        hi = max(hi, __shfl_xor_sync(FULL, hi, o));
+    }
+    if (lane) return;
+    const int64_t U = costOff[a1] - costOff[a0];
+    rowJlo[I] = lo;
+    rowJhi[I] = hi;
+    if (U == 0 || hi < lo) {
+        rowClass[I] = ROW_EMPTY;
+        nC[I] = 0;
+        return;
+    }
+    const int wb = bits_for((uint64_t)(hi - lo + 1));  // valid 0..hi-lo, sentinel hi-lo+1
+    const int ub = bits_for((uint64_t)(U > 1 ? U - 1 : 1));
+    if (U <= ROW_CAP && wb + ub <= 32 && (a1 - a0) < 65536) {
+        rowClass[I] = ROW_SMALL;
+        atomicMax(&cnt->max_u_small, (u64c)U);
+    } else {
+        rowClass[I] = ROW_BIG;
+        u64c k = atomicAdd(&cnt->nbig, 1ULL);
+        bigList[k] = (int32_t)I;
+        bigOff[I] = (int64_t)atomicAdd(&cnt->big_u, (u64c)U);
+    }
+}
+
+__device__ __forceinline__ int block_scan_int(int v, int *total, int *sm /* ROW_NW+1 ints */) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int incl = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        int o = __shfl_up_sync(FULL, incl, d);
+        if (lane >= d) incl += o;
+    }
+    if (lane == 31) sm[w] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int s = 0;
+        for (int k = 0; k < ROW_NW; k++) {
+            int x = sm[k];
+            sm[k] = s;
+            s += x;
+        }
+        sm[ROW_NW] = s;
+    }
+    __syncthreads();
+    int res = sm[w] + incl - v;
+    *total = sm[ROW_NW];
+    __syncthreads();
+    return res;
+}
+
+// in-place exclusive scan of hist[0..L) (L <= 256*ROW_NW) by the CTA
+__device__ void block_scan_array(uint32_t *hist, int L, int *sm) {
+    const int per = (L + ROW_T - 1) / ROW_T;
+    const int b = threadIdx.x * per, e = min(L, b + per);
+    int s = 0;
+    for (int i = b; i < e; i++) s += hist[i];
+    int tot;
+    int pre = block_scan_int(s, &tot, sm);
+    for (int i = b; i < e; i++) {
+        int x = hist[i];
+        hist[i] = pre;
+        pre += x;
+    }
+    __syncthreads();
+}
+
+// stable LSD radix sort of a[0..n) on bits [lo, lo+nbits); returns the buffer holding the result
+template <typename K>
+__device__ K *block_radix_sort(K *a, K *b, int64_t n, int lo, int nbits, uint32_t *hist, int *sm) {
+    if (nbits <= 0 || n <= 1) return a;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int passes = (nbits + 7) / 8;
+    const int dbits = (nbits + passes - 1) / passes;
+    const int64_t per = (((n + ROW_NW - 1) / ROW_NW) + 31) & ~(int64_t)31;
+    const int64_t w0 = min(n, (int64_t)w * per), w1 = min(n, w0 + per);
+    const unsigned lt = (1u << lane) - 1u;
+    for (int p = 0; p < passes; p++) {
+        const int shift = lo + p * dbits;
+        const int bits = min(dbits, nbits - p * dbits);
+        const uint32_t B = 1u << bits, dm = B - 1u;
+        for (uint32_t i = threadIdx.x; i < B * ROW_NW; i += ROW_T) hist[i] = 0;
+        __syncthreads();
+        for (int64_t base = w0; base < w1; base += 32) {
+            const int64_t i = base + lane;
+            const bool v = i < w1;
+            const uint32_t d = v ? (uint32_t)((a[i] >> shift) & dm) : B;
+            const unsigned peers = __match_any_sync(FULL, d);
+            if (v && lane == __ffs(peers) - 1) hist[d * ROW_NW + w] += __popc(peers);
+            __syncwarp();
+        }
+        __syncthreads();
+        block_scan_array(hist, (int)(B * ROW_NW), sm);
+        for (int64_t base = w0; base < w1; base += 32) {
+            const int64_t i = base + lane;
+            const bool v = i < w1;
+            K key = v ? a[i] : (K)0;
+            const uint32_t d = v ? (uint32_t)((key >> shift) & dm) : B;
+            const unsigned peers = __match_any_sync(FULL, d);
+            if (v) b[hist[d * ROW_NW + w] + __popc(peers & lt)] = key;
+            __syncwarp();
+            if (v && lane == __ffs(peers) - 1) hist[d * ROW_NW + w] += __popc(peers);
+            __syncwarp();
+        }
+        __syncthreads();
+        K *t = a;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
+template <typename K, typename KP>
+__device__ void row_sort_body(const S1Params &P, int64_t I, K *keysA, K *keysB, uint32_t *posB_s, KP *kpos_s,
+                              uint32_t *hist, int *sm, int ub) {
+    const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
+    const int nA = (int)(a1 - a0);
+    const int64_t base = P.costOff[a0];
+    const int64_t U = P.costOff[a1] - base;
+    const int jlo = P.rowJlo[I];
+    const uint32_t W = (uint32_t)(P.rowJhi[I] - jlo + 1);  // sentinel value for invalid candidates
+    const int wb = bits_for(W);
+    const K umask = (K)(((uint64_t)1 << ub) - 1);
+
+    // expansion (load-balanced over the row's candidates)
+    int nv = 0;
+    for (int64_t u = threadIdx.x; u < U; u += ROW_T) {
+        const int64_t target = base + u;
+        int lo = 0, hi = nA - 1;
+        while (lo < hi) {
+            int mid = (lo + hi + 1) >> 1;
+            if (P.costOff[a0 + mid] <= target) lo = mid;
+            else hi = mid - 1;
+        }
+        const int64_t t = a0 + lo;
+        const int64_t s = target - P.costOff[t];
+        const int64_t st = P.startA[t];
+        uint32_t posB;
+        bool valid;
+        if (st < 0) {
+            posB = P.list[-st - 1 + s];
+            valid = true;
+        } else {
+            posB = (uint32_t)(st + s);
+            valid = (P.rowOccB[posB] & P.colOccA[t]) != 0;
+        }
+        const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : W;
+        keysA[u] = ((K)jr << ub) | (K)u;
+        posB_s[u] = posB;
+        kpos_s[u] = (KP)lo;
+        nv += valid;
+    }
+    int nvalid;
+    block_scan_int(nv, &nvalid, sm);
+
+    K *R = block_radix_sort<K>(keysA, keysB, U, ub, wb, hist, sm);
+
+    // heads: blocked ownership so ranks follow from one CTA scan
+    const int64_t ipt = (nvalid + ROW_T - 1) / ROW_T;
+    const int64_t i0 = min((int64_t)nvalid, (int64_t)threadIdx.x * ipt), i1 = min((int64_t)nvalid, i0 + ipt);
+    int h = 0;
+    {
+        int64_t prev = (i0 > 0) ? (int64_t)(R[i0 - 1] >> ub) : -1;
+        for (int64_t i = i0; i < i1; i++) {
+            int64_t jr = (int64_t)(R[i] >> ub);
+            h += (jr != prev);
+            prev = jr;
+        }
+    }
+    int nCrow;
+    int rank = block_scan_int(h, &nCrow, sm);
+    {
+        int64_t prev = (i0 > 0) ? (int64_t)(R[i0 - 1] >> ub) : -1;
+        for (int64_t i = i0; i < i1; i++) {
+            const K key = R[i];
+            const int64_t jr = (int64_t)(key >> ub);
+            const int64_t u = (int64_t)(key & umask);
+            const uint64_t pA = (uint64_t)(a0 + (int64_t)kpos_s[u]);
+            P.pairs[base + i] = (pA << 32) | (uint64_t)posB_s[u];
+            if (jr != prev) {
+                P.tJ[base + rank] = jlo + (int32_t)jr;
+                P.tStart[base + rank] = (uint32_t)i;
+                rank++;
+            }
+            prev = jr;
+        }
+    }
+    __syncthreads();
+    for (int r = threadIdx.x; r < nCrow; r += ROW_T) {
+        const uint32_t b = P.tStart[base + r];
+        const uint32_t e = (r + 1 < nCrow) ? P.tStart[base + r + 1] : (uint32_t)nvalid;
+        P.tCnt[base + r] = e - b;
+        // work estimate for step 2's class split: number of (pair, c) items, i.e. columns c of
+        // A_IK whose B_KJ row c is non-empty
+        uint32_t w = 0;
+        for (uint32_t i = b; i < e; i++) {
+            const int64_t u = (int64_t)(R[i] & umask);
+            w += __popc((uint32_t)P.colOccA[a0 + (int64_t)kpos_s[u]] & (uint32_t)P.rowOccB[posB_s[u]]);
+        }
+        P.tWork[base + r] = w;
+    }
+    if (threadIdx.x == 0) {
+        P.nC[I] = nCrow;
+        atomicAdd(&P.cnt->pairs, (u64c)nvalid);
+    }
+}
+
+__global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int64_t tm, int cap) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ uint32_t hist[256 * ROW_NW];
+    __shared__ int sm[ROW_NW + 1];
+    const int64_t I = blockIdx.x;
+    if (I >= tm || P.rowClass[I] != ROW_SMALL) return;
+    uint32_t *keysA = reinterpret_cast<uint32_t *>(smem);
+    uint32_t *keysB = keysA + cap;
+    uint32_t *posB = keysB + cap;
+    uint16_t *kpos = reinterpret_cast<uint16_t *>(posB + cap);
+    const int64_t U = P.costOff[P.tpA[I + 1]] - P.costOff[P.tpA[I]];
+    const int ub = bits_for((uint64_t)(U > 1 ? U - 1 : 1));
+    row_sort_body<uint32_t, uint16_t>(P, I, keysA, keysB, posB, kpos, hist, sm, ub);
+}
+
+__global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) {
+    __shared__ uint32_t hist[256 * ROW_NW];
+    __shared__ int sm[ROW_NW + 1];
+    const int64_t I = P.bigList[blockIdx.x];
+    const int64_t o = P.bigOff[I];
+    row_sort_body<uint64_t, uint32_t>(P, I, P.bigKeysA + o, P.bigKeysB + o, P.bigPosB + o, P.bigKpos + o, hist, sm,
+                                      32);
+}
+
+// transposed tile masks: maskT[c] bit r <=> nonzero (r,c)  (used by the item-driven paths)
+__global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ maskT) {
+    int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= nt) return;
+    const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
+    uint4 a = __ldg(p), b = __ldg(p + 1);
+    uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    uint32_t col[TILE];
+#pragma unroll
+    for (int c = 0; c < TILE; c++) col[c] = 0;
+#pragma unroll
+    for (int r = 0; r < TILE; r++) {
+        uint32_t m = (w[r >> 1] >> (16 * (r & 1))) & 0xffffu;
+#pragma unroll
+        for (int c = 0; c < TILE; c++) col[c] |= ((m >> c) & 1u) << r;
+    }
+    uint4 *o = reinterpret_cast<uint4 *>(maskT + t * TILE);
+    o[0] = make_uint4(col[0] | col[1] << 16, col[2] | col[3] << 16, col[4] | col[5] << 16, col[6] | col[7] << 16);
+    o[1] = make_uint4(col[8] | col[9] << 16, col[10] | col[11] << 16, col[12] | col[13] << 16,
+                      col[14] | col[15] << 16);
+}
+
+// ------------------------------------------------------------------------------------------
+// compaction: per-C-tile arrays (tile column, pair range, work estimate) from the per-row step-1
+// results, one warp per tile row
+// ------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_compact(CompactParams P) {
+    const int lane = threadIdx.x & 31;
+    const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (I >= P.tm) return;
+    const int64_t base = P.costOff[P.tpA[I]];
+    const int64_t t0 = P.tilePtrC[I], n = P.tilePtrC[I + 1] - t0;
+    for (int64_t r = lane; r < n; r += 32) {
+        const int64_t slot = base + r, t = t0 + r;
+        P.tile_col[t] = P.tJ[slot];
+        P.pairBeg[t] = base + P.tStart[slot];
+        P.pairCnt[t] = P.tCnt[slot];
+        P.work[t] = P.tWork[slot];
+    }
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+// launchers
+// ------------------------------------------------------------------------------------------
+void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s) {
+    TSG_LAUNCH(k_occupancy, grid_for(nt, 256), 256, 0, s, mask, nt, row_occ, col_occ);
+}
+
+void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
+                    uint32_t *list, cudaStream_t s) {
+    TSG_LAUNCH(k_rowlist, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, lptr, lcnt, list);
+}
+
+void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int64_t ntA, const int32_t *tcA,
+                     const uint16_t *maskA, int32_t *rnnz, DevCounters *cnt, cudaStream_t s) {
+    TSG_LAUNCH(k_brow_nnz, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, rnnz);
+    TSG_LAUNCH(k_products, grid_for(ntA, 256), 256, 0, s, ntA, tcA, maskA, (const int32_t *)rnnz, cnt);
+}
+
+void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA, const int64_t *tpB,
+                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, bool scan_only, int64_t *cost,
+                       int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s) {
+    TSG_LAUNCH(k_atile_plan, grid_for(ntA, 256), 256, 0, s, ntA, tcA, colOccA, tpB, tcB, lptr, list, scan_only, cost,
+               start, jlo, jhi, cnt);
+}
+
+void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
+                     const int32_t *jhiA, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass, int64_t *nC,
+                     int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s) {
+    TSG_LAUNCH(k_row_plan, grid_for(tmA, 8), 256, 0, s, tmA, tpA, costOff, jloA, jhiA, rowJlo, rowJhi, rowClass, nC,
+               bigList, bigOff, cnt);
+}
+
+void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s) {
+    TSG_LAUNCH(k_transpose, grid_for(nt, 256), 256, 0, s, mask, nt, maskT);
+}
+
+void launch_compact(const CompactParams &P, cudaStream_t s) {
+    TSG_LAUNCH(k_compact, grid_for(P.tm, 8), 256, 0, s, P);
+}
+
+void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, cudaStream_t s) {
+    if (max_u_small > 0) {
+        const int cap = (int)((max_u_small + 31) & ~31LL);
+        const size_t smem = (size_t)cap * (4 + 4 + 4 + 2);
+        TSG_CUDA(cudaFuncSetAttribute(k_row_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        TSG_LAUNCH(k_row_small, (unsigned)tm, ROW_T, smem, s, P, tm, cap);
+    }
+    if (nbig > 0) TSG_LAUNCH(k_row_big, (unsigned)nbig, ROW_T, 0, s, P);
+}
+
+
+}  // namespace tsg
