@@ -1,0 +1,68 @@
+#!/usr/bin/env python
+"""Summarise ncu captures into text for profiles/ (the .ncu-rep files stay in gpurun_out/).
+
+    python profiles/summarize.py launches <launches.csv>            # per-kernel time shares
+    python profiles/summarize.py full <a.ncu-rep> [<b.ncu-rep> ...]  # key --set full metrics
+"""
+import collections
+import csv
+import subprocess
+import sys
+
+KEYS = [
+    ("gpu__time_duration.sum", "duration"),
+    ("dram__bytes_read.sum", "DRAM read"),
+    ("dram__bytes_write.sum", "DRAM write"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "DRAM % of peak"),
+    ("lts__t_sector_hit_rate.pct", "L2 hit %"),
+    ("l1tex__t_sector_hit_rate.pct", "L1 hit %"),
+    ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "SM throughput %"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue active %"),
+    ("smsp__inst_executed.sum", "warp instructions"),
+    ("smsp__thread_inst_executed_per_inst_executed.ratio", "threads / instruction"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy %"),
+    ("launch__registers_per_thread", "registers / thread"),
+    ("launch__occupancy_limit_shared_mem", "occupancy limit (smem, CTAs)"),
+    ("launch__occupancy_limit_registers", "occupancy limit (regs, CTAs)"),
+    ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "long-scoreboard stalls / issue"),
+    ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum", "smem ld bank conflicts"),
+    ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum", "smem st bank conflicts"),
+]
+
+
+def launches(path):
+    rows = list(csv.reader(open(path)))
+    hi = [i for i, r in enumerate(rows) if r and r[0] == "ID"][0]
+    h = rows[hi]
+    ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
+    agg = collections.OrderedDict()
+    for r in rows[hi + 1:]:
+        name = r[ki].split("(")[0].split("::")[-1]
+        v = float(r[vi].replace(",", ""))
+        u = r[ui]
+        v = v / 1e3 if u in ("nsecond", "ns") else (v * 1e3 if u in ("msecond", "ms") else v)
+        agg.setdefault(name, []).append(v)
+    tot = sum(sum(v) for v in agg.values())
+    print(f"| kernel | launches | total us | mean us | share |\n|---|---|---|---|---|")
+    for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
+        print(f"| {k} | {len(v)} | {sum(v):.1f} | {sum(v) / len(v):.1f} | {sum(v) / tot * 100:.1f}% |")
+
+
+def full(paths):
+    for p in paths:
+        out = subprocess.run(["ncu", "-i", p, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+        r = list(csv.reader(out.splitlines()))
+        h, u, v = r[0], r[1], r[2]
+        kname = v[h.index("Kernel Name")] if "Kernel Name" in h else p
+        print(f"\n### {p.split('/')[-1]}  ({kname.split('(')[0]})\n\n| metric | value |\n|---|---|")
+        for key, label in KEYS:
+            if key in h:
+                i = h.index(key)
+                print(f"| {label} (`{key}`) | {v[i]} {u[i]} |")
+
+
+if __name__ == "__main__":
+    if sys.argv[1] == "launches":
+        launches(sys.argv[2])
+    else:
+        full(sys.argv[2:])
