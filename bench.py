@@ -174,6 +174,7 @@ def main():
     ap.add_argument("--cpu-budget-s", type=float, default=12.0)
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
+    ap.add_argument("--step3-rows", action="store_true", help="step 3 in the whole-tile-row kernel (experimental)")
     args = ap.parse_args()
     if args.warmup < 3 and not args.profile:
         args.warmup = 3
@@ -218,7 +219,7 @@ def main():
     flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev) if small_inputs else None
 
     def one_step(timing=True):
-        return tsg.spgemm(Ashard, T, stats=True, timing=timing)
+        return tsg.spgemm(Ashard, T, stats=True, timing=timing, step3_rows=args.step3_rows)
 
     for _ in range(args.warmup):
         C = one_step()

@@ -103,6 +103,8 @@ typedef struct {
     int32_t host_syncs;       /* blocking device->host scalar reads performed */
     float ms_index, ms_step1, ms_step2, ms_alloc, ms_step3, ms_total; /* CUDA-event times */
     float ms_host_sync, ms_host_alloc; /* host wall time blocked in scalar reads / allocation calls */
+    int64_t step3_row_tiles;  /* C tiles whose step 3 ran in the whole-tile-row kernel */
+    int64_t step3_rows;       /* tile rows handled by that kernel */
 } tsg_stats;
 
 /* flags for tsg_csr_to_tiles */
@@ -115,6 +117,7 @@ typedef struct {
 #define TSG_STEP1_SCAN_ONLY 0x4u  /* force mode (i) tile-row scans in step 1 */
 #define TSG_STEP1_LIST_ALWAYS 0x8u/* build B-row lists and use them wherever they are cheaper */
 #define TSG_STATS_PRODUCTS 0x10u  /* also count intermediate products into stats->products */
+#define TSG_STEP3_ROWS 0x20u      /* step 3 in the whole-tile-row kernel where rows fit (experimental; same results) */
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = 192; 257 disables dense) */
 
 /*
@@ -147,7 +150,9 @@ TSG_API tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int
  * Values: C(r,j) = sum over pairs in ascending K, over c ascending, of A(r,c)*B(c,j) with
  * fused multiply-add, i.e. ascending global k (reading A8/A16): deterministic run to run.
  * Syncs: 3 blocking scalar reads (candidate total, C tile count, nnz(C)).
- * Errors: INVALID_ARG, SHAPE, OVERFLOW, OOM, CUDA, INTERNAL.
+ * Alignment: mask and row_ptr of A and B must be 16-byte aligned, val 8-byte aligned (tiles are
+ * staged into shared memory in 16-byte chunks); handles made by this library always are.
+ * Errors: INVALID_ARG (incl. alignment), SHAPE, OVERFLOW, OOM, CUDA, INTERNAL.
  */
 TSG_API tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags,
                       const tsg_allocator *al, void *stream, tsg_tiles **C, tsg_stats *stats);

@@ -21,7 +21,9 @@ struct DevCounters {
     u64c n3small;      // step-3 class sizes
     u64c n3medium;
     u64c n3dense;
-    u64c pad;
+    u64c n3rows;       // tile rows handled by the row kernel of step 3
+    u64c n3fallback;   // C tiles left to the per-tile kernel of step 3
+    u64c next3;        // work counter of the step-3 row kernel
 };
 
 constexpr int ROW_T = 256;        // threads of a step-1 row CTA
@@ -100,6 +102,44 @@ struct StepParams {
     uint8_t *ixC;
     double *vC;
     const uint32_t *work;  // step-2 class split
+    const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
+    int dense_threshold;
+    DevCounters *cnt;
+};
+
+// ---------------- a4 step 3, row kernel: one CTA per C tile row, tiles staged by TMA bulk copies
+constexpr int R3_T = 256;          // threads
+constexpr int R3_NTC = 128;        // max C tiles of a row
+constexpr int R3_NAC = 32;         // max A tiles of a row (one warp plans them)
+constexpr int R3_NPC = 2048;       // max pairs of a row
+constexpr int R3_ACC = 8192;       // max accumulator doubles of a row (compact + dense blocks)
+constexpr int R3_SMEM = 100 * 1024;  // dynamic shared memory per CTA
+
+struct RowParams {
+    int64_t tm;
+    const int64_t *tpA;
+    const int32_t *tcA;
+    const int64_t *tnzA;
+    const uint8_t *rpA;
+    const uint16_t *mA;
+    const uint16_t *colOccA;
+    const double *vA;
+    const int64_t *tpB;
+    const int64_t *tnzB;
+    const uint8_t *rpB;
+    const uint16_t *mB;
+    const double *vB;
+    const uint64_t *pairs;
+    const int64_t *pairBeg;
+    const uint32_t *pairCnt;
+    const int64_t *tpC;
+    const int64_t *tnzC;  // offsets (ntC + 1)
+    const uint8_t *rpC;
+    const uint16_t *mC;
+    uint8_t *ixC;
+    double *vC;
+    int32_t *rowAcc;  // per tile row: accumulator doubles if the row kernel takes it, else -1
+    uint8_t *skip;    // per C tile
     int dense_threshold;
     DevCounters *cnt;
 };
@@ -123,5 +163,8 @@ void launch_compact(const CompactParams &P, cudaStream_t s);
 // launchers (tsg_step23.cu)
 void launch_step2(const StepParams &P, cudaStream_t s);
 void launch_step3(const StepParams &P, cudaStream_t s);
+// launchers (tsg_step3row.cu)
+void launch_step3_class(const RowParams &R, cudaStream_t s);
+void launch_step3_rows(const RowParams &R, cudaStream_t s);
 
 }  // namespace tsg

@@ -46,8 +46,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     reset_call_launches();
     TSG_REQUIRE(A->nt < ((int64_t)1 << 31) && B->nt < ((int64_t)1 << 31), TSG_ERR_OVERFLOW, "input has >= 2^31 tiles");
     TSG_REQUIRE(A->tn == B->tm, TSG_ERR_SHAPE, "tile shapes disagree");
-    TSG_REQUIRE(((uintptr_t)A->mask & 15) == 0 && ((uintptr_t)B->mask & 15) == 0, TSG_ERR_INVALID_ARG,
-                "mask arrays must be 16-byte aligned");
+    TSG_REQUIRE(((uintptr_t)A->mask & 15) == 0 && ((uintptr_t)B->mask & 15) == 0 && ((uintptr_t)A->row_ptr & 15) == 0 &&
+                    ((uintptr_t)B->row_ptr & 15) == 0 && ((uintptr_t)A->val & 7) == 0 && ((uintptr_t)B->val & 7) == 0,
+                TSG_ERR_INVALID_ARG, "mask and row_ptr arrays must be 16-byte aligned, val 8-byte aligned");
     int TH = (int)((flags >> TSG_DENSE_THRESHOLD_SHIFT) & 0x1ffu);
     if (TH == 0) TH = TSG_DENSE_NNZ;
     Timer tm_;
@@ -192,8 +193,40 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     // ---------------- a3: offsets of C's nonzeros, allocation
     exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp);
     tm_.mark(4);
+    // step-3 row classes: whole C tile rows for the row kernel, the rest per tile
+    RowParams R{};
+    R.tm = tmA;
+    R.tpA = A->tile_ptr;
+    R.tcA = A->tile_col;
+    R.tnzA = A->tile_nnz;
+    R.rpA = A->row_ptr;
+    R.mA = A->mask;
+    R.colOccA = colOccA;
+    R.vA = A->val;
+    R.tpB = B->tile_ptr;
+    R.tnzB = B->tile_nnz;
+    R.rpB = B->row_ptr;
+    R.mB = B->mask;
+    R.vB = B->val;
+    R.pairs = P1.pairs;
+    R.pairBeg = pairBeg;
+    R.pairCnt = pairCnt;
+    R.tpC = tile_ptr;
+    R.tnzC = tile_nnz;
+    R.rpC = row_ptr;
+    R.mC = mask;
+    R.dense_threshold = TH;
+    R.cnt = cnt;
+    const bool rowk = (flags & TSG_STEP3_ROWS) != 0;
+    if (rowk) {
+        R.rowAcc = tmp.get<int32_t>(tmA);
+        R.skip = tmp.get<uint8_t>(ntC);
+        launch_step3_class(R, s);
+    }
     int64_t nnzC = 0;
+    DevCounters hc2{};
     TSG_CUDA(cudaMemcpyAsync(&nnzC, tile_nnz + ntC, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    TSG_CUDA(cudaMemcpyAsync(&hc2, cnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
     {
         const double t0 = now_ms();
         TSG_CUDA(cudaStreamSynchronize(s));
@@ -207,7 +240,13 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     // ---------------- a4: step 3
     P.ixC = idx;
     P.vC = val;
-    launch_step3(P, s);
+    R.ixC = idx;
+    R.vC = val;
+    if (rowk && hc2.n3rows > 0) launch_step3_rows(R, s);
+    if (!rowk || hc2.n3fallback > 0) {
+        P.skip = rowk ? R.skip : nullptr;
+        launch_step3(P, s);
+    }
     tm_.mark(6);
 
     // ---------------- the result handle
@@ -243,6 +282,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         st->pairs = (int64_t)fin.pairs;
         st->tiles_dense = (int64_t)fin.n3dense;
         st->tiles_sparse = ntC - (int64_t)fin.n3dense;
+        st->step3_rows = (int64_t)fin.n3rows;
+        st->step3_row_tiles = rowk ? ntC - (int64_t)fin.n3fallback : 0;
         st->step1_list_tiles = (int32_t)fin.list_tiles;
         st->host_syncs = syncs;
         st->kernel_launches = call_launches();

@@ -392,7 +392,7 @@ __global__ void __launch_bounds__(T3) k_s3(StepParams P) {
     const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
     for (int64_t g = (int64_t)blockIdx.x * (T3 / 32) + w; g < ngroups; g += gstride) {
         const int64_t t = g * 32 + lane;
-        const bool v = t < P.ntC;
+        const bool v = t < P.ntC && !(P.skip && P.skip[t]);
         const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
         const bool dense = v && nz >= P.dense_threshold;
         const bool small = v && !dense && nz <= SMALL_NNZ;

@@ -161,16 +161,33 @@ def _abs_csr(A, B):
 
 
 @pytest.mark.parametrize("opts", [dict(scan_only=True), dict(list_always=True), dict(dense_threshold=1),
-                                  dict(dense_threshold=257), dict(dense_threshold=100)])
+                                  dict(dense_threshold=257), dict(dense_threshold=100), dict(step3_rows=True),
+                                  dict(step3_rows=True, dense_threshold=1)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
-    for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1")):
+    for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12)):
         T = tiles_of(tsg, A)
         base = host(tsg.spgemm(T, T))
         alt = host(tsg.spgemm(T, T, **opts))
         for k in ARRAYS[:-1]:
             assert np.array_equal(base[k], alt[k]), (opts, k)
         assert bitwise_equal_values(base["val"], alt["val"])
+
+
+def test_step3_row_kernel_coverage(tsg):
+    """Stencil/FEM tile rows go through the whole-row kernel; hub rows fall back per tile."""
+    for A, allrows in ((gen.stencil27(12), True), (gen.strip_fem(6, 20, 6), True),
+                       (gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004), False)):
+        T = tiles_of(tsg, A)
+        C = tsg.spgemm(T, T, stats=True, step3_rows=True)
+        st = C.stats
+        if allrows:
+            assert st["step3_row_tiles"] == C.num_tiles and st["step3_rows"] > 0
+        else:
+            assert st["step3_row_tiles"] < C.num_tiles
+        ref = oracle.expected_tiles(A, A, fma=True)
+        assert_tiles_equal(host(C), ref)
+        assert tsg.spgemm(T, T, stats=True).stats["step3_row_tiles"] == 0
 
 
 def test_threshold_boundary_tiles(tsg):
