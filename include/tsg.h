@@ -200,6 +200,13 @@ TSG_API void tsg_tiles_destroy(tsg_tiles *T, void *stream);
 /* Free an array returned by tsg_tiles_to_csr (same allocator; NULL al = cudaFreeAsync). */
 TSG_API void tsg_free(void *ptr, size_t bytes, const tsg_allocator *al, void *stream);
 
+/* Scratch workspace: with no user allocator, the temporary arrays of a call (step-1 pairs,
+ * occupancy words, scans, ...) come from a per-thread, per-device cached arena that grows to the
+ * largest call seen and is reused (so repeated calls do no device allocation besides C's arrays).
+ * This releases the calling thread's arena on the current device (stream-ordered on `stream`).
+ * Returns the bytes it held. */
+TSG_API size_t tsg_workspace_release(void *stream);
+
 TSG_API const char *tsg_status_string(tsg_status s);
 TSG_API const char *tsg_last_error(void);
 TSG_API int tsg_abi_version(void);

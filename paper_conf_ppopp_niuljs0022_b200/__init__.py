@@ -23,7 +23,7 @@ from . import _lib
 from ._lib import TILE, DENSE_NNZ, TsgError  # noqa: F401
 
 __all__ = ["Tiles", "csr_to_tiles", "spgemm", "tiles_to_csr", "slice_rows", "wrap", "TsgError",
-           "kernel_launch_count"]
+           "kernel_launch_count", "workspace_release"]
 
 _DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8)}
 
@@ -263,3 +263,8 @@ def wrap(m: int, n: int, arrays: dict, keepalive=None) -> Tiles:
 
 def kernel_launch_count() -> int:
     return int(_lib.load().tsg_kernel_launch_count())
+
+
+def workspace_release(stream=None) -> int:
+    """Free this thread's cached scratch arena on the current device (tsg_workspace_release)."""
+    return int(_lib.load().tsg_workspace_release(C.c_void_p(_stream_ptr(stream))))

@@ -39,6 +39,61 @@ static void ensure_pool_cached() {
     done.store(dev);
 }
 
+Arena &thread_arena() {
+    static thread_local Arena arenas[16];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0) dev = 0;
+    Arena &a = arenas[dev & 15];
+    a.dev = dev;
+    return a;
+}
+
+void Buffers::enter_arena() {
+    Arena &a = *arena_;
+    if (a.depth++ == 0) {
+        // the previous user of the arena may still run on another stream
+        if (a.done && a.last != s_) TSG_CUDA(cudaStreamWaitEvent(s_, a.done, 0));
+        // grow after a call that overflowed (stream-ordered free of the old buffer)
+        if (a.want > a.cap) {
+            if (a.base) cudaFreeAsync(a.base, s_);
+            a.base = nullptr;
+            a.cap = 0;
+            const size_t cap = (a.want + (a.want >> 3) + ((size_t)1 << 20)) & ~(size_t)255;
+            const double t0 = now_ms();
+            void *p = nullptr;
+            ensure_pool_cached();
+            if (cudaMallocAsync(&p, cap, s_) == cudaSuccess) {
+                a.base = static_cast<char *>(p);
+                a.cap = cap;
+            } else {
+                cudaGetLastError();
+            }
+            t_host_alloc_ms += now_ms() - t0;
+        }
+        a.want = 0;
+        a.off = 0;
+    }
+    mark_ = a.off;
+}
+
+void Buffers::leave_arena() {
+    Arena &a = *arena_;
+    a.off = mark_;
+    if (--a.depth == 0) {
+        if (!a.done) cudaEventCreateWithFlags(&a.done, cudaEventDisableTiming);
+        if (a.done) cudaEventRecord(a.done, s_);
+        a.last = s_;
+    }
+}
+
+void arena_release_all(cudaStream_t s) {
+    Arena &a = thread_arena();
+    if (a.depth) return;
+    if (a.base) cudaFreeAsync(a.base, s);
+    a.base = nullptr;
+    a.cap = a.off = a.want = 0;
+}
+
 void *Allocator::alloc(size_t bytes, cudaStream_t s) const {
     if (custom) return hook.alloc(bytes, (void *)s, hook.ctx);
     ensure_pool_cached();
@@ -144,7 +199,7 @@ tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *ro
         T->al = A;
         try {
             if (flags & TSG_INPUT_HOST) {
-                Buffers staging(A, s);
+                Buffers staging(A, s, true);
                 int64_t *drp = staging.get<int64_t>(m + 1);
                 int32_t *dci = staging.get<int32_t>(nnz);
                 double *dv = staging.get<double>(nnz);
@@ -330,6 +385,12 @@ void tsg_tiles_destroy(tsg_tiles *T, void *stream) { destroy_handle(T, (cudaStre
 
 void tsg_free(void *ptr, size_t bytes, const tsg_allocator *al, void *stream) {
     Allocator::from(al).free(ptr, bytes, (cudaStream_t)stream);
+}
+
+size_t tsg_workspace_release(void *stream) {
+    const size_t held = thread_arena().cap;
+    arena_release_all((cudaStream_t)stream);
+    return held;
 }
 
 }  // extern "C"

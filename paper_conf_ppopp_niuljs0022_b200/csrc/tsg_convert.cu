@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(256) k_t2c(int64_t m, int64_t tm, const int64_
 
 void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, const int32_t *ci, const double *v,
                          bool validate, const Allocator &al, cudaStream_t s, tsg_tiles *T) {
-    Buffers tmp(al, s), out(al, s);
+    Buffers tmp(al, s, true), out(al, s);
     const int64_t tm = ceil_div(m, TILE), tn = ceil_div(n, TILE);
     const unsigned grid = grid_for(ceil_div(tm, 2), 8);  // 8 warps x 2 tile rows per CTA
     if (validate && m > 0) {

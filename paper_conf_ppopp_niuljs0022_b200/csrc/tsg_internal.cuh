@@ -78,15 +78,53 @@ struct Allocator {
     void free(void *p, size_t bytes, cudaStream_t s) const;
 };
 
+// Scratch arena (per host thread and device): one cached device buffer handed out as a stack.
+// Scratch of a call never goes back to the allocator, so the stream-ordered pool only holds
+// outputs and its layout stays stable run to run (no pool growth -- i.e. no synchronous memory
+// mapping -- inside a timed call once the arena has reached the workload's peak).  The arena is
+// grown after a call that overflowed it; a CUDA event orders its reuse on another stream.
+struct Arena {
+    int dev = -1;
+    char *base = nullptr;
+    size_t cap = 0, off = 0, want = 0;
+    cudaEvent_t done = nullptr;
+    cudaStream_t last = nullptr;
+    int depth = 0;
+};
+Arena &thread_arena();
+void arena_release_all(cudaStream_t s);  // free the calling thread's arena (stream-ordered)
+
 // RAII list of device buffers; frees (stream-ordered) whatever is still owned at scope exit.
+// With scratch=true (and no user allocator) buffers come from the thread's arena.
 class Buffers {
    public:
-    Buffers(const Allocator &al, cudaStream_t s) : al_(al), s_(s) {}
-    ~Buffers() { release_all(); }
+    Buffers(const Allocator &al, cudaStream_t s, bool scratch = false) : al_(al), s_(s) {
+        if (scratch && !al.custom) {
+            arena_ = &thread_arena();
+            enter_arena();
+        }
+    }
+    ~Buffers() {
+        release_all();
+        if (arena_) leave_arena();
+    }
     template <typename T>
     T *get(int64_t count) {
         size_t bytes = sizeof(T) * (size_t)(count > 0 ? count : 0);
         if (bytes < 256) bytes = 256;  // never hand out NULL; keep 256-byte alignment
+        bytes = (bytes + 255) & ~(size_t)255;
+        if (arena_) {
+            Arena &a = *arena_;
+            if (a.off + bytes <= a.cap) {
+                void *p = a.base + a.off;
+                a.off += bytes;
+                return static_cast<T *>(p);
+            }
+            // overflow: served by the allocator below; keep counting so the arena is grown to
+            // this call's whole scratch peak for the next call
+            a.off += bytes;
+            if (a.off > a.want) a.want = a.off;
+        }
         const double t0 = now_ms();
         void *p = al_.alloc(bytes, s_);
         t_host_alloc_ms += now_ms() - t0;
@@ -111,6 +149,8 @@ class Buffers {
     }
 
    private:
+    void enter_arena();
+    void leave_arena();
     struct Item {
         void *p;
         size_t bytes;
@@ -118,6 +158,8 @@ class Buffers {
     Allocator al_;
     cudaStream_t s_;
     std::vector<Item> items_;
+    Arena *arena_ = nullptr;
+    size_t mark_ = 0;
 };
 
 }  // namespace tsg

@@ -55,7 +55,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     tm_.init((flags & TSG_STATS_TIMING) && st, s);
     tm_.mark(0);
 
-    Buffers tmp(al, s), out(al, s);
+    Buffers tmp(al, s, true), out(al, s);
     const int64_t ntA = A->nt, tmA = A->tm, tmB = B->tm;
     int syncs = 0;
     DevCounters *cnt = tmp.get<DevCounters>(1);
