@@ -226,14 +226,26 @@ __device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigne
     }
 }
 
-struct MedStage {  // per half warp: staged metadata of up to 16 pairs
-    uint32_t pA[BATCH], pB[BATCH];
+struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
+    uint16_t mA[BATCH][TILE], mB[BATCH][TILE];  // cp.async'd masks of A_IK and B_KJ
+    uint8_t rA[BATCH][TILE], rB[BATCH][TILE];   // and their row offsets
     int64_t zA[BATCH], zB[BATCH];
     uint16_t oB[BATCH];
 };
 
+__device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_wait_all() {
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+
 // medium tile: a half warp, lane r owns C row r; dense-in-j 16-slot row accumulator in shared
-// memory (conflict free), compacted through mask_C[r] at the end.  All 32 lanes must call.
+// memory (conflict free), compacted through mask_C[r] at the end.  Pairs go in batches of 16:
+// lane i stages pair i's A and B masks and row offsets (6 x 16-byte cp.async, all lanes and
+// pairs in flight at once), so a lane's walk over its row touches global memory only for the
+// values.  All 32 lanes must call.
 __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t t, double *acc, MedStage &S,
                                           int r) {
     uint32_t np = 0, mCr = 0;
@@ -255,37 +267,37 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
         const uint32_t q = bt * BATCH + r;
         if (q < np) {
             const uint64_t pr = pp[q];
-            const uint32_t pA = (uint32_t)(pr >> 32), pB = (uint32_t)pr;
-            S.pA[r] = pA;
-            S.pB[r] = pB;
+            const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+            cp16(&S.mA[r][0], P.mA + pA * TILE);
+            cp16(&S.mA[r][8], P.mA + pA * TILE + 8);
+            cp16(&S.mB[r][0], P.mB + pB * TILE);
+            cp16(&S.mB[r][8], P.mB + pB * TILE + 8);
+            cp16(&S.rA[r][0], P.rpA + pA * TILE);
+            cp16(&S.rB[r][0], P.rpB + pB * TILE);
             S.zA[r] = P.tnzA[pA];
             S.zB[r] = P.tnzB[pB];
             S.oB[r] = P.rowOccB[pB];
         }
+        cp_wait_all();
         __syncwarp();
         const uint32_t nb = np > bt * BATCH ? min((uint32_t)BATCH, np - bt * BATCH) : 0u;
         if (mCr)
             for (uint32_t i = 0; i < nb; i++) {
-                const int64_t pA = S.pA[i];
-                const uint32_t mAr = P.mA[pA * TILE + r];
+                const uint32_t mAr = S.mA[i][r];
                 uint32_t ma = mAr & S.oB[i];
                 if (!ma) continue;
-                const int64_t pB = S.pB[i];
-                const double *va = P.vA + S.zA[i] + P.rpA[pA * TILE + r];
+                const double *va = P.vA + S.zA[i] + S.rA[i][r];
                 const double *vbt = P.vB + S.zB[i];
-                const uint16_t *mbt = P.mB + pB * TILE;
-                const uint8_t *rbt = P.rpB + pB * TILE;
                 while (ma) {
                     const int c = __ffs(ma) - 1;
                     ma &= ma - 1;
                     const double a = va[__popc(mAr & ((1u << c) - 1u))];
-                    uint32_t mbc = mbt[c];
-                    const double *vb = vbt + rbt[c];
-                    int ib = 0;
+                    uint32_t mbc = S.mB[i][c];
+                    const double *vb = vbt + S.rB[i][c];
                     while (mbc) {
                         const int j = __ffs(mbc) - 1;
                         mbc &= mbc - 1;
-                        acc[j * 16] = fma(a, vb[ib++], acc[j * 16]);
+                        acc[j * 16] = fma(a, *vb++, acc[j * 16]);
                     }
                 }
             }
