@@ -241,6 +241,55 @@ __device__ __forceinline__ void cp_wait_all() {
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
 }
 
+// one column c of A's row r in flight: a = A(r,c), B's row c (mask, first 4 values, the rest)
+struct BRow {
+    double a, b0, b1, b2, b3;
+    uint32_t m;
+    const double *vb;
+};
+__device__ __forceinline__ BRow load_brow(const MedStage &S, int i, int c, uint32_t mAr, const double *va,
+                                          const double *vbt) {
+    BRow x;
+    x.m = S.mB[i][c];
+    x.vb = vbt + S.rB[i][c];
+    x.a = va[__popc(mAr & ((1u << c) - 1u))];
+    const int n = __popc(x.m);
+    x.b0 = x.vb[0];  // every row c here is non-empty (filtered by rowOcc(B))
+    x.b1 = n > 1 ? x.vb[1] : 0.0;
+    x.b2 = n > 2 ? x.vb[2] : 0.0;
+    x.b3 = n > 3 ? x.vb[3] : 0.0;
+    return x;
+}
+// acc[16 j] += a * B(c, j) over B's row c in ascending j (row accumulator: lane-strided slots).
+// The first four slots are distinct, so their loads, FMAs and stores are issued as a group
+// (independent shared-memory round trips instead of a chain of four).
+__device__ __forceinline__ void accumulate_brow(const BRow &x, double *acc) {
+    uint32_t m = x.m;
+    const int j0 = __ffs(m) - 1;
+    m &= m - 1;
+    const int j1 = m ? __ffs(m) - 1 : j0;
+    m &= m - 1;
+    const int j2 = m ? __ffs(m) - 1 : j0;
+    m &= m - 1;
+    const int j3 = m ? __ffs(m) - 1 : j0;
+    m &= m - 1;
+    const int n = __popc(x.m);
+    double c0 = acc[j0 * 16], c1 = 0.0, c2 = 0.0, c3 = 0.0;
+    if (n > 1) c1 = acc[j1 * 16];
+    if (n > 2) c2 = acc[j2 * 16];
+    if (n > 3) c3 = acc[j3 * 16];
+    acc[j0 * 16] = fma(x.a, x.b0, c0);
+    if (n > 1) acc[j1 * 16] = fma(x.a, x.b1, c1);
+    if (n > 2) acc[j2 * 16] = fma(x.a, x.b2, c2);
+    if (n > 3) acc[j3 * 16] = fma(x.a, x.b3, c3);
+    const double *vb = x.vb + 4;
+    while (m) {
+        const int j = __ffs(m) - 1;
+        m &= m - 1;
+        acc[j * 16] = fma(x.a, *vb++, acc[j * 16]);
+    }
+}
+
 // medium tile: a half warp, lane r owns C row r; dense-in-j 16-slot row accumulator in shared
 // memory (conflict free), compacted through mask_C[r] at the end.  Pairs go in batches of 16:
 // lane i stages pair i's A and B masks and row offsets (6 x 16-byte cp.async, all lanes and
@@ -288,17 +337,23 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
                 if (!ma) continue;
                 const double *va = P.vA + S.zA[i] + S.rA[i][r];
                 const double *vbt = P.vB + S.zB[i];
-                while (ma) {
-                    const int c = __ffs(ma) - 1;
-                    ma &= ma - 1;
-                    const double a = va[__popc(mAr & ((1u << c) - 1u))];
-                    uint32_t mbc = S.mB[i][c];
-                    const double *vb = vbt + S.rB[i][c];
-                    while (mbc) {
-                        const int j = __ffs(mbc) - 1;
-                        mbc &= mbc - 1;
-                        acc[j * 16] = fma(a, *vb++, acc[j * 16]);
+                // software pipeline over the columns c of A's row: the loads of column c+1 (its A
+                // value and the first 4 values of B's row c+1) are in flight while column c's
+                // products are accumulated
+                int c = __ffs(ma) - 1;
+                ma &= ma - 1;
+                BRow cur = load_brow(S, i, c, mAr, va, vbt);
+                for (;;) {
+                    const bool more = ma != 0;
+                    BRow nxt;
+                    if (more) {
+                        c = __ffs(ma) - 1;
+                        ma &= ma - 1;
+                        nxt = load_brow(S, i, c, mAr, va, vbt);
                     }
+                    accumulate_brow(cur, acc);
+                    if (!more) break;
+                    cur = nxt;
                 }
             }
         __syncwarp();
