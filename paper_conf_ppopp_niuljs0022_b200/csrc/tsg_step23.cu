@@ -77,9 +77,14 @@ __device__ __forceinline__ void s2_light(const StepParams &P, int64_t t, uint32_
     P.tnzC[t] = total;
 }
 
+__device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+
 __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     __shared__ uint32_t wsm[8 * T2];
-    __shared__ uint32_t sPA[T2 / 16][BATCH], sPB[T2 / 16][BATCH];
+    __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
     const int64_t ngroups = (P.ntC + 31) / 32;
@@ -90,7 +95,8 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
         const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;
         if (light) s2_light(P, t, wsm + threadIdx.x, T2);
         unsigned hm = __ballot_sync(FULL, v && !light);
-        // heavy tiles: two at a time, a half warp each, lane r owns row r
+        // heavy tiles: two at a time, a half warp each, lane r owns row r; per batch of 16 pairs
+        // lane i stages pair i's A and B masks (4 x 16-byte cp.async, all in flight at once)
         while (hm) {
             const int f0 = __ffs(hm) - 1;
             hm &= hm - 1;
@@ -111,17 +117,19 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
                 const uint32_t q = bt * BATCH + r;
                 if (q < np) {
                     const uint64_t pr = pp[q];
-                    const uint32_t pB = (uint32_t)pr;
-                    sPA[hw][r] = (uint32_t)(pr >> 32);
-                    sPB[hw][r] = pB;
+                    const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+                    cp16s(&sMA[hw][r][0], P.mA + pA * TILE);
+                    cp16s(&sMA[hw][r][8], P.mA + pA * TILE + 8);
+                    cp16s(&sMB[hw][r][0], P.mB + pB * TILE);
+                    cp16s(&sMB[hw][r][8], P.mB + pB * TILE + 8);
                     sOB[hw][r] = P.rowOccB[pB];
                 }
+                asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
                 __syncwarp();
                 const uint32_t nb = np > bt * BATCH ? min((uint32_t)BATCH, np - bt * BATCH) : 0u;
                 for (uint32_t i = 0; i < nb; i++) {
-                    const int64_t pA = sPA[hw][i], pB = sPB[hw][i];
-                    uint32_t ma = P.mA[pA * TILE + r] & sOB[hw][i];
-                    const uint16_t *mb = P.mB + pB * TILE;
+                    uint32_t ma = sMA[hw][i][r] & sOB[hw][i];
+                    const uint16_t *mb = sMB[hw][i];
                     while (ma) {
                         const int c = __ffs(ma) - 1;
                         ma &= ma - 1;
