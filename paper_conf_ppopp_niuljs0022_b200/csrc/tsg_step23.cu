@@ -166,13 +166,30 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
 constexpr int WREG = 5632;  // bytes of per-warp shared scratch (small: 4 KB acc + 1.5 KB masks;
                             // medium: 4 KB of row accumulators; dense: 4.2 KB of staged tiles)
 
+struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
+    uint16_t mA[BATCH][TILE], mB[BATCH][TILE];  // cp.async'd masks of A_IK and B_KJ
+    uint16_t mT[BATCH][TILE];                   // transposed A mask (small-tile path)
+    uint8_t rA[BATCH][TILE], rB[BATCH][TILE];   // and their row offsets
+    int64_t zA[BATCH], zB[BATCH];
+    uint16_t oB[BATCH];
+};
+
+__device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_wait_all() {
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+
 // small tile (nnz <= 16): one thread, item driven.  Slot of C(r,j) is row_ptr_C[r] +
 // popc(mask_C[r] & ((1<<j)-1)) (the mask-addressed accumulator); slots, masks and
 // row offsets are thread-private (lane-strided words of the warp's scratch).
-__device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigned char *wr, int lane) {
+__device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigned char *wr, int lane, MedStage &S) {
     double *acc = reinterpret_cast<double *>(wr) + lane;                        // acc[q*32]
     uint32_t *ms = reinterpret_cast<uint32_t *>(wr + SMALL_NNZ * 32 * 8) + lane;  // ms[k*32], k < 8
     uint32_t *rs = ms + 8 * 32;                                                 // rs[k*32], k < 4
+    const int sl = lane & 15;  // this thread's staging slot in its half warp's MedStage
     const int64_t z0 = P.tnzC[t];
     const int nz = (int)(P.tnzC[t + 1] - z0);
     {
@@ -189,25 +206,31 @@ __device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigne
     for (uint32_t p = 0; p < np; p++) {
         const uint64_t pr = pp[p];
         const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+        // the pair's masks, row offsets and transposed A mask: one round of cp.async instead of a
+        // chain of dependent reads
+        cp16(&S.mA[sl][0], P.mA + pA * TILE);
+        cp16(&S.mA[sl][8], P.mA + pA * TILE + 8);
+        cp16(&S.mB[sl][0], P.mB + pB * TILE);
+        cp16(&S.mB[sl][8], P.mB + pB * TILE + 8);
+        cp16(&S.rA[sl][0], P.rpA + pA * TILE);
+        cp16(&S.rB[sl][0], P.rpB + pB * TILE);
+        cp16(&S.mT[sl][0], P.mTA + pA * TILE);
+        cp16(&S.mT[sl][8], P.mTA + pA * TILE + 8);
         uint32_t x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
-        if (!x) continue;
-        const uint16_t *mbt = P.mB + pB * TILE;
-        const uint8_t *rbt = P.rpB + pB * TILE;
-        const uint16_t *mat = P.mA + pA * TILE;
-        const uint8_t *rat = P.rpA + pA * TILE;
-        const uint16_t *att = P.mTA + pA * TILE;
         const double *vbt = P.vB + P.tnzB[pB];
         const double *vat = P.vA + P.tnzA[pA];
+        cp_wait_all();
+        // columns c ascending, rows of A's column c: every slot (r, j) sees ascending c
         while (x) {
             const int c = __ffs(x) - 1;
             x &= x - 1;
-            const uint32_t mbc = mbt[c];
-            const double *vb = vbt + rbt[c];
-            uint32_t rows = att[c];
+            const uint32_t mbc = S.mB[sl][c];
+            const double *vb = vbt + S.rB[sl][c];
+            uint32_t rows = S.mT[sl][c];
             while (rows) {
                 const int r = __ffs(rows) - 1;
                 rows &= rows - 1;
-                const double a = vat[rat[r] + __popc((uint32_t)mat[r] & ((1u << c) - 1u))];
+                const double a = vat[S.rA[sl][r] + __popc((uint32_t)S.mA[sl][r] & ((1u << c) - 1u))];
                 const uint32_t mcr = (ms[(r >> 1) * 32] >> (16 * (r & 1))) & 0xffffu;
                 const int base = (rs[(r >> 2) * 32] >> (8 * (r & 3))) & 0xff;
                 uint32_t mb = mbc;
@@ -232,21 +255,6 @@ __device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigne
             q++;
         }
     }
-}
-
-struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
-    uint16_t mA[BATCH][TILE], mB[BATCH][TILE];  // cp.async'd masks of A_IK and B_KJ
-    uint8_t rA[BATCH][TILE], rB[BATCH][TILE];   // and their row offsets
-    int64_t zA[BATCH], zB[BATCH];
-    uint16_t oB[BATCH];
-};
-
-__device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_wait_all() {
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
 }
 
 // one column c of A's row r in flight: a = A(r,c), B's row c (mask, first 4 values, the rest)
@@ -474,7 +482,7 @@ __global__ void __launch_bounds__(T3) k_s3(StepParams P) {
         const unsigned sm = __ballot_sync(FULL, small);
         const unsigned dm = __ballot_sync(FULL, dense);
         unsigned mm = __ballot_sync(FULL, v) & ~sm & ~dm;
-        if (small) s3_small(P, t, wr, lane);
+        if (small) s3_small(P, t, wr, lane, med[threadIdx.x >> 4]);
         __syncwarp();
         // medium tiles: two at a time, a half warp each
         double *acc = reinterpret_cast<double *>(wr) + half * (TILE * TILE) + r;
