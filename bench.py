@@ -31,6 +31,7 @@ sys.path.insert(0, ROOT)
 METRIC = "fp64 C=A^2 GFLOPS (2×products/time) at 1/2/4/8 B200; % HBM roofline"
 UNIT = "GFLOPS"
 L2_BYTES = 126 * 2 ** 20
+ROW_BLOCKS = {"C5": 4}  # tile-row blocks per step on one GPU (C5's C is ~144 GB in tile form)
 
 
 def peaks():
@@ -175,6 +176,9 @@ def main():
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
     ap.add_argument("--step3-rows", action="store_true", help="step 3 in the whole-tile-row kernel (experimental)")
+    ap.add_argument("--row-blocks", type=int, default=0,
+                    help="compute each rank's C in this many tile-row blocks, one after the other (0 = "
+                         "config default: C5 needs 4 on one GPU, its C alone is ~144 GB in tile form)")
     args = ap.parse_args()
     if args.warmup < 3 and not args.profile:
         args.warmup = 3
@@ -201,29 +205,38 @@ def main():
     stream = torch.cuda.current_stream()
     T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.col).to(dev),
                          torch.from_numpy(A.val).to(dev), (A.m, A.n))
-    # shard C tile rows across ranks (strong scaling of one matrix)
-    if world > 1:
-        from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
+    # shard C tile rows across ranks (strong scaling of one matrix), and within a
+    # rank optionally into row blocks computed one after the other (C does not fit otherwise)
+    K = args.row_blocks or max(1, ROW_BLOCKS.get(args.config, 1) // world)
+    from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
 
-        cuts = tdist.partition_tile_rows(A, A, world)
-        I0, I1 = int(cuts[rank]), int(cuts[rank + 1])
-        Ashard = tsg.slice_rows(T, I0, I1)
-    else:
-        I0, I1 = 0, T.tile_m
-        Ashard = T
+    cuts = tdist.partition_tile_rows(A, A, world * K) if world * K > 1 else np.array([0, T.tile_m])
+    blocks = [(int(cuts[rank * K + b]), int(cuts[rank * K + b + 1])) for b in range(K)]
+    I0, I1 = blocks[0][0], blocks[-1][1]
+    shards = [tsg.slice_rows(T, b0, b1) if (b0, b1) != (0, T.tile_m) else T for b0, b1 in blocks]
+    Ashard = tsg.slice_rows(T, I0, I1) if (I0, I1) != (0, T.tile_m) else T
+
+    def run_blocks(timing=True, products=False, keep=False):
+        """One step: C = A_shard * A block by block; returns summed stats (and C if one block)."""
+        tot, last = {}, None
+        for Ab in shards:
+            C = tsg.spgemm(Ab, T, stats=True, timing=timing, products=products, step3_rows=args.step3_rows)
+            for k, v in C.stats.items():
+                tot[k] = tot.get(k, 0) + v
+            last = C if (keep and len(shards) == 1) else None
+            del C
+        return tot, last
+
     # one instrumented call for the exact counts (products are a property of the input)
-    C0 = tsg.spgemm(Ashard, T, stats=True, products=True)
-    st0 = C0.stats
-    del C0
+    st0, _ = run_blocks(timing=False, products=True)
     small_inputs = tile_bytes(T.tile_m, T.num_tiles, T.nnz) < 2 * L2_BYTES
     flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev) if small_inputs else None
 
     def one_step(timing=True):
-        return tsg.spgemm(Ashard, T, stats=True, timing=timing, step3_rows=args.step3_rows)
+        return run_blocks(timing=timing)[0]
 
     for _ in range(args.warmup):
-        C = one_step()
-        del C
+        one_step()
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -239,18 +252,16 @@ def main():
                 flush.fill_(1)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            C = one_step()
+            st = one_step()
             e1.record(stream)
             e1.synchronize()
             step_ms.append(e0.elapsed_time(e1))
-            st = C.stats
             s1_ms.append(st["ms_step1"] + st["ms_index"])
             s2_ms.append(st["ms_step2"])
             s3_ms.append(st["ms_step3"])
             sa_ms.append(st["ms_alloc"])
             host_ms.append((st["ms_host_sync"], st["ms_host_alloc"]))
             stats_last = st
-            del C
         torch.cuda.synchronize()
         if dist:
             dist.barrier()
@@ -274,9 +285,10 @@ def main():
     steps_ms = {"step1": float(np.mean(s1_ms)), "step2": float(np.mean(s2_ms)), "step3": float(np.mean(s3_ms))}
     alloc_ms = float(np.mean(sa_ms))
     alg = {  # algorithmic bytes per launch of each step's kernels
-        "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + 6 * T.num_tiles + 8 * (T.tile_m + 1) + 12 * ntC,
-        "step2": 32 * (Ashard.num_tiles + T.num_tiles) + 60 * ntC,
-        "step3": 9 * (Ashard.nnz + T.nnz + nnzC) + 48 * (Ashard.num_tiles + T.num_tiles) + 56 * ntC,
+        # (B is read once per row block)
+        "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + K * (6 * T.num_tiles + 8 * (T.tile_m + 1)) + 12 * ntC,
+        "step2": 32 * (Ashard.num_tiles + K * T.num_tiles) + 60 * ntC,
+        "step3": 9 * (Ashard.nnz + K * T.nnz + nnzC) + 48 * (Ashard.num_tiles + K * T.num_tiles) + 56 * ntC,
     }
     dom = max(steps_ms, key=steps_ms.get)
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
@@ -284,7 +296,7 @@ def main():
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(dom)
-    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + tile_bytes(T.tile_m, T.num_tiles, T.nnz) + \
+    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + K * tile_bytes(T.tile_m, T.num_tiles, T.nnz) + \
         tile_bytes(Ashard.tile_m, ntC, nnzC)
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",
             "frac": achieved / bw, "traffic": traffic, "algorithmic_bytes": alg[dom], "peak_source": bw_src,
@@ -296,24 +308,32 @@ def main():
         h_rp = torch.from_numpy(A.rowptr).pin_memory()
         h_ci = torch.from_numpy(A.col).pin_memory()
         h_v = torch.from_numpy(A.val).pin_memory()
-        Cx = one_step(timing=False)
-        bufs = {k: torch.empty(v.numel(), dtype=_host_dtype(v), pin_memory=True) for k, v in Cx.arrays().items()}
-        bo = sum(b.numel() * b.element_size() for b in bufs.values())
+        # host buffers sized for the largest block's C (blocks are copied one after the other)
+        sizes, bo = {}, 0
+        for Ab in shards:
+            Cx = tsg.spgemm(Ab, T)
+            for k, v in Cx.arrays().items():
+                sizes[k] = max(sizes.get(k, 0), v.numel())
+                bo += v.numel() * v.element_size()
+            dts = {k: _host_dtype(v) for k, v in Cx.arrays().items()}
+            del Cx
+        bufs = {k: torch.empty(n, dtype=dts[k], pin_memory=True) for k, n in sizes.items()}
         bi = h_rp.numel() * 8 + h_ci.numel() * 4 + h_v.numel() * 8
-        del Cx
         torch.cuda.synchronize()
         e2e_ms = []
         for _ in range(args.e2e_steps):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             Th = tsg.csr_to_tiles(h_rp, h_ci, h_v, (A.m, A.n))
-            Ah = tsg.slice_rows(Th, I0, I1) if world > 1 else Th
-            Cx = tsg.spgemm(Ah, Th)
-            Cx.copy_to_host(bufs)
+            for b0, b1 in blocks:
+                Ah = tsg.slice_rows(Th, b0, b1) if (b0, b1) != (0, Th.tile_m) else Th
+                Cx = tsg.spgemm(Ah, Th)
+                Cx.copy_to_host(bufs)
+                del Cx, Ah
             e1.record(stream)
             e1.synchronize()
             e2e_ms.append(e0.elapsed_time(e1))
-            del Cx, Ah, Th
+            del Th
         em = float(np.mean(e2e_ms))
         if dist:
             t = torch.tensor([em], dtype=torch.float64, device=dev)
@@ -339,7 +359,8 @@ def main():
         "data": "synthetic",
         "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}", "n": A.m, "nnz_a": A.nnz,
                    "products": prods, "nnz_c": nnzC if world == 1 else None, "tiles_c": ntC if world == 1 else None,
-                   "parallelism": f"tile-row shards x{world}" if world > 1 else "single GPU",
+                   "parallelism": (f"tile-row shards x{world}" if world > 1 else "single GPU") +
+                                  (f", {K} tile-row blocks per rank computed in turn" if K > 1 else ""),
                    "l2": ("512 MB flush between timed steps" if flush is not None else
                           f"inputs larger than L2 (A tiles {tile_bytes(T.tile_m, T.num_tiles, T.nnz) / 1e6:.0f} MB > 126 MB)"),
                    "step_ms": {k: round(v, 4) for k, v in steps_ms.items()}, "alloc_sync_ms": round(alloc_ms, 4),
