@@ -52,13 +52,14 @@ def full(paths):
     for p in paths:
         out = subprocess.run(["ncu", "-i", p, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
         r = list(csv.reader(out.splitlines()))
-        h, u, v = r[0], r[1], r[2]
-        kname = v[h.index("Kernel Name")] if "Kernel Name" in h else p
-        print(f"\n### {p.split('/')[-1]}  ({kname.split('(')[0]})\n\n| metric | value |\n|---|---|")
-        for key, label in KEYS:
-            if key in h:
-                i = h.index(key)
-                print(f"| {label} (`{key}`) | {v[i]} {u[i]} |")
+        h, u = r[0], r[1]
+        for v in r[2:]:
+            kname = v[h.index("Kernel Name")] if "Kernel Name" in h else p
+            print(f"\n### {p.split('/')[-1]}  ({kname.split('(')[0]})\n\n| metric | value |\n|---|---|")
+            for key, label in KEYS:
+                if key in h:
+                    i = h.index(key)
+                    print(f"| {label} (`{key}`) | {v[i]} {u[i]} |")
 
 
 if __name__ == "__main__":
