@@ -306,6 +306,28 @@ __device__ __forceinline__ void accumulate_brow(const BRow &x, double *acc) {
     }
 }
 
+// a lane's position in its flat (pair, c) item sequence of a batch
+struct ItemCursor {
+    uint32_t rel = 0, ma = 0, mAr = 0;
+    int i = 0;
+    const double *va = nullptr, *vbt = nullptr;
+};
+__device__ __forceinline__ bool next_item(const StepParams &P, const MedStage &S, int r, ItemCursor &it, BRow &out) {
+    if (!it.ma) {
+        if (!it.rel) return false;
+        it.i = __ffs(it.rel) - 1;
+        it.rel &= it.rel - 1;
+        it.mAr = S.mA[it.i][r];
+        it.ma = it.mAr & S.oB[it.i];
+        it.va = P.vA + S.zA[it.i] + S.rA[it.i][r];
+        it.vbt = P.vB + S.zB[it.i];
+    }
+    const int c = __ffs(it.ma) - 1;
+    it.ma &= it.ma - 1;
+    out = load_brow(S, it.i, c, it.mAr, it.va, it.vbt);
+    return true;
+}
+
 // medium tile: a half warp, lane r owns C row r; dense-in-j 16-slot row accumulator in shared
 // memory (conflict free), compacted through mask_C[r] at the end.  Pairs go in batches of 16:
 // lane i stages pair i's A and B masks and row offsets (6 x 16-byte cp.async, all lanes and
@@ -346,32 +368,25 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
         cp_wait_all();
         __syncwarp();
         const uint32_t nb = np > bt * BATCH ? min((uint32_t)BATCH, np - bt * BATCH) : 0u;
-        if (mCr)
-            for (uint32_t i = 0; i < nb; i++) {
-                const uint32_t mAr = S.mA[i][r];
-                uint32_t ma = mAr & S.oB[i];
-                if (!ma) continue;
-                const double *va = P.vA + S.zA[i] + S.rA[i][r];
-                const double *vbt = P.vB + S.zB[i];
-                // software pipeline over the columns c of A's row: the loads of column c+1 (its A
-                // value and the first 4 values of B's row c+1) are in flight while column c's
-                // products are accumulated
-                int c = __ffs(ma) - 1;
-                ma &= ma - 1;
-                BRow cur = load_brow(S, i, c, mAr, va, vbt);
-                for (;;) {
-                    const bool more = ma != 0;
-                    BRow nxt;
-                    if (more) {
-                        c = __ffs(ma) - 1;
-                        ma &= ma - 1;
-                        nxt = load_brow(S, i, c, mAr, va, vbt);
-                    }
-                    accumulate_brow(cur, acc);
-                    if (!more) break;
-                    cur = nxt;
-                }
+        if (mCr) {
+            // the batch's pairs that touch row r, then one flat loop over this lane's (pair, c)
+            // items in order (pairs ascending, c ascending): lanes whose rows see different pairs
+            // (e.g. the 1-nonzero corner tiles of stencils touch one row) stay in step, and the
+            // next item's loads are in flight while the current one accumulates
+            uint32_t rel = 0;
+            for (uint32_t i = 0; i < nb; i++) rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
+            ItemCursor it;
+            it.rel = rel;
+            BRow cur;
+            bool have = next_item(P, S, r, it, cur);
+            while (have) {
+                BRow nxt;
+                const bool hn = next_item(P, S, r, it, nxt);
+                accumulate_brow(cur, acc);
+                cur = nxt;
+                have = hn;
             }
+        }
         __syncwarp();
     }
     if (hv && mCr) {
