@@ -30,7 +30,7 @@ constexpr int ROW_T = 256;        // threads of a step-1 row CTA
 constexpr int ROW_NW = ROW_T / 32;
 constexpr int ROW_CAP = 4096;     // max candidates of a row sorted in shared memory
 constexpr int LIGHT_WORK = 16;    // step-2 thread-per-tile class: (pair, c) items of the tile
-constexpr int SMALL_NNZ = 16;     // step-3 thread-per-tile class: C tile nnz
+constexpr int SMALL_NNZ = 8;      // step-3 thread-per-tile class: C tile nnz
 
 // ---------------- a1 row sort
 struct S1Params {

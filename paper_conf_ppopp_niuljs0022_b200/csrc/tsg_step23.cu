@@ -31,7 +31,8 @@ namespace {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int T2 = 256;    // step-2 CTA
 constexpr int T3 = 128;    // step-3 CTA (4 warps; 5.5 KB of shared memory per warp)
-constexpr int BATCH = 16;  // pairs staged per half warp at a time
+constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
+constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
 
 // ==========================================================================================
 // step 2
@@ -163,15 +164,15 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
 // ==========================================================================================
 // step 3
 // ==========================================================================================
-constexpr int WREG = 5632;  // bytes of per-warp shared scratch (small: 4 KB acc + 1.5 KB masks;
+constexpr int WREG = 4224;  // bytes of per-warp shared scratch (small: 4 KB acc + 1.5 KB masks;
                             // medium: 4 KB of row accumulators; dense: 4.2 KB of staged tiles)
 
 struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
-    uint16_t mA[BATCH][TILE], mB[BATCH][TILE];  // cp.async'd masks of A_IK and B_KJ
-    uint16_t mT[BATCH][TILE];                   // transposed A mask (small-tile path)
-    uint8_t rA[BATCH][TILE], rB[BATCH][TILE];   // and their row offsets
-    int64_t zA[BATCH], zB[BATCH];
-    uint16_t oB[BATCH];
+    uint16_t mA[BATCH3][TILE], mB[BATCH3][TILE];  // cp.async'd masks of A_IK and B_KJ
+    uint16_t mT[BATCH3][TILE];                   // transposed A mask (small-tile path)
+    uint8_t rA[BATCH3][TILE], rB[BATCH3][TILE];   // and their row offsets
+    int64_t zA[BATCH3], zB[BATCH3];
+    uint16_t oB[BATCH3];
 };
 
 __device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
@@ -348,11 +349,11 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
             acc[j * 16] = 0.0;
         }
     }
-    const uint32_t nbat = (np + BATCH - 1) / BATCH;
+    const uint32_t nbat = (np + BATCH3 - 1) / BATCH3;
     const uint32_t nbw = max(nbat, __shfl_xor_sync(FULL, nbat, 16));
     for (uint32_t bt = 0; bt < nbw; bt++) {
-        const uint32_t q = bt * BATCH + r;
-        if (q < np) {
+        const uint32_t q = bt * BATCH3 + r;
+        if (r < BATCH3 && q < np) {
             const uint64_t pr = pp[q];
             const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
             cp16(&S.mA[r][0], P.mA + pA * TILE);
@@ -367,7 +368,7 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
         }
         cp_wait_all();
         __syncwarp();
-        const uint32_t nb = np > bt * BATCH ? min((uint32_t)BATCH, np - bt * BATCH) : 0u;
+        const uint32_t nb = np > bt * BATCH3 ? min((uint32_t)BATCH3, np - bt * BATCH3) : 0u;
         if (mCr) {
             // the batch's pairs that touch row r, then one flat loop over this lane's (pair, c)
             // items in order (pairs ascending, c ascending): lanes whose rows see different pairs
@@ -481,7 +482,7 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
     __syncwarp();
 }
 
-__global__ void __launch_bounds__(T3) k_s3(StepParams P) {
+__global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
     __shared__ MedStage med[T3 / 16];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
