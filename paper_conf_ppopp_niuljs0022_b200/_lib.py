@@ -13,7 +13,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TSG_LIBRARY", os.path.join(_HERE, "libtsg.so"))
 
 TILE = 16
-DENSE_NNZ = 192
+DENSE_NNZ = 96  # include/tsg.h TSG_DENSE_NNZ
 
 # flags (include/tsg.h)
 INPUT_HOST = 0x1

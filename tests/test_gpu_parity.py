@@ -147,7 +147,7 @@ def test_spgemm_matches_oracle(tsg, name, A, B):
     assert st["nnz_c"] == d["nnz_c"]
     assert st["pairs"] == d["pairs"]
     assert st["products"] == d["products"]
-    assert st["tiles_dense"] == int((np.diff(ref.tile_nnz) >= 192).sum())
+    assert st["tiles_dense"] == int((np.diff(ref.tile_nnz) >= tsg.DENSE_NNZ).sum())
     # CSR assembly of the result
     rp, ci, v = tsg.tiles_to_csr(C)
     O = oracle.spgemm(A, B, fma=True)
@@ -190,16 +190,18 @@ def test_step3_row_kernel_coverage(tsg):
         assert tsg.spgemm(T, T, stats=True).stats["step3_row_tiles"] == 0
 
 
-def test_threshold_boundary_tiles(tsg):
-    """C tiles with nnz 191, 192, 193 straddle t_nnz = 192."""
+@pytest.mark.parametrize("th", [None, 192])
+def test_threshold_boundary_tiles(tsg, th):
+    """C tiles with nnz t-1, t, t+1 straddle t_nnz (the default, and the paper's 192)."""
     rng = np.random.default_rng(0)
-    for target in (191, 192, 193):
+    t = th or tsg.DENSE_NNZ
+    for target in (t - 1, t, t + 1):
         # C = I16 * B where B is one 16x16 tile with `target` nonzeros -> C tile nnz = target
         cells = rng.choice(256, target, replace=False)
         B = gen.from_coo(16, 16, cells // 16, cells % 16, rng.uniform(-1, 1, target))
         I = gen.identity(16, 1.5)
-        C = tsg.spgemm(tiles_of(tsg, I), tiles_of(tsg, B), stats=True)
-        assert C.stats["tiles_dense"] == (1 if target >= 192 else 0)
+        C = tsg.spgemm(tiles_of(tsg, I), tiles_of(tsg, B), stats=True, dense_threshold=th)
+        assert C.stats["tiles_dense"] == (1 if target >= t else 0)
         ref = oracle.expected_tiles(I, B, fma=True)
         assert_tiles_equal(host(C), ref)
 
