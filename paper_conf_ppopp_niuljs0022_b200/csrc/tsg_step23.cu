@@ -420,11 +420,13 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
     for (int j = 0; j < 8; j++) acc[j] = 0.0;
     const uint64_t *pp = P.pairs + P.pairBeg[t];
     const uint32_t np = P.pairCnt[t];
+    // A is read only at its structural positions (c in mask_A[r]), so it is never cleared; B is
+    // cleared per pair (four 16-byte stores per lane) and its nonzeros scattered over it
     for (uint32_t p = 0; p < np; p++) {
         const uint64_t pr = pp[p];
         const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-        for (int e = lane; e < TILE * AP; e += 32) Ad[e] = 0.0;
-        for (int e = lane; e < TILE * TILE; e += 32) Bd[e] = 0.0;
+#pragma unroll
+        for (int e = lane; e < TILE * TILE / 2; e += 32) reinterpret_cast<double2 *>(Bd)[e] = make_double2(0.0, 0.0);
         __syncwarp();
         bool nf = false;
         for (int64_t e = P.tnzA[pA] + lane; e < P.tnzA[pA + 1]; e += 32) {
