@@ -167,6 +167,17 @@ TSG_API tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t f
 TSG_API tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *stream,
                             int64_t **row_ptr, int32_t **col_idx, double **val, int64_t *nnz);
 
+/*
+ * tsg_tiles_transpose -- A^T in sparse-tile form, for the paper's second workload C = A*A^T
+ * (SURVEY §8(f) f1): tile (I, J) becomes tile (J, I) with its pattern and
+ * values transposed.  Exact (a permutation of T's data); stream-ordered on `stream`, no host sync.
+ *   T       input handle (borrowed; m < 2^31 so that A^T's column ids fit int32)
+ *   al      allocator for the result's arrays (NULL = cudaMallocAsync)
+ *   out     receives a new handle (destroy with tsg_tiles_destroy)
+ * Errors: INVALID_ARG (NULL, unaligned mask), OVERFLOW, OOM, CUDA.
+ */
+TSG_API tsg_status tsg_tiles_transpose(const tsg_tiles *T, const tsg_allocator *al, void *stream, tsg_tiles **out);
+
 /* Fill *out with the handle's arrays and sizes (pointers stay owned by the handle). */
 TSG_API tsg_status tsg_tiles_get_view(const tsg_tiles *T, tsg_tiles_view *out);
 

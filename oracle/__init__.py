@@ -8,7 +8,7 @@ A thin ctypes/numpy layer over ``oracle/tsg_oracle.c`` (plain single-threaded C,
 ``-O2 -ffp-contract=off``).  See the C file for the per-function citations into PAPER.md.
 
 Parity status: O1 (Gustavson), O2/O3 (tile format), O4 (C' and Algorithm-2 masks), O5
-(products) are all pinned by tests/test_oracle_pins.py (closed forms, brute force, invariants,
+(products), O6 (CSR transpose, for C = A*A^T) are all pinned by tests/test_oracle_pins.py (closed forms, brute force, invariants,
 the paper's Fig 5 mask fact, and two-formulation cross-checks).  Nothing here is "parity
 unpinned".
 """
@@ -130,6 +130,32 @@ class OracleTiles:
 def products(A, B) -> int:
     """O5: number of intermediate products of A*B (Table 2 caption)."""
     return int(lib().orc_products(A.m, _arr(A.rowptr, np.int64), _arr(A.col, np.int32), _arr(B.rowptr, np.int64)))
+
+
+def transpose(A) -> OracleCSR:
+    """O6: A^T in CSR for the paper's second workload C = A*A^T.
+
+    The definition written out: entry (i, j, v) of A becomes (j, i, v); rows of A^T are filled by
+    walking A's rows in ascending i, so every row of A^T lists its columns ascending (a stable
+    counting sort by column)."""
+    rowptr = np.asarray(A.rowptr, np.int64)
+    col = np.asarray(A.col, np.int64)
+    val = np.asarray(A.val, np.float64)
+    nnz = int(rowptr[-1]) if rowptr.size else 0
+    counts = np.zeros(A.n + 1, np.int64)
+    for j in col[:nnz]:
+        counts[j + 1] += 1
+    rpT = np.cumsum(counts)
+    cur = rpT[:-1].copy()
+    colT = np.empty(nnz, np.int32)
+    valT = np.empty(nnz, np.float64)
+    for i in range(A.m):
+        for p in range(rowptr[i], rowptr[i + 1]):
+            j = col[p]
+            colT[cur[j]] = i
+            valT[cur[j]] = val[p]
+            cur[j] += 1
+    return OracleCSR(A.n, A.m, rpT, colT, valT)
 
 
 def spgemm(A, B, fma: bool = False, rows=None) -> OracleCSR:

@@ -23,7 +23,7 @@ from . import _lib
 from ._lib import TILE, DENSE_NNZ, TsgError  # noqa: F401
 
 __all__ = ["Tiles", "csr_to_tiles", "spgemm", "tiles_to_csr", "slice_rows", "wrap", "TsgError",
-           "kernel_launch_count", "workspace_release"]
+           "kernel_launch_count", "workspace_release", "transpose"]
 
 _DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8)}
 
@@ -199,6 +199,13 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
                       C.byref(st) if st is not None else None)
     _lib.check(rc)
     return _from_handle(out.value, st.as_dict() if st is not None else None)
+
+
+def transpose(T: Tiles, stream=None) -> Tiles:
+    """A^T in the sparse-tile format (tsg_tiles_transpose), e.g. for C = A * A^T."""
+    out = C.c_void_p()
+    _lib.check(_lib.load().tsg_tiles_transpose(T.ptr, None, C.c_void_p(_stream_ptr(stream)), C.byref(out)))
+    return _from_handle(out.value)
 
 
 def tiles_to_csr(T: Tiles, stream=None):

@@ -66,7 +66,7 @@ class Allocator(C.Structure):
 SYMBOLS = ["tsg_csr_to_tiles", "tsg_spgemm", "tsg_tiles_to_csr", "tsg_tiles_get_view", "tsg_tiles_wrap",
            "tsg_tiles_slice_rows", "tsg_tiles_copy_to_host", "tsg_tiles_destroy", "tsg_free",
            "tsg_status_string", "tsg_last_error", "tsg_abi_version", "tsg_kernel_launch_count",
-           "tsg_workspace_release"]
+           "tsg_workspace_release", "tsg_tiles_transpose"]
 
 _lib = None
 
@@ -106,6 +106,8 @@ def load():
     L.tsg_last_error.argtypes = []
     L.tsg_abi_version.restype = C.c_int
     L.tsg_kernel_launch_count.restype = i64
+    L.tsg_tiles_transpose.restype = C.c_int
+    L.tsg_tiles_transpose.argtypes = [vp, vp, vp, pp]
     L.tsg_workspace_release.restype = C.c_size_t
     L.tsg_workspace_release.argtypes = [vp]
     _lib = L

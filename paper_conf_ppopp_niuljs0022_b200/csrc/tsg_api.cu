@@ -240,6 +240,26 @@ tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, co
     });
 }
 
+tsg_status tsg_tiles_transpose(const tsg_tiles *T, const tsg_allocator *al, void *stream, tsg_tiles **out) {
+    if (out) *out = nullptr;
+    return guarded([&] {
+        TSG_REQUIRE(T && out, TSG_ERR_INVALID_ARG, "NULL argument");
+        TSG_REQUIRE(T->m < ((int64_t)1 << 31), TSG_ERR_OVERFLOW, "A^T would have >= 2^31 columns");
+        TSG_REQUIRE(((uintptr_t)T->mask & 15) == 0, TSG_ERR_INVALID_ARG, "mask must be 16-byte aligned");
+        cudaStream_t s = (cudaStream_t)stream;
+        Allocator A = Allocator::from(al);
+        tsg_tiles *O = new tsg_tiles();
+        O->al = A;
+        try {
+            launch_transpose_tiles(T, A, s, O);
+        } catch (...) {
+            destroy_handle(O, s);
+            throw;
+        }
+        *out = O;
+    });
+}
+
 tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *stream, int64_t **row_ptr,
                             int32_t **col_idx, double **val, int64_t *nnz) {
     if (row_ptr) *row_ptr = nullptr;

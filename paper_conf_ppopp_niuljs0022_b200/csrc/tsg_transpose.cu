@@ -1,0 +1,151 @@
+// tsg_transpose.cu -- tile-level transpose of a sparse-tile matrix, for the paper's second
+// workload C = A*A^T (Fig 8).
+//
+// Tile (I, J) of A becomes tile (J, I) of A^T with its 16x16 pattern transposed: the new row
+// masks are A's column masks, the new row offsets their prefix popcounts, and the values are
+// re-ordered from A's row-major (r, c) order to (c, r) order.  Steps:
+//   1. tiles per tile column J of A (atomic counts) -> scan -> tile_ptr of A^T
+//   2. each tile row I drops its tiles into their column's slot range (atomic cursor per column)
+//   3. a warp per column ranks its slots by I (tile rows are unique within a column), which
+//      gives the ascending-I order of A^T's tile row J without a global sort
+//   4. nnz offsets of A^T (scan), then a thread per tile writes the transposed tile.
+// Exact (a permutation of A's data): compared bit for bit with the oracle's CSR transpose.
+#include "tsg_kernels.cuh"
+
+namespace tsg {
+namespace {
+
+__global__ void k_tp_count(int64_t nt, const int32_t *__restrict__ tcol, unsigned long long *__restrict__ cnt) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < nt) atomicAdd(&cnt[tcol[t]], 1ULL);
+}
+
+// warp per tile row I of A: its tiles go to their column's slot range (any order)
+__global__ void k_tp_place(int64_t tm, const int64_t *__restrict__ tp, const int32_t *__restrict__ tcol,
+                           unsigned long long *__restrict__ cursor, int32_t *__restrict__ slotI,
+                           int64_t *__restrict__ slotSrc) {
+    const int lane = threadIdx.x & 31;
+    const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (I >= tm) return;
+    for (int64_t t = tp[I] + lane; t < tp[I + 1]; t += 32) {
+        const int64_t s = (int64_t)atomicAdd(&cursor[tcol[t]], 1ULL);
+        slotI[s] = (int32_t)I;
+        slotSrc[s] = t;
+    }
+}
+
+// warp per tile column J: rank each slot by its tile row I -> A^T's tile (J, I) in ascending I
+__global__ void k_tp_rank(int64_t tn, const int64_t *__restrict__ tpT, const int32_t *__restrict__ slotI,
+                          const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
+                          int32_t *__restrict__ tcolT) {
+    const int lane = threadIdx.x & 31;
+    const int64_t J = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (J >= tn) return;
+    const int64_t b = tpT[J], e = tpT[J + 1];
+    for (int64_t s = b + lane; s < e; s += 32) {
+        const int32_t I = slotI[s];
+        int64_t rank = 0;
+        for (int64_t s2 = b; s2 < e; s2++) rank += slotI[s2] < I;
+        perm[b + rank] = slotSrc[s];
+        tcolT[b + rank] = I;
+    }
+}
+
+__global__ void k_tp_nnz(int64_t nt, const int64_t *__restrict__ perm, const int64_t *__restrict__ tnz,
+                         int64_t *__restrict__ tnzT) {
+    const int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (d < nt) tnzT[d] = tnz[perm[d] + 1] - tnz[perm[d]];
+}
+
+// thread per tile of A^T: transpose source tile perm[d] (whose column masks are maskTs)
+__global__ void k_tp_fill(int64_t nt, const int64_t *__restrict__ perm, const int64_t *__restrict__ tnz,
+                          const uint16_t *__restrict__ mask, const uint16_t *__restrict__ maskTs,
+                          const double *__restrict__ val, const int64_t *__restrict__ tnzT,
+                          uint8_t *__restrict__ rpT, uint16_t *__restrict__ maskT, uint8_t *__restrict__ idxT,
+                          double *__restrict__ valT) {
+    const int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (d >= nt) return;
+    const int64_t t = perm[d];
+    const uint4 *pc = reinterpret_cast<const uint4 *>(maskTs + t * TILE);
+    const uint4 c0 = pc[0], c1 = pc[1];
+    reinterpret_cast<uint4 *>(maskT + d * TILE)[0] = c0;
+    reinterpret_cast<uint4 *>(maskT + d * TILE)[1] = c1;
+    const uint32_t cw[8] = {c0.x, c0.y, c0.z, c0.w, c1.x, c1.y, c1.z, c1.w};
+    uint32_t rpw[4] = {0, 0, 0, 0};
+    int offs[TILE];
+    int run = 0;
+#pragma unroll
+    for (int c = 0; c < TILE; c++) {
+        offs[c] = run;
+        rpw[c >> 2] |= (uint32_t)run << (8 * (c & 3));
+        run += __popc((cw[c >> 1] >> (16 * (c & 1))) & 0xffffu);
+    }
+    *reinterpret_cast<uint4 *>(rpT + d * TILE) = make_uint4(rpw[0], rpw[1], rpw[2], rpw[3]);
+    // source entries in row-major (r, c) order; entry (r, c) lands in A^T's row c at rank of r
+    int64_t z = tnz[t];
+    const int64_t zT = tnzT[d];
+    for (int r = 0; r < TILE; r++) {
+        uint32_t m = mask[t * TILE + r];
+        while (m) {
+            const int c = __ffs(m) - 1;
+            m &= m - 1;
+            const uint32_t col = (cw[c >> 1] >> (16 * (c & 1))) & 0xffffu;  // rows r' of source column c
+            const int pos = offs[c] + __popc(col & ((1u << r) - 1u));
+            valT[zT + pos] = val[z];
+            idxT[zT + pos] = (uint8_t)((c << 4) | r);
+            z++;
+        }
+    }
+}
+
+}  // namespace
+
+void launch_transpose_tiles(const tsg_tiles *T, const Allocator &al, cudaStream_t s, tsg_tiles *O) {
+    Buffers tmp(al, s, true), out(al, s);
+    const int64_t nt = T->nt, tmT = T->tn, tnT = T->tm;
+    unsigned long long *cnt = tmp.get<unsigned long long>(tmT + 1);
+    TSG_CUDA(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (tmT + 1), s));
+    TSG_LAUNCH(k_tp_count, grid_for(nt, 256), 256, 0, s, nt, T->tile_col, cnt);
+    int64_t *tpT = out.get<int64_t>(tmT + 1);
+    exclusive_scan<int64_t>(reinterpret_cast<const int64_t *>(cnt), tpT, tmT, s, tmp);
+    unsigned long long *cursor = tmp.get<unsigned long long>(tmT + 1);
+    TSG_CUDA(cudaMemcpyAsync(cursor, tpT, sizeof(int64_t) * (tmT + 1), cudaMemcpyDeviceToDevice, s));
+    int32_t *slotI = tmp.get<int32_t>(nt);
+    int64_t *slotSrc = tmp.get<int64_t>(nt);
+    TSG_LAUNCH(k_tp_place, grid_for(T->tm, 8), 256, 0, s, T->tm, T->tile_ptr, T->tile_col, cursor, slotI, slotSrc);
+    int64_t *perm = tmp.get<int64_t>(nt);
+    int32_t *tcolT = out.get<int32_t>(nt);
+    TSG_LAUNCH(k_tp_rank, grid_for(tmT, 8), 256, 0, s, tmT, tpT, slotI, slotSrc, perm, tcolT);
+    int64_t *tnzT = out.get<int64_t>(nt + 1);
+    TSG_LAUNCH(k_tp_nnz, grid_for(nt, 256), 256, 0, s, nt, perm, T->tile_nnz, tnzT);
+    exclusive_scan<int64_t>(tnzT, tnzT, nt, s, tmp);
+    uint16_t *mTs = tmp.get<uint16_t>(TILE * nt);
+    launch_transpose(T->mask, nt, mTs, s);
+    uint8_t *rpT = out.get<uint8_t>(TILE * nt);
+    uint16_t *maskT = out.get<uint16_t>(TILE * nt);
+    uint8_t *idxT = out.get<uint8_t>(T->nnz);
+    double *valT = out.get<double>(T->nnz);
+    TSG_LAUNCH(k_tp_fill, grid_for(nt, 128), 128, 0, s, nt, perm, T->tile_nnz, T->mask, mTs, T->val, tnzT, rpT, maskT,
+               idxT, valT);
+    O->m = T->n;
+    O->n = T->m;
+    O->tm = tmT;
+    O->tn = tnT;
+    O->nt = nt;
+    O->nnz = T->nnz;
+    O->tile_ptr = tpT;
+    O->tile_col = tcolT;
+    O->tile_nnz = tnzT;
+    O->row_ptr = rpT;
+    O->mask = maskT;
+    O->idx = idxT;
+    O->val = valT;
+    void *arr[7] = {tpT, tcolT, tnzT, rpT, maskT, idxT, valT};
+    for (int k = 0; k < 7; k++) {
+        O->bytes[k] = out.take(arr[k]);
+        O->owns[k] = true;
+    }
+    O->al = al;
+}
+
+}  // namespace tsg

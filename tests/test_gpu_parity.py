@@ -325,3 +325,38 @@ def test_full_size_sampled_rows(tsg, cfg):
         s0, s1 = int(sub.rowptr[t]), int(sub.rowptr[t + 1])
         assert np.array_equal(cci[b:e].cpu().numpy(), sub.col[s0:s1]), i
         assert bitwise_equal_values(cv[b:e].cpu().numpy(), sub.val[s0:s1]), i
+
+
+# ------------------------------------------------------------------------------------------
+# tile transpose and C = A * A^T (the paper's second workload)
+# ------------------------------------------------------------------------------------------
+TRANSPOSE_CASES = [
+    ("rect", gen.random_sparse(37, 50, 0.08, 1)),
+    ("ragged", gen.random_sparse(100, 115, 0.03, 3)),
+    ("rmat-11", gen.rmat(11)),
+    ("hub", gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)),
+    ("C1", gen.config("C1")),
+    ("empty", gen.random_sparse(40, 24, 0.0, 1)),
+    ("single", gen.from_coo(20, 33, [7], [31], [2.5])),
+]
+
+
+@pytest.mark.parametrize("name,A", TRANSPOSE_CASES, ids=[c[0] for c in TRANSPOSE_CASES])
+def test_transpose_bitwise(tsg, name, A):
+    T = tiles_of(tsg, A)
+    At = tsg.transpose(T)
+    assert (At.m, At.n) == (A.n, A.m)
+    assert_tiles_equal(host(At), oracle.csr_to_tiles(oracle.transpose(A)))
+    Att = tsg.transpose(At)
+    assert_tiles_equal(host(Att), oracle.csr_to_tiles(A))
+
+
+@pytest.mark.parametrize("name,A", [c for c in TRANSPOSE_CASES if c[0] in ("rect", "ragged", "rmat-11", "C1")],
+                         ids=["rect", "ragged", "rmat-11", "C1"])
+def test_aat_matches_oracle(tsg, name, A):
+    T = tiles_of(tsg, A)
+    C = tsg.spgemm(T, tsg.transpose(T), stats=True, products=True)
+    At = oracle.transpose(A)
+    ref = oracle.expected_tiles(A, At, fma=True)
+    assert_tiles_equal(host(C), ref)
+    assert C.stats["products"] == oracle.products(A, At)

@@ -339,3 +339,37 @@ def test_generators_deterministic_and_chunk_independent():
     for i in range(A.m):
         seg = A.col[A.rowptr[i]:A.rowptr[i + 1]]
         assert np.all(np.diff(seg) > 0)
+
+
+# ------------------------------------------------------------------------------------------
+# O6: CSR transpose (for the paper's second workload C = A*A^T)
+# ------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("m,n,d", [(1, 1, 1.0), (37, 50, 0.1), (64, 17, 0.3), (100, 100, 0.02), (20, 30, 0.0)])
+def test_transpose_matches_dense_and_scipy(m, n, d):
+    A = gen.random_sparse(m, n, d, seed=m * 7 + n)
+    T = oracle.transpose(A)
+    assert (T.m, T.n) == (n, m)
+    # dense brute force: every entry lands at the mirrored position
+    assert np.array_equal(csr_dense(T.m, T.n, T.rowptr, T.col, T.val), csr_dense(A.m, A.n, A.rowptr, A.col, A.val).T)
+    # rows of A^T list columns ascending, values carried bitwise (scipy's CSC view of A)
+    S = sp.csr_matrix((A.val, A.col, A.rowptr), shape=(m, n)).tocsc()
+    S.sort_indices()
+    assert np.array_equal(T.rowptr, S.indptr) and np.array_equal(T.col, S.indices)
+    assert bitwise_equal_values(T.val, S.data)
+
+
+def test_transpose_involution_and_product_rule():
+    A = gen.random_sparse(48, 40, 0.08, seed=5)
+    B = gen.random_sparse(40, 33, 0.1, seed=6)
+    TT = oracle.transpose(oracle.transpose(A))
+    assert np.array_equal(TT.rowptr, A.rowptr) and np.array_equal(TT.col, A.col) and bitwise_equal_values(TT.val, A.val)
+    # (A B)^T = B^T A^T: same structure; values agree within the sum-of-|products| bound
+    L = oracle.transpose(oracle.spgemm(A, B))
+    R = oracle.spgemm(oracle.transpose(B), oracle.transpose(A))
+    assert np.array_equal(L.rowptr, R.rowptr) and np.array_equal(L.col, R.col)
+    assert np.allclose(L.val, R.val, rtol=0, atol=1e-12 * np.abs(R.val).max())
+    # A A^T is symmetric for any A (structure exactly; values are the same dot products)
+    Q = oracle.spgemm(A, oracle.transpose(A))
+    QT = oracle.transpose(Q)
+    assert np.array_equal(Q.rowptr, QT.rowptr) and np.array_equal(Q.col, QT.col)
+    assert np.allclose(Q.val, QT.val, rtol=0, atol=1e-12 * np.abs(Q.val).max())
