@@ -103,16 +103,17 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def oracle_baseline(A, budget_s: float = 12.0, max_rows=None):
-    """The oracle as it stands (single thread) on a bounded row sample of A*A."""
+def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None):
+    """The oracle as it stands (single thread) on a bounded row sample of A*B (B = A by default)."""
     import oracle
 
     oracle.build()
+    B = A if B is None else B
     m = A.m
     # calibrate on a small row block, then size the sample to ~budget_s seconds
     probe = np.arange(0, min(m, 256), dtype=np.int64)
     t0 = time.perf_counter()
-    oracle.spgemm(A, A, rows=probe)
+    oracle.spgemm(A, B, rows=probe)
     dt = max(time.perf_counter() - t0, 1e-4)
     rows_per_s = len(probe) / dt
     R = int(min(m, max(len(probe), rows_per_s * budget_s)))
@@ -120,9 +121,9 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None):
         R = min(R, max_rows)
     rows = np.arange(0, R, dtype=np.int64)
     sub = gen_row_block(A, R)
-    prods = oracle.products(sub, A)
+    prods = oracle.products(sub, B)
     t0 = time.perf_counter()
-    C = oracle.spgemm(A, A, rows=rows)
+    C = oracle.spgemm(A, B, rows=rows)
     el = time.perf_counter() - t0
     return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
@@ -143,20 +144,22 @@ def run_reference(args):
     from workloads import gen
 
     A = gen.config(args.config)
+    B = _csr_transpose(A) if args.aat else A
     for _ in range(args.warmup):
-        oracle_baseline(A, budget_s=2.0)
+        oracle_baseline(A, budget_s=2.0, B=B)
     vals, secs, prods = [], 0.0, 0
     last = None
     for _ in range(args.steps):
-        last = oracle_baseline(A, budget_s=args.ref_step_s)
+        last = oracle_baseline(A, budget_s=args.ref_step_s, B=B)
         vals.append(last["value"])
         secs += last["seconds"]
         prods += last["products"]
     value = 2.0 * prods / secs / 1e9
-    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+    line = {"impl": "reference", "metric": _metric(args), "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}", "n": A.m, "nnz_a": A.nnz},
+            "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}" + (", C = A*A^T" if args.aat else ""),
+                       "n": A.m, "nnz_a": A.nnz},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": last["sample"]},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -176,6 +179,9 @@ def main():
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
     ap.add_argument("--step3-rows", action="store_true", help="step 3 in the whole-tile-row kernel (experimental)")
+    ap.add_argument("--aat", action="store_true",
+                    help="C = A * A^T (the paper's second workload, SURVEY f1); A^T is formed once with "
+                         "tsg_tiles_transpose outside the timed region, like the CSR->tile conversion")
     ap.add_argument("--row-blocks", type=int, default=0,
                     help="compute each rank's C in this many tile-row blocks, one after the other (0 = "
                          "config default: C5 needs 4 on one GPU, its C alone is ~144 GB in tile form)")
@@ -205,12 +211,15 @@ def main():
     stream = torch.cuda.current_stream()
     T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.col).to(dev),
                          torch.from_numpy(A.val).to(dev), (A.m, A.n))
+    # the right operand: A itself (C = A^2, BASELINE's metric) or A^T (C = A A^T)
+    Bt = tsg.transpose(T) if args.aat else T
+    Bcsr = _csr_transpose(A) if args.aat else A
     # shard C tile rows across ranks (strong scaling of one matrix), and within a
     # rank optionally into row blocks computed one after the other (C does not fit otherwise)
     K = args.row_blocks or max(1, ROW_BLOCKS.get(args.config, 1) // world)
     from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
 
-    cuts = tdist.partition_tile_rows(A, A, world * K) if world * K > 1 else np.array([0, T.tile_m])
+    cuts = tdist.partition_tile_rows(A, Bcsr, world * K) if world * K > 1 else np.array([0, T.tile_m])
     blocks = [(int(cuts[rank * K + b]), int(cuts[rank * K + b + 1])) for b in range(K)]
     I0, I1 = blocks[0][0], blocks[-1][1]
     shards = [tsg.slice_rows(T, b0, b1) if (b0, b1) != (0, T.tile_m) else T for b0, b1 in blocks]
@@ -220,7 +229,7 @@ def main():
         """One step: C = A_shard * A block by block; returns summed stats (and C if one block)."""
         tot, last = {}, None
         for Ab in shards:
-            C = tsg.spgemm(Ab, T, stats=True, timing=timing, products=products, step3_rows=args.step3_rows)
+            C = tsg.spgemm(Ab, Bt, stats=True, timing=timing, products=products, step3_rows=args.step3_rows)
             for k, v in C.stats.items():
                 tot[k] = tot.get(k, 0) + v
             last = C if (keep and len(shards) == 1) else None
@@ -286,9 +295,9 @@ def main():
     alloc_ms = float(np.mean(sa_ms))
     alg = {  # algorithmic bytes per launch of each step's kernels
         # (B is read once per row block)
-        "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + K * (6 * T.num_tiles + 8 * (T.tile_m + 1)) + 12 * ntC,
-        "step2": 32 * (Ashard.num_tiles + K * T.num_tiles) + 60 * ntC,
-        "step3": 9 * (Ashard.nnz + K * T.nnz + nnzC) + 48 * (Ashard.num_tiles + K * T.num_tiles) + 56 * ntC,
+        "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + K * (6 * Bt.num_tiles + 8 * (Bt.tile_m + 1)) + 12 * ntC,
+        "step2": 32 * (Ashard.num_tiles + K * Bt.num_tiles) + 60 * ntC,
+        "step3": 9 * (Ashard.nnz + K * Bt.nnz + nnzC) + 48 * (Ashard.num_tiles + K * Bt.num_tiles) + 56 * ntC,
     }
     dom = max(steps_ms, key=steps_ms.get)
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
@@ -296,7 +305,7 @@ def main():
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(dom)
-    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + K * tile_bytes(T.tile_m, T.num_tiles, T.nnz) + \
+    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + K * tile_bytes(Bt.tile_m, Bt.num_tiles, Bt.nnz) + \
         tile_bytes(Ashard.tile_m, ntC, nnzC)
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",
             "frac": achieved / bw, "traffic": traffic, "algorithmic_bytes": alg[dom], "peak_source": bw_src,
@@ -311,7 +320,7 @@ def main():
         # host buffers sized for the largest block's C (blocks are copied one after the other)
         sizes, bo = {}, 0
         for Ab in shards:
-            Cx = tsg.spgemm(Ab, T)
+            Cx = tsg.spgemm(Ab, Bt)
             for k, v in Cx.arrays().items():
                 sizes[k] = max(sizes.get(k, 0), v.numel())
                 bo += v.numel() * v.element_size()
@@ -325,15 +334,16 @@ def main():
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             Th = tsg.csr_to_tiles(h_rp, h_ci, h_v, (A.m, A.n))
+            Bh = tsg.transpose(Th) if args.aat else Th
             for b0, b1 in blocks:
                 Ah = tsg.slice_rows(Th, b0, b1) if (b0, b1) != (0, Th.tile_m) else Th
-                Cx = tsg.spgemm(Ah, Th)
+                Cx = tsg.spgemm(Ah, Bh)
                 Cx.copy_to_host(bufs)
                 del Cx, Ah
             e1.record(stream)
             e1.synchronize()
             e2e_ms.append(e0.elapsed_time(e1))
-            del Th
+            del Th, Bh
         em = float(np.mean(e2e_ms))
         if dist:
             t = torch.tensor([em], dtype=torch.float64, device=dev)
@@ -349,15 +359,16 @@ def main():
         return 0
     cpu = None
     if not args.no_cpu_baseline and not args.profile and world == 1:
-        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s)
+        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr)
         cpu.pop("seconds", None)
         cpu.pop("products", None)
     clocks = clk.summary() if not args.profile else None
     line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "metric": _metric(args), "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
-        "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}", "n": A.m, "nnz_a": A.nnz,
+        "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}" + (", C = A*A^T" if args.aat else ""),
+                   "n": A.m, "nnz_a": A.nnz,
                    "products": prods, "nnz_c": nnzC if world == 1 else None, "tiles_c": ntC if world == 1 else None,
                    "parallelism": (f"tile-row shards x{world}" if world > 1 else "single GPU") +
                                   (f", {K} tile-row blocks per rank computed in turn" if K > 1 else ""),
@@ -378,6 +389,22 @@ def main():
     if dist:
         dist.destroy_process_group()
     return 0
+
+
+def _metric(args):
+    return METRIC.replace("C=A^2", "C=A*A^T") if args.aat else METRIC
+
+
+def _csr_transpose(A):
+    """Host CSR of A^T (only for the row-partition weights of C = A A^T; the product uses the
+    library's tile transpose)."""
+    from workloads.gen import CSR
+
+    rows = np.repeat(np.arange(A.m, dtype=np.int64), np.diff(A.rowptr))
+    order = np.lexsort((rows, A.col))
+    rp = np.zeros(A.n + 1, np.int64)
+    np.add.at(rp, A.col.astype(np.int64) + 1, 1)
+    return CSR(A.n, A.m, np.cumsum(rp), rows[order].astype(np.int32), A.val[order])
 
 
 def _host_dtype(t):
