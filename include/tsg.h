@@ -106,6 +106,7 @@ typedef struct {
     float ms_host_sync, ms_host_alloc; /* host wall time blocked in scalar reads / allocation calls */
     int64_t step3_row_tiles;  /* C tiles whose step 3 ran in the whole-tile-row kernel */
     int64_t step3_rows;       /* tile rows handled by that kernel */
+    int64_t step1_merge_rows; /* tile rows whose step 1 ran as a warp k-way merge (<= 32 A tiles) */
 } tsg_stats;
 
 /* flags for tsg_csr_to_tiles */
@@ -119,6 +120,7 @@ typedef struct {
 #define TSG_STEP1_LIST_ALWAYS 0x8u/* build B-row lists and use them wherever they are cheaper */
 #define TSG_STATS_PRODUCTS 0x10u  /* also count intermediate products into stats->products */
 #define TSG_STEP3_ROWS 0x20u      /* step 3 in the whole-tile-row kernel where rows fit (experimental; same results) */
+#define TSG_STEP1_SORT_ONLY 0x40u /* step 1: no warp merge; every tile row expands + radix-sorts (same results) */
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = TSG_DENSE_NNZ; 257 disables dense) */
 
 /*

@@ -24,6 +24,7 @@ STEP1_SCAN_ONLY = 0x4
 STEP1_LIST_ALWAYS = 0x8
 STATS_PRODUCTS = 0x10
 STEP3_ROWS = 0x20
+STEP1_SORT_ONLY = 0x40
 DENSE_THRESHOLD_SHIFT = 16
 
 STATUS = {0: "TSG_OK", 1: "TSG_ERR_INVALID_ARG", 2: "TSG_ERR_SHAPE", 3: "TSG_ERR_UNSORTED",
@@ -52,7 +53,8 @@ class Stats(C.Structure):
                 ("ms_index", C.c_float), ("ms_step1", C.c_float), ("ms_step2", C.c_float),
                 ("ms_alloc", C.c_float), ("ms_step3", C.c_float), ("ms_total", C.c_float),
                 ("ms_host_sync", C.c_float), ("ms_host_alloc", C.c_float),
-                ("step3_row_tiles", C.c_int64), ("step3_rows", C.c_int64)]
+                ("step3_row_tiles", C.c_int64), ("step3_rows", C.c_int64),
+                ("step1_merge_rows", C.c_int64)]
 
     def as_dict(self) -> dict:
         return {f[0]: getattr(self, f[0]) for f in self._fields_}

@@ -24,13 +24,15 @@ struct DevCounters {
     u64c n3rows;       // tile rows handled by the row kernel of step 3
     u64c n3fallback;   // C tiles left to the per-tile kernel of step 3
     u64c next3;        // work counter of the step-3 row kernel
+    u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
 };
 
 constexpr int ROW_T = 256;        // threads of a step-1 row CTA
 constexpr int ROW_NW = ROW_T / 32;
 constexpr int ROW_CAP = 4096;     // max candidates of a row sorted in shared memory
 constexpr int LIGHT_WORK = 16;    // step-2 thread-per-tile class: (pair, c) items of the tile
-constexpr int SMALL_NNZ = 8;      // step-3 thread-per-tile class: C tile nnz
+constexpr int SMALL_NNZ = 8;      // step-3 lane-per-entry class (k_s3_small): C tile nnz (<= 16)
+constexpr int MERGE_MAX_A = 32;   // step-1 warp-merge class: A tiles of the tile row (one lane each)
 
 // ---------------- a1 row sort
 struct S1Params {
@@ -45,6 +47,7 @@ struct S1Params {
     const int32_t *rowJlo;
     const int32_t *rowJhi;
     const uint8_t *rowClass;
+    int64_t tnB;       // tile columns of B (the merge packs a tile column into 27 bits)
     uint64_t *pairs;   // [Utot]  (posA << 32) | posB, at costOff[a0] + i
     int32_t *tJ;       // [Utot]  C tile column of rank r, at costOff[a0] + r
     uint32_t *tStart;  // [Utot]  first pair (row-relative)
@@ -93,6 +96,7 @@ struct StepParams {
     const uint8_t *rpB;
     const uint16_t *mB;
     const uint16_t *rowOccB;
+    const uint16_t *mTB;      // transposed masks (column j of B_KJ: bit c <=> B(c,j) != 0)
     const uint8_t *ixB;
     const double *vB;
     // C
@@ -104,6 +108,7 @@ struct StepParams {
     const uint32_t *work;  // step-2 class split
     const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
     int dense_threshold;
+    int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     DevCounters *cnt;
 };
 
@@ -154,9 +159,10 @@ void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA,
                        const int32_t *tcB, const int64_t *lptr, const uint32_t *list, bool scan_only, int64_t *cost,
                        int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s);
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
-                     const int32_t *jhiA, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass, int64_t *nC,
-                     int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s);
-void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, cudaStream_t s);
+                     const int32_t *jhiA, bool merge, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass,
+                     int64_t *nC, int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s);
+void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
+                     cudaStream_t s);
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s);
 void launch_compact(const CompactParams &P, cudaStream_t s);
 

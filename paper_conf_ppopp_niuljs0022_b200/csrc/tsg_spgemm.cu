@@ -10,6 +10,7 @@
 // Blocking device->host reads: (0) candidate total and row classes, (1) number of C tiles,
 // (2) nnz(C).  Everything else is stream-ordered.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "tsg_kernels.cuh"
@@ -68,6 +69,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
     uint16_t *mTA = tmp.get<uint16_t>(TILE * ntA);
     launch_transpose(A->mask, ntA, mTA, s);
+    uint16_t *mTB = mTA;  // A^2 (and any call with B's masks == A's): one transpose serves both
+    if (B->mask != A->mask) {
+        mTB = tmp.get<uint16_t>(TILE * B->nt);
+        launch_transpose(B->mask, B->nt, mTB, s);
+    }
     const bool lists = !(flags & TSG_STEP1_SCAN_ONLY) &&
                        ((flags & TSG_STEP1_LIST_ALWAYS) || (B->nt > 0 && B->nnz < 2 * B->nt));
     int64_t *lptr = nullptr;
@@ -101,7 +107,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     int64_t *nC = tmp.get<int64_t>(tmA + 1);
     int32_t *bigList = tmp.get<int32_t>(tmA);
     int64_t *bigOff = tmp.get<int64_t>(tmA);
-    launch_row_plan(tmA, A->tile_ptr, costOff, jloA, jhiA, rowJlo, rowJhi, rowClass, nC, bigList, bigOff, cnt, s);
+    launch_row_plan(tmA, A->tile_ptr, costOff, jloA, jhiA, !(flags & TSG_STEP1_SORT_ONLY), rowJlo, rowJhi, rowClass,
+                    nC, bigList, bigOff, cnt, s);
     // sync #0: candidate total and row classes
     DevCounters hc{};
     int64_t Utot = 0;
@@ -127,6 +134,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.rowJlo = rowJlo;
     P1.rowJhi = rowJhi;
     P1.rowClass = rowClass;
+    P1.tnB = B->tn;
     P1.pairs = tmp.get<uint64_t>(Utot);
     P1.tJ = tmp.get<int32_t>(Utot);
     P1.tStart = tmp.get<uint32_t>(Utot);
@@ -142,7 +150,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         P1.bigPosB = tmp.get<uint32_t>(hc.big_u);
         P1.bigKpos = tmp.get<uint32_t>(hc.big_u);
     }
-    launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, s);
+    launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, (int64_t)hc.nmerge, s);
     int64_t *tile_ptr = out.get<int64_t>(tmA + 1);
     exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
     tm_.mark(2);
@@ -181,6 +189,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.rpB = B->row_ptr;
     P.mB = B->mask;
     P.rowOccB = rowOccB;
+    P.mTB = mTB;
     P.ixB = B->idx;
     P.vB = B->val;
     P.tnzC = tile_nnz;
@@ -188,6 +197,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.mC = mask;
     P.work = work;
     P.dense_threshold = TH;
+    P.small_max = SMALL_NNZ;
+    if (const char *e = getenv("TSG_SMALL_NNZ")) P.small_max = std::max(0, std::min(16, atoi(e)));  // tuning only
     P.cnt = cnt;
     launch_step2(P, s);
     // ---------------- a3: offsets of C's nonzeros, allocation
@@ -285,6 +296,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         st->step3_rows = (int64_t)fin.n3rows;
         st->step3_row_tiles = rowk ? ntC - (int64_t)fin.n3fallback : 0;
         st->step1_list_tiles = (int32_t)fin.list_tiles;
+        st->step1_merge_rows = (int64_t)fin.nmerge;
         st->host_syncs = syncs;
         st->kernel_launches = call_launches();
         st->ms_host_sync = (float)t_host_sync_ms;

@@ -13,7 +13,7 @@ namespace tsg {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-enum RowClass : uint8_t { ROW_EMPTY = 0, ROW_SMALL = 1, ROW_BIG = 2 };
+enum RowClass : uint8_t { ROW_EMPTY = 0, ROW_SMALL = 1, ROW_BIG = 2, ROW_MERGE = 3 };
 
 __device__ __forceinline__ int bits_for(uint64_t v) {  // bits needed to represent v (>= 1)
     return v ? 64 - __clzll((long long)v) : 1;
@@ -137,7 +137,7 @@ __global__ void k_atile_plan(int64_t ntA, const int32_t *__restrict__ tcA, const
 
 // a1 (row plan): candidate window and class of every tile row (one warp per row)
 __global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const int64_t *__restrict__ costOff,
-                           const int32_t *__restrict__ jloA, const int32_t *__restrict__ jhiA,
+                           const int32_t *__restrict__ jloA, const int32_t *__restrict__ jhiA, bool merge,
                            int32_t *__restrict__ rowJlo, int32_t *__restrict__ rowJhi, uint8_t *__restrict__ rowClass,
                            int64_t *__restrict__ nC, int32_t *__restrict__ bigList, int64_t *__restrict__ bigOff,
                            DevCounters *cnt) {
@@ -162,6 +162,11 @@ __global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const i
     if (U == 0 || hi < lo) {
         rowClass[I] = ROW_EMPTY;
         nC[I] = 0;
+        return;
+    }
+    if (merge && a1 - a0 <= MERGE_MAX_A) {
+        rowClass[I] = ROW_MERGE;
+        atomicAdd(&cnt->nmerge, 1ULL);
         return;
     }
     const int wb = bits_for((uint64_t)(hi - lo + 1));  // valid 0..hi-lo, sentinel hi-lo+1
@@ -359,6 +364,178 @@ __device__ void row_sort_body(const S1Params &P, int64_t I, K *keysA, K *keysB, 
     }
 }
 
+// ------------------------------------------------------------------------------------------
+// a1 (merge): tile rows with at most 32 A tiles.  Lane l owns A tile a0+l; its candidate B tiles
+// (scan mode: B tile row K; list mode: the B row list) are already sorted by tile column J, so
+// the row's C tiles are a k-way merge of <= 32 sorted lists: per step the warp takes the minimum
+// head J (redux), the lanes holding J (ballot, lane order = ascending K) are that C tile's pairs,
+// and they advance.  Candidates without products are skipped lane-locally (reading B3).  Same
+// outputs, in the same candidate-space slots, as the expand/radix-sort path below; no shared
+// memory, no barriers, one step per C tile.
+// ------------------------------------------------------------------------------------------
+// C tile records of a merge: lane (n & 31) keeps step n's record, flushed 32 at a time (coalesced)
+struct MergeOut {
+    uint32_t rJ = 0, rS = 0, rC = 0, rW = 0, np = 0, ntl = 0;
+    __device__ __forceinline__ void emit(const S1Params &P, int64_t base, int lane, uint32_t J, unsigned hm,
+                                         uint32_t ws) {
+        if (lane == (int)(ntl & 31)) {
+            rJ = J;
+            rS = np;
+            rC = (uint32_t)__popc(hm);
+            rW = ws;
+        }
+        np += (uint32_t)__popc(hm);
+        ntl++;
+        if ((ntl & 31) == 0) flush(P, base, lane, 32);
+    }
+    __device__ __forceinline__ void flush(const S1Params &P, int64_t base, int lane, uint32_t n) {
+        if (lane < (int)n) {
+            const int64_t o = base + ((ntl - 1) & ~31u) + lane;
+            P.tJ[o] = (int32_t)rJ;
+            P.tStart[o] = rS;
+            P.tCnt[o] = rC;
+            P.tWork[o] = rW;
+        }
+    }
+    __device__ __forceinline__ void finish(const S1Params &P, int64_t base, int lane, int64_t I) {
+        if (ntl & 31) flush(P, base, lane, ntl & 31);
+        if (lane == 0) {
+            P.nC[I] = ntl;
+            atomicAdd(&P.cnt->pairs, (u64c)np);
+        }
+    }
+};
+
+constexpr int MERGE_W = 4;       // warps (tile rows) per merge CTA
+constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (8 B each)
+
+__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
+    constexpr uint32_t INF = 0xffffffffu;
+    constexpr uint32_t JM = (1u << 27) - 1u;  // tile column bits (n < 2^31); bits 27..31: work
+    __shared__ uint32_t sJ[MERGE_W][MERGE_CAP], sP[MERGE_W][MERGE_CAP];
+    __shared__ int64_t sSt[MERGE_W][32];
+    __shared__ uint32_t sOff[MERGE_W][33], sCo[MERGE_W][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
+    if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
+    const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
+    const int nA = (int)(a1 - a0);
+    const int64_t base = P.costOff[a0];
+    const int64_t U = P.costOff[a1] - base;
+    const int64_t t = a0 + lane;
+    int64_t len = 0, st = 0, off = 0;
+    bool isl = false;
+    uint32_t co = 0;
+    if (t < a1) {
+        off = P.costOff[t] - base;
+        len = P.costOff[t + 1] - base - off;
+        st = P.startA[t];
+        isl = st < 0;
+        if (isl) st = -st - 1;
+        co = P.colOccA[t];
+    }
+    const unsigned lt = (1u << lane) - 1u;
+    MergeOut out;
+    if (U <= MERGE_CAP && P.tnB < (int64_t)JM) {
+        // stage: every candidate's tile column (INF if it has no product, reading B3) + work in the
+        // top bits, and its B tile position; coalesced, all loads of the row in flight at once
+        sOff[w][lane] = t < a1 ? (uint32_t)off : (uint32_t)U;
+        sSt[w][lane] = isl ? -st - 1 : st;
+        sCo[w][lane] = co;
+        __syncwarp();
+        for (int u = lane; u < (int)U; u += 32) {
+            int lo = 0, hi = nA - 1;
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if ((int)sOff[w][mid] <= u) lo = mid;
+                else hi = mid - 1;
+            }
+            const int64_t sl = sSt[w][lo];
+            const int64_t k = u - (int)sOff[w][lo];
+            const bool il = sl < 0;
+            const uint32_t pos = il ? P.list[-sl - 1 + k] : (uint32_t)(sl + k);
+            const uint32_t J = (uint32_t)P.tcB[pos];
+            const uint32_t wk = il ? 1u : (uint32_t)__popc(sCo[w][lo] & (uint32_t)P.rowOccB[pos]);
+            sJ[w][u] = wk ? (J | (wk << 27)) : INF;
+            sP[w][u] = pos;
+        }
+        __syncwarp();
+        const uint32_t *mj = &sJ[w][off];
+        int64_t s = 0;
+        uint32_t hv = INF;
+        auto adv = [&]() {
+            while (s < len && (hv = mj[s]) == INF) s++;
+            if (s >= len) hv = INF;
+        };
+        adv();
+        for (;;) {
+            const uint32_t J = __reduce_min_sync(FULL, hv & JM);
+            if (J == JM) break;  // every lane exhausted (INF & JM == JM > any tile column)
+            const bool hit = hv != INF && (hv & JM) == J;
+            const unsigned hm = __ballot_sync(FULL, hit);
+            const uint32_t ws = __reduce_add_sync(FULL, hit ? hv >> 27 : 0u);
+            if (hit) P.pairs[base + out.np + __popc(hm & lt)] = ((uint64_t)t << 32) | sP[w][off + s];
+            out.emit(P, base, lane, J, hm, ws);
+            if (hit) {
+                s++;
+                adv();
+            }
+        }
+        out.finish(P, base, lane, I);
+        return;
+    }
+    // rows with more candidates than the stage holds: each lane keeps four candidates in flight
+    constexpr uint32_t JINF = 0x7fffffffu;
+    int64_t s = 0;
+    uint32_t bJ[4], bP[4], bO[4];
+    int bn = 0;
+    uint32_t head = JINF, hpos = 0, hocc = 0;
+    auto advance = [&]() {
+        for (;;) {
+            if (bn == 0) {
+                if (s >= len) {
+                    head = JINF;
+                    return;
+                }
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    const bool v = s + k < len;
+                    uint32_t pos = 0;
+                    if (v) pos = isl ? P.list[st + s + k] : (uint32_t)(st + s + k);
+                    bP[k] = pos;
+                    bJ[k] = v ? (uint32_t)P.tcB[pos] : JINF;
+                    bO[k] = v ? (uint32_t)P.rowOccB[pos] : 0u;
+                }
+                bn = (int)min((int64_t)4, len - s);
+                s += bn;
+            }
+            const uint32_t J = bJ[0], pos = bP[0], occ = bO[0];
+            bJ[0] = bJ[1]; bJ[1] = bJ[2]; bJ[2] = bJ[3];
+            bP[0] = bP[1]; bP[1] = bP[2]; bP[2] = bP[3];
+            bO[0] = bO[1]; bO[1] = bO[2]; bO[2] = bO[3];
+            bn--;
+            if (isl || (occ & co)) {
+                head = J;
+                hpos = pos;
+                hocc = occ;
+                return;
+            }
+        }
+    };
+    advance();
+    for (;;) {
+        const uint32_t J = __reduce_min_sync(FULL, head);
+        if (J == JINF) break;
+        const bool hit = head == J;
+        const unsigned hm = __ballot_sync(FULL, hit);
+        const uint32_t ws = __reduce_add_sync(FULL, hit ? (isl ? 1u : (uint32_t)__popc(co & hocc)) : 0u);
+        if (hit) P.pairs[base + out.np + __popc(hm & lt)] = ((uint64_t)t << 32) | hpos;
+        out.emit(P, base, lane, J, hm, ws);
+        if (hit) advance();
+    }
+    out.finish(P, base, lane, I);
+}
+
 __global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int64_t tm, int cap) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t hist[256 * ROW_NW];
@@ -452,10 +629,10 @@ void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA,
 }
 
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
-                     const int32_t *jhiA, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass, int64_t *nC,
-                     int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s) {
-    TSG_LAUNCH(k_row_plan, grid_for(tmA, 8), 256, 0, s, tmA, tpA, costOff, jloA, jhiA, rowJlo, rowJhi, rowClass, nC,
-               bigList, bigOff, cnt);
+                     const int32_t *jhiA, bool merge, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass,
+                     int64_t *nC, int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s) {
+    TSG_LAUNCH(k_row_plan, grid_for(tmA, 8), 256, 0, s, tmA, tpA, costOff, jloA, jhiA, merge, rowJlo, rowJhi,
+               rowClass, nC, bigList, bigOff, cnt);
 }
 
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s) {
@@ -466,7 +643,9 @@ void launch_compact(const CompactParams &P, cudaStream_t s) {
     TSG_LAUNCH(k_compact, grid_for(P.tm, 8), 256, 0, s, P);
 }
 
-void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, cudaStream_t s) {
+void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
+                     cudaStream_t s) {
+    if (nmerge > 0) TSG_LAUNCH(k_row_merge, grid_for(tm, MERGE_W), MERGE_W * 32, 0, s, P, tm);
     if (max_u_small > 0) {
         const int cap = (int)((max_u_small + 31) & ~31LL);
         const size_t smem = (size_t)cap * (4 + 4 + 4 + 2);

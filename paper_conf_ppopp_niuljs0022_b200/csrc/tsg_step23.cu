@@ -37,45 +37,69 @@ constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also
 // ==========================================================================================
 // step 2
 // ==========================================================================================
-// light tile (<= LIGHT_WORK items): one thread, item driven; row masks in 8 thread-private words
-__device__ __forceinline__ void s2_light(const StepParams &P, int64_t t, uint32_t *w, int stride) {
+// light tiles (<= LIGHT_WORK (pair, c) items): one thread per tile, item driven, row masks in 8
+// thread-private shared words.  A separate kernel at full occupancy: the work is a chain of
+// dependent loads (pair -> occupancy words -> masks), so the next pair's occupancy words are
+// loaded while the current pair is OR-ed.
+constexpr int T2L = 256;
+
+__global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
+    __shared__ uint32_t wsm[8 * T2L];
+    uint32_t *w = wsm + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * T2L;
+    u64c nl = 0;
+    for (int64_t t = (int64_t)blockIdx.x * T2L + threadIdx.x; t < P.ntC; t += stride) {
+        if (P.work[t] > (uint32_t)LIGHT_WORK) continue;
+        nl++;
 #pragma unroll
-    for (int q = 0; q < 8; q++) w[q * stride] = 0;
-    const uint64_t *pp = P.pairs + P.pairBeg[t];
-    const uint32_t np = P.pairCnt[t];
-    for (uint32_t p = 0; p < np; p++) {
-        const uint64_t pr = pp[p];
-        const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+        for (int q = 0; q < 8; q++) w[q * T2L] = 0;
+        const uint64_t *pp = P.pairs + P.pairBeg[t];
+        const uint32_t np = P.pairCnt[t];
+        uint64_t pr = pp[0];
+        int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
         uint32_t x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
-        const uint16_t *mb = P.mB + pB * TILE;
-        const uint16_t *at = P.mTA + pA * TILE;
-        while (x) {
-            const int c = __ffs(x) - 1;
-            x &= x - 1;
-            const uint32_t bits = mb[c];
-            uint32_t rows = at[c];
-            while (rows) {
-                const int r = __ffs(rows) - 1;
-                rows &= rows - 1;
-                w[(r >> 1) * stride] |= bits << (16 * (r & 1));
+        if (np > 1) pr = pp[1];
+        for (uint32_t p = 0; p < np; p++) {
+            const int64_t cA = pA, cB = pB;
+            uint32_t cx = x;
+            if (p + 1 < np) {
+                pA = (int64_t)(pr >> 32);
+                pB = (int64_t)(uint32_t)pr;
+                x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
+                if (p + 2 < np) pr = pp[p + 2];
+            }
+            const uint16_t *mb = P.mB + cB * TILE;
+            const uint16_t *at = P.mTA + cA * TILE;
+            while (cx) {
+                const int c = __ffs(cx) - 1;
+                cx &= cx - 1;
+                const uint32_t bits = mb[c];
+                uint32_t rows = at[c];
+                while (rows) {
+                    const int r = __ffs(rows) - 1;
+                    rows &= rows - 1;
+                    w[(r >> 1) * T2L] |= bits << (16 * (r & 1));
+                }
             }
         }
-    }
-    uint32_t m[8];
-    uint32_t rp[4] = {0, 0, 0, 0};
-    int total = 0;
+        uint32_t m[8];
+        uint32_t rp[4] = {0, 0, 0, 0};
+        int total = 0;
 #pragma unroll
-    for (int q = 0; q < 8; q++) m[q] = w[q * stride];
+        for (int q = 0; q < 8; q++) m[q] = w[q * T2L];
 #pragma unroll
-    for (int r = 0; r < 16; r++) {
-        rp[r >> 2] |= (uint32_t)total << (8 * (r & 3));
-        total += __popc((m[r >> 1] >> (16 * (r & 1))) & 0xffffu);
+        for (int r = 0; r < 16; r++) {
+            rp[r >> 2] |= (uint32_t)total << (8 * (r & 3));
+            total += __popc((m[r >> 1] >> (16 * (r & 1))) & 0xffffu);
+        }
+        uint4 *dm = reinterpret_cast<uint4 *>(P.mC + t * TILE);
+        dm[0] = make_uint4(m[0], m[1], m[2], m[3]);
+        dm[1] = make_uint4(m[4], m[5], m[6], m[7]);
+        *reinterpret_cast<uint4 *>(P.rpC + t * TILE) = make_uint4(rp[0], rp[1], rp[2], rp[3]);
+        P.tnzC[t] = total;
     }
-    uint4 *dm = reinterpret_cast<uint4 *>(P.mC + t * TILE);
-    dm[0] = make_uint4(m[0], m[1], m[2], m[3]);
-    dm[1] = make_uint4(m[4], m[5], m[6], m[7]);
-    *reinterpret_cast<uint4 *>(P.rpC + t * TILE) = make_uint4(rp[0], rp[1], rp[2], rp[3]);
-    P.tnzC[t] = total;
+    for (int o = 16; o > 0; o >>= 1) nl += __shfl_xor_sync(FULL, nl, o);
+    if ((threadIdx.x & 31) == 0 && nl) atomicAdd(&P.cnt->n2light, nl);
 }
 
 __device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
@@ -84,7 +108,6 @@ __device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
 }
 
 __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
-    __shared__ uint32_t wsm[8 * T2];
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
@@ -93,8 +116,7 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     for (int64_t g = (int64_t)blockIdx.x * (T2 / 32) + (threadIdx.x >> 5); g < ngroups; g += gstride) {
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC;
-        const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;
-        if (light) s2_light(P, t, wsm + threadIdx.x, T2);
+        const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;  // k_s2_light's class
         unsigned hm = __ballot_sync(FULL, v && !light);
         // heavy tiles: two at a time, a half warp each, lane r owns row r; per batch of 16 pairs
         // lane i stages pair i's A and B masks (4 x 16-byte cp.async, all in flight at once)
@@ -154,10 +176,7 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
             }
         }
         const unsigned lm = __ballot_sync(FULL, light), vm = __ballot_sync(FULL, v);
-        if (lane == 0) {
-            atomicAdd(&P.cnt->n2light, (u64c)__popc(lm));
-            atomicAdd(&P.cnt->n2heavy, (u64c)(__popc(vm) - __popc(lm)));
-        }
+        if (lane == 0 && vm != lm) atomicAdd(&P.cnt->n2heavy, (u64c)(__popc(vm) - __popc(lm)));
     }
 }
 
@@ -169,7 +188,6 @@ constexpr int WREG = 4224;  // bytes of per-warp shared scratch (small: 4 KB acc
 
 struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
     uint16_t mA[BATCH3][TILE], mB[BATCH3][TILE];  // cp.async'd masks of A_IK and B_KJ
-    uint16_t mT[BATCH3][TILE];                   // transposed A mask (small-tile path)
     uint8_t rA[BATCH3][TILE], rB[BATCH3][TILE];   // and their row offsets
     int64_t zA[BATCH3], zB[BATCH3];
     uint16_t oB[BATCH3];
@@ -183,157 +201,161 @@ __device__ __forceinline__ void cp_wait_all() {
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
 }
 
-// small tile (nnz <= 16): one thread, item driven.  Slot of C(r,j) is row_ptr_C[r] +
-// popc(mask_C[r] & ((1<<j)-1)) (the mask-addressed accumulator); slots, masks and
-// row offsets are thread-private (lane-strided words of the warp's scratch).
-__device__ __forceinline__ void s3_small(const StepParams &P, int64_t t, unsigned char *wr, int lane, MedStage &S) {
-    double *acc = reinterpret_cast<double *>(wr) + lane;                        // acc[q*32]
-    uint32_t *ms = reinterpret_cast<uint32_t *>(wr + SMALL_NNZ * 32 * 8) + lane;  // ms[k*32], k < 8
-    uint32_t *rs = ms + 8 * 32;                                                 // rs[k*32], k < 4
-    const int sl = lane & 15;  // this thread's staging slot in its half warp's MedStage
-    const int64_t z0 = P.tnzC[t];
-    const int nz = (int)(P.tnzC[t + 1] - z0);
-    {
-        const uint4 *pm = reinterpret_cast<const uint4 *>(P.mC + t * TILE);
-        const uint4 a = pm[0], b = pm[1];
-        ms[0] = a.x; ms[32] = a.y; ms[64] = a.z; ms[96] = a.w;
-        ms[128] = b.x; ms[160] = b.y; ms[192] = b.z; ms[224] = b.w;
-        const uint4 rp = *reinterpret_cast<const uint4 *>(P.rpC + t * TILE);
-        rs[0] = rp.x; rs[32] = rp.y; rs[64] = rp.z; rs[96] = rp.w;
-    }
-    for (int q = 0; q < nz; q++) acc[q * 32] = 0.0;
-    const uint64_t *pp = P.pairs + P.pairBeg[t];
-    const uint32_t np = P.pairCnt[t];
-    for (uint32_t p = 0; p < np; p++) {
-        const uint64_t pr = pp[p];
-        const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-        // the pair's masks, row offsets and transposed A mask: one round of cp.async instead of a
-        // chain of dependent reads
-        cp16(&S.mA[sl][0], P.mA + pA * TILE);
-        cp16(&S.mA[sl][8], P.mA + pA * TILE + 8);
-        cp16(&S.mB[sl][0], P.mB + pB * TILE);
-        cp16(&S.mB[sl][8], P.mB + pB * TILE + 8);
-        cp16(&S.rA[sl][0], P.rpA + pA * TILE);
-        cp16(&S.rB[sl][0], P.rpB + pB * TILE);
-        cp16(&S.mT[sl][0], P.mTA + pA * TILE);
-        cp16(&S.mT[sl][8], P.mTA + pA * TILE + 8);
-        uint32_t x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
-        const double *vbt = P.vB + P.tnzB[pB];
-        const double *vat = P.vA + P.tnzA[pA];
-        cp_wait_all();
-        // columns c ascending, rows of A's column c: every slot (r, j) sees ascending c
-        while (x) {
-            const int c = __ffs(x) - 1;
-            x &= x - 1;
-            const uint32_t mbc = S.mB[sl][c];
-            const double *vb = vbt + S.rB[sl][c];
-            uint32_t rows = S.mT[sl][c];
-            while (rows) {
-                const int r = __ffs(rows) - 1;
-                rows &= rows - 1;
-                const double a = vat[S.rA[sl][r] + __popc((uint32_t)S.mA[sl][r] & ((1u << c) - 1u))];
-                const uint32_t mcr = (ms[(r >> 1) * 32] >> (16 * (r & 1))) & 0xffffu;
-                const int base = (rs[(r >> 2) * 32] >> (8 * (r & 3))) & 0xff;
-                uint32_t mb = mbc;
-                int ib = 0;
-                while (mb) {
-                    const int j = __ffs(mb) - 1;
-                    mb &= mb - 1;
-                    const int q = base + __popc(mcr & ((1u << j) - 1u));
-                    acc[q * 32] = fma(a, vb[ib++], acc[q * 32]);
+// small tiles (nnz <= small_max): one lane per C nonzero (output-stationary; the paper's sparse
+// accumulator, with each slot owned by one lane).  Entry q of tile t is (r, j): r =
+// the last row whose offset row_ptr_C[r] <= q, j = the (q - row_ptr_C[r])-th set bit of
+// mask_C[r].  The lane walks its tile's pairs in ascending K; for each, the intersection
+// mask_A[r] & colmask_B[j] gives the contributing c (ascending), and A(r,c), B(c,j) are found by
+// popcount addressing.  The kernel is latency bound (dependent chains pair -> tile metadata ->
+// values), so it runs alone at full occupancy (no staging, few registers) and pipelines the
+// per-pair metadata one pair ahead.
+constexpr int TS = 256;  // small-class CTA
+constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <= 16)
+
+__global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
+    __shared__ uint8_t mapsm[TS / 32][SMAP];
+    const int lane = threadIdx.x & 31;
+    uint8_t *map = mapsm[threadIdx.x >> 5];
+    const int64_t ngroups = (P.ntC + 31) / 32;
+    const int64_t gstride = (int64_t)gridDim.x * (TS / 32);
+    for (int64_t g = (int64_t)blockIdx.x * (TS / 32) + (threadIdx.x >> 5); g < ngroups; g += gstride) {
+        const int64_t tl = g * 32 + lane;
+        const bool v = tl < P.ntC && !(P.skip && P.skip[tl]);
+        const int nz = v ? (int)(P.tnzC[tl + 1] - P.tnzC[tl]) : 0;
+        const bool small = v && nz < P.dense_threshold && nz <= P.small_max;
+        const int mine = small ? nz : 0;
+        int incl = mine;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int o = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl += o;
+        }
+        const int excl = incl - mine;
+        const int tot = __shfl_sync(FULL, incl, 31);
+        const unsigned smask = __ballot_sync(FULL, small);
+        if (lane == 0 && smask) atomicAdd(&P.cnt->n3small, (u64c)__popc(smask));
+        if (tot == 0) continue;
+        for (int q = 0; q < mine; q++) map[excl + q] = (uint8_t)lane;
+        __syncwarp();
+        for (int e0 = 0; e0 < tot; e0 += 32) {
+            const int e = e0 + lane;
+            const bool act = e < tot;
+            const int f = act ? map[e] : 0;
+            const int q = e - __shfl_sync(FULL, excl, f);
+            if (act) {
+                const int64_t t = g * 32 + f;
+                const uint4 rp = *reinterpret_cast<const uint4 *>(P.rpC + t * TILE);
+                const uint64_t *pp = P.pairs + P.pairBeg[t];
+                const uint32_t np = P.pairCnt[t];
+                const int64_t o = P.tnzC[t] + q;
+                // r = #{r' in 1..15 : row_ptr[r'] <= q}  (bytewise compare; row_ptr[0] = 0)
+                const uint32_t qq = (uint32_t)q * 0x01010101u;
+                const int r = (__popc(__vcmpleu4(rp.x, qq)) + __popc(__vcmpleu4(rp.y, qq)) +
+                               __popc(__vcmpleu4(rp.z, qq)) + __popc(__vcmpleu4(rp.w, qq))) / 8 - 1;
+                const uint32_t rpw = r < 4 ? rp.x : r < 8 ? rp.y : r < 12 ? rp.z : rp.w;
+                const int k = q - (int)((rpw >> (8 * (r & 3))) & 0xffu);
+                const int j = (int)__fns((uint32_t)P.mC[t * TILE + r], 0, k + 1);
+                const uint32_t lowj = (1u << j) - 1u;
+                double acc = 0.0;
+                // pair p's metadata is loaded while pair p-1 is being multiplied
+                uint64_t prn = pp[0];
+                int64_t pA = (int64_t)(prn >> 32), pB = (int64_t)(uint32_t)prn;
+                uint32_t mAr = P.mA[pA * TILE + r], mTj = P.mTB[pB * TILE + j];
+                int64_t zA = P.tnzA[pA] + P.rpA[pA * TILE + r], zB = P.tnzB[pB];
+                if (np > 1) prn = pp[1];
+                for (uint32_t p = 0; p < np; p++) {
+                    const int64_t cB = pB, czA = zA, czB = zB;
+                    uint32_t x = mAr & mTj;
+                    const uint32_t cmA = mAr;
+                    if (p + 1 < np) {
+                        pA = (int64_t)(prn >> 32);
+                        pB = (int64_t)(uint32_t)prn;
+                        mAr = P.mA[pA * TILE + r];
+                        mTj = P.mTB[pB * TILE + j];
+                        zA = P.tnzA[pA] + P.rpA[pA * TILE + r];
+                        zB = P.tnzB[pB];
+                        if (p + 2 < np) prn = pp[p + 2];
+                    }
+                    while (x) {
+                        const int c = __ffs(x) - 1;
+                        x &= x - 1;
+                        const double a = P.vA[czA + __popc(cmA & ((1u << c) - 1u))];
+                        const double b = P.vB[czB + P.rpB[cB * TILE + c] + __popc((uint32_t)P.mB[cB * TILE + c] & lowj)];
+                        acc = fma(a, b, acc);
+                    }
                 }
+                P.ixC[o] = (uint8_t)((r << 4) | j);
+                P.vC[o] = acc;
             }
         }
-    }
-    int q = 0;
-    for (int r = 0; r < TILE; r++) {
-        uint32_t m = (ms[(r >> 1) * 32] >> (16 * (r & 1))) & 0xffffu;
-        while (m) {
-            const int j = __ffs(m) - 1;
-            m &= m - 1;
-            P.ixC[z0 + q] = (uint8_t)((r << 4) | j);
-            P.vC[z0 + q] = acc[q * 32];
-            q++;
-        }
+        __syncwarp();
     }
 }
 
-// one column c of A's row r in flight: a = A(r,c), B's row c (mask, first 4 values, the rest)
-struct BRow {
-    double a, b0, b1, b2, b3;
-    uint32_t m;
-    const double *vb;
+// A lane's item stream of one batch (medium tiles, lane r owns C row r).  An item is (pair i, c)
+// with c in mask_A_i[r] & rowOcc(B_i): a = A_i(r,c) and B_i's row c (mask, first three values,
+// pointer to the rest).  Items come pair-ascending then c-ascending, so every C(r,j) receives its
+// products in ascending k.
+struct ItemStream {
+    int pi = -1;
+    uint32_t mAr = 0, ma = 0;
+    const double *va = nullptr, *vbt = nullptr;
+    // next item -> (a, b0..b2, mb, vb); false when the batch is exhausted
+    __device__ __forceinline__ bool fetch(const StepParams &P, const MedStage &S, int r, int nb, double &a,
+                                          double &b0, double &b1, double &b2, uint32_t &mb, const double *&vb) {
+        while (!ma) {
+            if (pi + 1 >= nb) return false;
+            ++pi;
+            mAr = S.mA[pi][r];
+            ma = mAr & S.oB[pi];
+            va = P.vA + S.zA[pi] + S.rA[pi][r];
+            vbt = P.vB + S.zB[pi];
+        }
+        const int c = __ffs(ma) - 1;
+        ma &= ma - 1;
+        a = va[__popc(mAr & ((1u << c) - 1u))];
+        mb = S.mB[pi][c];
+        vb = vbt + S.rB[pi][c];
+        const int n = __popc(mb);  // >= 1: row c of B_i is non-empty (rowOcc filter)
+        b0 = vb[0];
+        b1 = n > 1 ? vb[1] : 0.0;
+        b2 = n > 2 ? vb[2] : 0.0;
+        return true;
+    }
 };
-__device__ __forceinline__ BRow load_brow(const MedStage &S, int i, int c, uint32_t mAr, const double *va,
-                                          const double *vbt) {
-    BRow x;
-    x.m = S.mB[i][c];
-    x.vb = vbt + S.rB[i][c];
-    x.a = va[__popc(mAr & ((1u << c) - 1u))];
-    const int n = __popc(x.m);
-    x.b0 = x.vb[0];  // every row c here is non-empty (filtered by rowOcc(B))
-    x.b1 = n > 1 ? x.vb[1] : 0.0;
-    x.b2 = n > 2 ? x.vb[2] : 0.0;
-    x.b3 = n > 3 ? x.vb[3] : 0.0;
-    return x;
-}
-// acc[16 j] += a * B(c, j) over B's row c in ascending j (row accumulator: lane-strided slots).
-// The first four slots are distinct, so their loads, FMAs and stores are issued as a group
-// (independent shared-memory round trips instead of a chain of four).
-__device__ __forceinline__ void accumulate_brow(const BRow &x, double *acc) {
-    uint32_t m = x.m;
-    const int j0 = __ffs(m) - 1;
+
+// acc[16 j] += a * B(c, j) over B's row c in ascending j; the first three slots are distinct, so
+// their loads, FMAs and stores are independent
+__device__ __forceinline__ void accumulate_row(double a, double b0, double b1, double b2, uint32_t mb,
+                                               const double *vb, double *acc) {
+    const int j0 = __ffs(mb) - 1;
+    uint32_t m = mb & (mb - 1);
+    const int j1 = __ffs(m) - 1;
     m &= m - 1;
-    const int j1 = m ? __ffs(m) - 1 : j0;
+    const int j2 = __ffs(m) - 1;
     m &= m - 1;
-    const int j2 = m ? __ffs(m) - 1 : j0;
-    m &= m - 1;
-    const int j3 = m ? __ffs(m) - 1 : j0;
-    m &= m - 1;
-    const int n = __popc(x.m);
-    double c0 = acc[j0 * 16], c1 = 0.0, c2 = 0.0, c3 = 0.0;
-    if (n > 1) c1 = acc[j1 * 16];
-    if (n > 2) c2 = acc[j2 * 16];
-    if (n > 3) c3 = acc[j3 * 16];
-    acc[j0 * 16] = fma(x.a, x.b0, c0);
-    if (n > 1) acc[j1 * 16] = fma(x.a, x.b1, c1);
-    if (n > 2) acc[j2 * 16] = fma(x.a, x.b2, c2);
-    if (n > 3) acc[j3 * 16] = fma(x.a, x.b3, c3);
-    const double *vb = x.vb + 4;
+    double *p0 = acc + j0 * 16;
+    double *p1 = acc + (j1 >= 0 ? j1 : j0) * 16;
+    double *p2 = acc + (j2 >= 0 ? j2 : j0) * 16;
+    const double c0 = *p0, c1 = *p1, c2 = *p2;
+    *p0 = fma(a, b0, c0);
+    if (j1 >= 0) *p1 = fma(a, b1, c1);
+    if (j2 >= 0) *p2 = fma(a, b2, c2);
+    const double *q = vb + 3;
     while (m) {
         const int j = __ffs(m) - 1;
         m &= m - 1;
-        acc[j * 16] = fma(x.a, *vb++, acc[j * 16]);
+        acc[j * 16] = fma(a, *q++, acc[j * 16]);
     }
-}
-
-// a lane's position in its flat (pair, c) item sequence of a batch
-struct ItemCursor {
-    uint32_t rel = 0, ma = 0, mAr = 0;
-    int i = 0;
-    const double *va = nullptr, *vbt = nullptr;
-};
-__device__ __forceinline__ bool next_item(const StepParams &P, const MedStage &S, int r, ItemCursor &it, BRow &out) {
-    if (!it.ma) {
-        if (!it.rel) return false;
-        it.i = __ffs(it.rel) - 1;
-        it.rel &= it.rel - 1;
-        it.mAr = S.mA[it.i][r];
-        it.ma = it.mAr & S.oB[it.i];
-        it.va = P.vA + S.zA[it.i] + S.rA[it.i][r];
-        it.vbt = P.vB + S.zB[it.i];
-    }
-    const int c = __ffs(it.ma) - 1;
-    it.ma &= it.ma - 1;
-    out = load_brow(S, it.i, c, it.mAr, it.va, it.vbt);
-    return true;
 }
 
 // medium tile: a half warp, lane r owns C row r; dense-in-j 16-slot row accumulator in shared
 // memory (conflict free), compacted through mask_C[r] at the end.  Pairs go in batches of 16:
 // lane i stages pair i's A and B masks and row offsets (6 x 16-byte cp.async, all lanes and
 // pairs in flight at once), so a lane's walk over its row touches global memory only for the
-// values.  All 32 lanes must call.
+// values.  Each lane then runs its own flat item stream over the batch with two register sets
+// (the next item's loads are in flight while the current one accumulates).  All 32 lanes must
+// call.
 __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t t, double *acc, MedStage &S,
                                           int r) {
     uint32_t np = 0, mCr = 0;
@@ -353,7 +375,7 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
     const uint32_t nbw = max(nbat, __shfl_xor_sync(FULL, nbat, 16));
     for (uint32_t bt = 0; bt < nbw; bt++) {
         const uint32_t q = bt * BATCH3 + r;
-        if (r < BATCH3 && q < np) {
+        if (q < np) {
             const uint64_t pr = pp[q];
             const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
             cp16(&S.mA[r][0], P.mA + pA * TILE);
@@ -368,24 +390,19 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
         }
         cp_wait_all();
         __syncwarp();
-        const uint32_t nb = np > bt * BATCH3 ? min((uint32_t)BATCH3, np - bt * BATCH3) : 0u;
+        const int nb = np > bt * BATCH3 ? (int)min((uint32_t)BATCH3, np - bt * BATCH3) : 0;
         if (mCr) {
-            // the batch's pairs that touch row r, then one flat loop over this lane's (pair, c)
-            // items in order (pairs ascending, c ascending): lanes whose rows see different pairs
-            // (e.g. the 1-nonzero corner tiles of stencils touch one row) stay in step, and the
-            // next item's loads are in flight while the current one accumulates
-            uint32_t rel = 0;
-            for (uint32_t i = 0; i < nb; i++) rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
-            ItemCursor it;
-            it.rel = rel;
-            BRow cur;
-            bool have = next_item(P, S, r, it, cur);
-            while (have) {
-                BRow nxt;
-                const bool hn = next_item(P, S, r, it, nxt);
-                accumulate_brow(cur, acc);
-                cur = nxt;
-                have = hn;
+            ItemStream it;
+            double aX, bX0, bX1, bX2, aY, bY0, bY1, bY2;
+            uint32_t mX, mY;
+            const double *vX, *vY;
+            bool hX = it.fetch(P, S, r, nb, aX, bX0, bX1, bX2, mX, vX);
+            while (hX) {
+                const bool hY = it.fetch(P, S, r, nb, aY, bY0, bY1, bY2, mY, vY);
+                accumulate_row(aX, bX0, bX1, bX2, mX, vX, acc);
+                if (!hY) break;
+                hX = it.fetch(P, S, r, nb, aX, bX0, bX1, bX2, mX, vX);
+                accumulate_row(aY, bY0, bY1, bY2, mY, vY, acc);
             }
         }
         __syncwarp();
@@ -496,12 +513,10 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         const bool v = t < P.ntC && !(P.skip && P.skip[t]);
         const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
         const bool dense = v && nz >= P.dense_threshold;
-        const bool small = v && !dense && nz <= SMALL_NNZ;
+        const bool small = v && !dense && nz <= P.small_max;  // k_s3_small's class
         const unsigned sm = __ballot_sync(FULL, small);
         const unsigned dm = __ballot_sync(FULL, dense);
         unsigned mm = __ballot_sync(FULL, v) & ~sm & ~dm;
-        if (small) s3_small(P, t, wr, lane, med[threadIdx.x >> 4]);
-        __syncwarp();
         // medium tiles: two at a time, a half warp each
         double *acc = reinterpret_cast<double *>(wr) + half * (TILE * TILE) + r;
         while (mm) {
@@ -521,7 +536,6 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         }
         const unsigned vm = __ballot_sync(FULL, v);
         if (lane == 0) {
-            atomicAdd(&P.cnt->n3small, (u64c)__popc(sm));
             atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
             atomicAdd(&P.cnt->n3medium, (u64c)(__popc(vm) - __popc(sm) - __popc(dm)));
         }
@@ -538,11 +552,13 @@ unsigned grid_groups(int64_t ntC, int warps_per_cta) {
 
 void launch_step2(const StepParams &P, cudaStream_t s) {
     if (P.ntC <= 0) return;
+    TSG_LAUNCH(k_s2_light, (unsigned)std::min<int64_t>(ceil_div(P.ntC, T2L), 148LL * 8 * 4), T2L, 0, s, P);
     TSG_LAUNCH(k_s2, grid_groups(P.ntC, T2 / 32), T2, 0, s, P);
 }
 
 void launch_step3(const StepParams &P, cudaStream_t s) {
     if (P.ntC <= 0) return;
+    if (P.small_max > 0) TSG_LAUNCH(k_s3_small, grid_groups(P.ntC, TS / 32), TS, 0, s, P);
     TSG_LAUNCH(k_s3, grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
 }
 

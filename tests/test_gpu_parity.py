@@ -162,7 +162,8 @@ def _abs_csr(A, B):
 
 @pytest.mark.parametrize("opts", [dict(scan_only=True), dict(list_always=True), dict(dense_threshold=1),
                                   dict(dense_threshold=257), dict(dense_threshold=100), dict(step3_rows=True),
-                                  dict(step3_rows=True, dense_threshold=1)])
+                                  dict(step3_rows=True, dense_threshold=1), dict(sort_only=True),
+                                  dict(sort_only=True, list_always=True), dict(sort_only=True, scan_only=True)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
     for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12)):
@@ -172,6 +173,22 @@ def test_modes_give_identical_results(tsg, opts):
         for k in ARRAYS[:-1]:
             assert np.array_equal(base[k], alt[k]), (opts, k)
         assert bitwise_equal_values(base["val"], alt["val"])
+
+
+def test_step1_merge_coverage(tsg):
+    """Tile rows with <= 32 A tiles take the warp merge, wider rows the expand/sort path; both exact."""
+    hub = gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.0005)  # 2 tile rows of 128 tiles
+    for A, allmerge in ((gen.stencil27(12), True), (gen.strip_fem(6, 20, 6), True), (hub, False)):
+        T = tiles_of(tsg, A)
+        C = tsg.spgemm(T, T, stats=True)
+        nrows = int(np.count_nonzero(np.diff(T.tile_ptr.cpu().numpy())))
+        st = C.stats
+        if allmerge:
+            assert st["step1_merge_rows"] == nrows
+        else:
+            assert 0 < st["step1_merge_rows"] < nrows
+        assert tsg.spgemm(T, T, stats=True, sort_only=True).stats["step1_merge_rows"] == 0
+        assert_tiles_equal(host(C), oracle.expected_tiles(A, A, fma=True))
 
 
 def test_step3_row_kernel_coverage(tsg):
