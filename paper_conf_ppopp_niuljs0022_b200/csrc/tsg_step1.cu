@@ -407,14 +407,15 @@ struct MergeOut {
 };
 
 constexpr int MERGE_W = 4;       // warps (tile rows) per merge CTA
-constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (8 B each)
+constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (6 B each)
 
 __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
     constexpr uint32_t INF = 0xffffffffu;
     constexpr uint32_t JM = (1u << 27) - 1u;  // tile column bits (n < 2^31); bits 27..31: work
-    __shared__ uint32_t sJ[MERGE_W][MERGE_CAP], sP[MERGE_W][MERGE_CAP];
+    __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
+    __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
     __shared__ int64_t sSt[MERGE_W][32];
-    __shared__ uint32_t sOff[MERGE_W][33], sCo[MERGE_W][32];
+    __shared__ uint32_t sOff[MERGE_W][33], sCo[MERGE_W][32], sCnt[MERGE_W][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
     if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
@@ -437,44 +438,63 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
     const unsigned lt = (1u << lane) - 1u;
     MergeOut out;
     if (U <= MERGE_CAP && P.tnB < (int64_t)JM) {
-        // stage: every candidate's tile column (INF if it has no product, reading B3) + work in the
-        // top bits, and its B tile position; coalesced, all loads of the row in flight at once
+        // stage: the candidates that have products (reading B3), compacted per lane segment in
+        // order: tile column + work in the top bits, and the candidate's index k in its segment
+        // (16 bits; the B tile position is st + k, or list[st + k] in list mode).  The rank inside
+        // a segment comes from a ballot over the lanes of the same segment plus its count so far.
         sOff[w][lane] = t < a1 ? (uint32_t)off : (uint32_t)U;
         sSt[w][lane] = isl ? -st - 1 : st;
         sCo[w][lane] = co;
+        sCnt[w][lane] = 0;
         __syncwarp();
-        for (int u = lane; u < (int)U; u += 32) {
-            int lo = 0, hi = nA - 1;
-            while (lo < hi) {
-                const int mid = (lo + hi + 1) >> 1;
-                if ((int)sOff[w][mid] <= u) lo = mid;
-                else hi = mid - 1;
+        for (int u0 = 0; u0 < (int)U; u0 += 32) {
+            const int u = u0 + lane;
+            const bool in = u < (int)U;
+            int lo = 0, k = 0;
+            uint32_t val = 0;
+            bool ok = false;
+            if (in) {
+                int hi = nA - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if ((int)sOff[w][mid] <= u) lo = mid;
+                    else hi = mid - 1;
+                }
+                const int64_t sl = sSt[w][lo];
+                k = u - (int)sOff[w][lo];
+                const bool il = sl < 0;
+                const uint32_t pos = il ? P.list[-sl - 1 + k] : (uint32_t)(sl + k);
+                const uint32_t wk = il ? 1u : (uint32_t)__popc(sCo[w][lo] & (uint32_t)P.rowOccB[pos]);
+                ok = wk != 0;
+                val = (uint32_t)P.tcB[pos] | (wk << 27);
             }
-            const int64_t sl = sSt[w][lo];
-            const int64_t k = u - (int)sOff[w][lo];
-            const bool il = sl < 0;
-            const uint32_t pos = il ? P.list[-sl - 1 + k] : (uint32_t)(sl + k);
-            const uint32_t J = (uint32_t)P.tcB[pos];
-            const uint32_t wk = il ? 1u : (uint32_t)__popc(sCo[w][lo] & (uint32_t)P.rowOccB[pos]);
-            sJ[w][u] = wk ? (J | (wk << 27)) : INF;
-            sP[w][u] = pos;
+            const unsigned peers = __match_any_sync(FULL, in ? lo : -1);
+            const unsigned vb = __ballot_sync(FULL, ok) & peers;
+            if (ok) {
+                const int d = (int)sOff[w][lo] + (int)sCnt[w][lo] + __popc(vb & lt);
+                sJ[w][d] = val;
+                sK[w][d] = (uint16_t)k;
+            }
+            __syncwarp();
+            if (in && lane == 31 - __clz(peers)) sCnt[w][lo] += (uint32_t)__popc(vb);
+            __syncwarp();
         }
-        __syncwarp();
+        const int64_t vlen = t < a1 ? (int64_t)sCnt[w][lane] : 0;
         const uint32_t *mj = &sJ[w][off];
         int64_t s = 0;
-        uint32_t hv = INF;
-        auto adv = [&]() {
-            while (s < len && (hv = mj[s]) == INF) s++;
-            if (s >= len) hv = INF;
-        };
-        adv();
+        uint32_t hv = vlen > 0 ? mj[0] : INF;
+        auto adv = [&]() { hv = s < vlen ? mj[s] : INF; };
         for (;;) {
             const uint32_t J = __reduce_min_sync(FULL, hv & JM);
             if (J == JM) break;  // every lane exhausted (INF & JM == JM > any tile column)
             const bool hit = hv != INF && (hv & JM) == J;
             const unsigned hm = __ballot_sync(FULL, hit);
             const uint32_t ws = __reduce_add_sync(FULL, hit ? hv >> 27 : 0u);
-            if (hit) P.pairs[base + out.np + __popc(hm & lt)] = ((uint64_t)t << 32) | sP[w][off + s];
+            if (hit) {
+                const int64_t k = sK[w][off + s];
+                const uint32_t pos = isl ? P.list[st + k] : (uint32_t)(st + k);
+                P.pairs[base + out.np + __popc(hm & lt)] = ((uint64_t)t << 32) | pos;
+            }
             out.emit(P, base, lane, J, hm, ws);
             if (hit) {
                 s++;

@@ -297,15 +297,17 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
 // pointer to the rest).  Items come pair-ascending then c-ascending, so every C(r,j) receives its
 // products in ascending k.
 struct ItemStream {
-    int pi = -1;
+    uint32_t rel;  // batch pairs that touch row r (mask_A_i[r] & rowOcc(B_i) != 0), not yet started
+    int pi = 0;
     uint32_t mAr = 0, ma = 0;
     const double *va = nullptr, *vbt = nullptr;
     // next item -> (a, b0..b2, mb, vb); false when the batch is exhausted
-    __device__ __forceinline__ bool fetch(const StepParams &P, const MedStage &S, int r, int nb, double &a,
-                                          double &b0, double &b1, double &b2, uint32_t &mb, const double *&vb) {
-        while (!ma) {
-            if (pi + 1 >= nb) return false;
-            ++pi;
+    __device__ __forceinline__ bool fetch(const StepParams &P, const MedStage &S, int r, double &a, double &b0,
+                                          double &b1, double &b2, uint32_t &mb, const double *&vb) {
+        if (!ma) {
+            if (!rel) return false;
+            pi = __ffs(rel) - 1;
+            rel &= rel - 1;
             mAr = S.mA[pi][r];
             ma = mAr & S.oB[pi];
             va = P.vA + S.zA[pi] + S.rA[pi][r];
@@ -356,14 +358,34 @@ __device__ __forceinline__ void accumulate_row(double a, double b0, double b1, d
 // values.  Each lane then runs its own flat item stream over the batch with two register sets
 // (the next item's loads are in flight while the current one accumulates).  All 32 lanes must
 // call.
-__device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t t, double *acc, MedStage &S,
-                                          int r) {
+// per-lane metadata of a medium tile, loaded one tile ahead (the chain tile -> pair list -> masks
+// would otherwise be exposed at the start of every tile)
+struct MedMeta {
+    bool hv = false;
+    int64_t t = 0;
+    const uint64_t *pp = nullptr;
     uint32_t np = 0, mCr = 0;
-    const uint64_t *pp = P.pairs;
-    if (hv) {
-        pp += P.pairBeg[t];
-        np = P.pairCnt[t];
-        mCr = P.mC[t * TILE + r];
+    int64_t ob = 0;    // output offset of row r
+    uint64_t pr = 0;   // pair r of the first batch
+    __device__ __forceinline__ void load(const StepParams &P, int mine, int64_t g, int r) {
+        hv = mine >= 0;
+        t = g * 32 + (hv ? mine : 0);
+        np = 0;
+        mCr = 0;
+        if (hv) {
+            pp = P.pairs + P.pairBeg[t];
+            np = P.pairCnt[t];
+            mCr = P.mC[t * TILE + r];
+            ob = P.tnzC[t] + P.rpC[t * TILE + r];
+            if ((uint32_t)r < np) pr = pp[r];
+        }
+    }
+};
+
+__device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M, double *acc, MedStage &S, int r) {
+    const uint32_t np = M.np, mCr = M.mCr;
+    const uint64_t *pp = M.pp;
+    {
         uint32_t m = mCr;
         while (m) {
             const int j = __ffs(m) - 1;
@@ -376,7 +398,7 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
     for (uint32_t bt = 0; bt < nbw; bt++) {
         const uint32_t q = bt * BATCH3 + r;
         if (q < np) {
-            const uint64_t pr = pp[q];
+            const uint64_t pr = bt == 0 ? M.pr : pp[q];
             const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
             cp16(&S.mA[r][0], P.mA + pA * TILE);
             cp16(&S.mA[r][8], P.mA + pA * TILE + 8);
@@ -393,22 +415,24 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, bool hv, int64_t 
         const int nb = np > bt * BATCH3 ? (int)min((uint32_t)BATCH3, np - bt * BATCH3) : 0;
         if (mCr) {
             ItemStream it;
+            it.rel = 0;
+            for (int i = 0; i < nb; i++) it.rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
             double aX, bX0, bX1, bX2, aY, bY0, bY1, bY2;
             uint32_t mX, mY;
             const double *vX, *vY;
-            bool hX = it.fetch(P, S, r, nb, aX, bX0, bX1, bX2, mX, vX);
+            bool hX = it.fetch(P, S, r, aX, bX0, bX1, bX2, mX, vX);
             while (hX) {
-                const bool hY = it.fetch(P, S, r, nb, aY, bY0, bY1, bY2, mY, vY);
+                const bool hY = it.fetch(P, S, r, aY, bY0, bY1, bY2, mY, vY);
                 accumulate_row(aX, bX0, bX1, bX2, mX, vX, acc);
                 if (!hY) break;
-                hX = it.fetch(P, S, r, nb, aX, bX0, bX1, bX2, mX, vX);
+                hX = it.fetch(P, S, r, aX, bX0, bX1, bX2, mX, vX);
                 accumulate_row(aY, bY0, bY1, bY2, mY, vY, acc);
             }
         }
         __syncwarp();
     }
-    if (hv && mCr) {
-        const int64_t ob = P.tnzC[t] + P.rpC[t * TILE + r];
+    if (mCr) {
+        const int64_t ob = M.ob;
         uint32_t m = mCr;
         int qq = 0;
         while (m) {
@@ -519,13 +543,23 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         unsigned mm = __ballot_sync(FULL, v) & ~sm & ~dm;
         // medium tiles: two at a time, a half warp each
         double *acc = reinterpret_cast<double *>(wr) + half * (TILE * TILE) + r;
-        while (mm) {
+        auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
             const int f0 = __ffs(mm) - 1;
             mm &= mm - 1;
             const int f1 = mm ? __ffs(mm) - 1 : -1;
             if (mm) mm &= mm - 1;
-            const int mine = half ? f1 : f0;
-            s3_medium(P, mine >= 0, g * 32 + (mine >= 0 ? mine : 0), acc, med[threadIdx.x >> 4], r);
+            return half ? f1 : f0;
+        };
+        if (mm) {
+            MedMeta cur, nxt;
+            cur.load(P, pop2(), g, r);
+            for (;;) {
+                const bool more = mm != 0;  // warp-uniform
+                if (more) nxt.load(P, pop2(), g, r);
+                s3_medium(P, cur, acc, med[threadIdx.x >> 4], r);
+                if (!more) break;
+                cur = nxt;
+            }
         }
         // dense tiles: the whole warp each
         unsigned dd = dm;
