@@ -107,6 +107,8 @@ typedef struct {
     int64_t step3_row_tiles;  /* C tiles whose step 3 ran in the whole-tile-row kernel */
     int64_t step3_rows;       /* tile rows handled by that kernel */
     int64_t step1_merge_rows; /* tile rows whose step 1 ran as a warp k-way merge (<= 32 A tiles) */
+    int64_t bytes_scratch;    /* device scratch of the call (its peak; f4, cf. Fig 9 peak space P:2938-2968) */
+    int64_t bytes_out;        /* device bytes of C's seven arrays (allocation sizes; Fig 11) */
 } tsg_stats;
 
 /* flags for tsg_csr_to_tiles */

@@ -96,6 +96,15 @@ class Tiles:
     def arrays(self) -> dict:
         return {k: getattr(self, k) for k in ("tile_ptr", "tile_col", "tile_nnz", "row_ptr", "mask", "idx", "val")}
 
+    def space(self) -> dict:
+        """Bytes of this matrix in the tile format vs CSR (the paper's Fig 11,
+        P:2991-3057).  Tile format: tile_ptr 8(tm+1) + per tile 4 (col) + 8 (nnz offset) + 16
+        (row_ptr) + 32 (mask) + per nonzero 1 (idx) + 8 (val); CSR: 8(m+1) row offsets (int64, reading
+        A4) + per nonzero 4 (col) + 8 (val)."""
+        tile = 8 * (self.tile_m + 1) + 8 + 60 * self.num_tiles + 9 * self.nnz
+        csr = 8 * (self.m + 1) + 12 * self.nnz
+        return {"tile_bytes": tile, "csr_bytes": csr, "ratio": tile / csr if csr else float("nan")}
+
     def copy_to_host(self, out: dict | None = None, stream=None) -> dict:
         """Copy the seven arrays into host buffers (numpy or pinned torch CPU tensors) via the C ABI."""
         sizes = {"tile_ptr": (self.tile_m + 1, np.int64), "tile_col": (self.num_tiles, np.int32),

@@ -54,7 +54,7 @@ class Stats(C.Structure):
                 ("ms_alloc", C.c_float), ("ms_step3", C.c_float), ("ms_total", C.c_float),
                 ("ms_host_sync", C.c_float), ("ms_host_alloc", C.c_float),
                 ("step3_row_tiles", C.c_int64), ("step3_rows", C.c_int64),
-                ("step1_merge_rows", C.c_int64)]
+                ("step1_merge_rows", C.c_int64), ("bytes_scratch", C.c_int64), ("bytes_out", C.c_int64)]
 
     def as_dict(self) -> dict:
         return {f[0]: getattr(self, f[0]) for f in self._fields_}

@@ -113,6 +113,7 @@ class Buffers {
         size_t bytes = sizeof(T) * (size_t)(count > 0 ? count : 0);
         if (bytes < 256) bytes = 256;  // never hand out NULL; keep 256-byte alignment
         bytes = (bytes + 255) & ~(size_t)255;
+        handed_ += bytes;
         if (arena_) {
             Arena &a = *arena_;
             if (a.off + bytes <= a.cap) {
@@ -147,6 +148,8 @@ class Buffers {
         for (auto &it : items_) al_.free(it.p, it.bytes, s_);
         items_.clear();
     }
+    // bytes handed out by get() so far (scratch is a stack within a call: this is its peak)
+    size_t handed() const { return handed_; }
 
    private:
     void enter_arena();
@@ -160,6 +163,7 @@ class Buffers {
     std::vector<Item> items_;
     Arena *arena_ = nullptr;
     size_t mark_ = 0;
+    size_t handed_ = 0;
 };
 
 }  // namespace tsg

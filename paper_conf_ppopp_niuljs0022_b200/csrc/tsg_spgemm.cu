@@ -297,6 +297,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         st->step3_row_tiles = rowk ? ntC - (int64_t)fin.n3fallback : 0;
         st->step1_list_tiles = (int32_t)fin.list_tiles;
         st->step1_merge_rows = (int64_t)fin.nmerge;
+        st->bytes_scratch = (int64_t)tmp.handed();
+        st->bytes_out = 0;
+        for (int k = 0; k < 7; k++) st->bytes_out += (int64_t)C->bytes[k];
         st->host_syncs = syncs;
         st->kernel_launches = call_launches();
         st->ms_host_sync = (float)t_host_sync_ms;

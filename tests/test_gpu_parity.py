@@ -377,3 +377,19 @@ def test_aat_matches_oracle(tsg, name, A):
     ref = oracle.expected_tiles(A, At, fma=True)
     assert_tiles_equal(host(C), ref)
     assert C.stats["products"] == oracle.products(A, At)
+
+
+def test_space_and_peak_memory_reporting(tsg):
+    """tile-format bytes vs CSR (Fig 11) and the call's device memory
+    (Fig 9) are reported and consistent with the arrays actually held."""
+    for A in (gen.config("C1"), gen.strip_fem(6, 20, 6), gen.rmat(11)):
+        T = tiles_of(tsg, A)
+        C = tsg.spgemm(T, T, stats=True)
+        for M in (T, C):
+            sp = M.space()
+            held = sum(x.numel() * x.element_size() for x in M.arrays().values())
+            assert sp["tile_bytes"] == held
+            assert sp["csr_bytes"] == 8 * (M.m + 1) + 12 * M.nnz
+        st = C.stats
+        assert st["bytes_out"] >= C.space()["tile_bytes"]
+        assert st["bytes_scratch"] > 0
