@@ -45,7 +45,7 @@ extern "C" {
 #define TSG_TILE 16          /* tile size, fixed by the paper */
 #define TSG_DENSE_NNZ 96     /* t_nnz: dense accumulator iff tile nnz >= 96 (the paper's 192, re-tuned
                                 for these kernels on B200: reading A7) */
-#define TSG_ABI_VERSION 1
+#define TSG_ABI_VERSION 2
 
 typedef enum {
     TSG_OK = 0,
@@ -68,6 +68,12 @@ typedef struct {
 /* Opaque, device-resident matrix in sparse-tile form; owns (or borrows) its arrays. */
 typedef struct tsg_tiles tsg_tiles;
 
+/* Value types.  The paper's main runs are fp64; its Section 4.7 runs TileSpGEMM
+ * with half-precision input and single-precision output.  A product's C type:
+ * F64 x F64 -> F64, F32 x F32 -> F32, F16 x F16 -> F32 (accumulated in fp32); any other mix is
+ * TSG_ERR_INVALID_ARG.  Steps 1 and 2 do not look at values. */
+typedef enum { TSG_F64 = 0, TSG_F32 = 1, TSG_F16 = 2 } tsg_dtype;
+
 /* Read-only view of the Section 3.2 arrays, all device pointers.
  *   tile_ptr [tile_m+1]     int64  offsets of the tiles of each tile row
  *   tile_col [num_tiles]    int32  tile column ids, strictly ascending per row
@@ -75,7 +81,7 @@ typedef struct tsg_tiles tsg_tiles;
  *   row_ptr  [16*num_tiles] uint8  local row offsets, 16 per tile, no 17th       (A3)
  *   mask     [16*num_tiles] uint16 bit c of row r <=> nonzero at (r,c)           (A2)
  *   idx      [nnz]          uint8  (r<<4)|c of each nonzero                      (A1)
- *   val      [nnz]          double values in tile order
+ *   val      [nnz]          dtype  values in tile order (double/float/half)
  * Every stored tile is non-empty (reading A6). */
 typedef struct {
     int64_t m, n, tile_m, tile_n, num_tiles, nnz;
@@ -85,7 +91,8 @@ typedef struct {
     const uint8_t *row_ptr;
     const uint16_t *mask;
     const uint8_t *idx;
-    const double *val;
+    const void *val;
+    int32_t dtype;            /* tsg_dtype of val */
 } tsg_tiles_view;
 
 /* Per-call statistics of tsg_spgemm (all counts exact; times only with TSG_STATS_TIMING). */
@@ -142,6 +149,12 @@ TSG_API tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int
                             const int32_t *col_idx, const double *val, uint32_t flags,
                             const tsg_allocator *al, void *stream, tsg_tiles **out);
 
+/* tsg_csr_to_tiles_typed -- the same with values of type `dtype` (val: [nnz] double, float or
+ * IEEE half; f3).  The handle records the dtype. */
+TSG_API tsg_status tsg_csr_to_tiles_typed(int64_t m, int64_t n, int64_t nnz, const int64_t *row_ptr,
+                                  const int32_t *col_idx, const void *val, int32_t dtype, uint32_t flags,
+                                  const tsg_allocator *al, void *stream, tsg_tiles **out);
+
 /*
  * tsg_spgemm -- C = A*B, both in sparse-tile form; the three steps of Section 3.3
  * (P:880-1888): step 1 tile layout of C, step 2 bit-mask symbolic phase with
@@ -154,6 +167,8 @@ TSG_API tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int
  *   stats   optional (NULL allowed)
  * Values: C(r,j) = sum over pairs in ascending K, over c ascending, of A(r,c)*B(c,j) with
  * fused multiply-add, i.e. ascending global k (reading A8/A16): deterministic run to run.
+ * Value types: C's dtype follows tsg_dtype's rules (F16 inputs are widened exactly to fp32 and
+ * accumulated with fp32 FMA); mixed input dtypes are INVALID_ARG.
  * Syncs: 3 blocking scalar reads (candidate total, C tile count, nnz(C)).
  * Alignment: mask and row_ptr of A and B must be 16-byte aligned, val 8-byte aligned (tiles are
  * staged into shared memory in 16-byte chunks); handles made by this library always are.
@@ -166,10 +181,10 @@ TSG_API tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t f
  * tsg_tiles_to_csr -- sparse tiles -> CSR (inverse of tsg_csr_to_tiles; used for checking,
  * P:4637-4639).  Outputs are new device arrays allocated through `al` (free them with
  * tsg_free using the same allocator):  row_ptr int64 [m+1], col_idx int32 [nnz],
- * val double [nnz]; *nnz receives nnz.  Syncs: none beyond reading the handle's own sizes.
+ * val [nnz] of T's dtype; *nnz receives nnz.  Syncs: none beyond reading the handle's own sizes.
  */
 TSG_API tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *stream,
-                            int64_t **row_ptr, int32_t **col_idx, double **val, int64_t *nnz);
+                            int64_t **row_ptr, int32_t **col_idx, void **val, int64_t *nnz);
 
 /*
  * tsg_tiles_transpose -- A^T in sparse-tile form, for the paper's second workload C = A*A^T
@@ -204,11 +219,12 @@ TSG_API tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t tile_row_beg
 
 /*
  * tsg_tiles_copy_to_host -- copy the seven arrays into caller-provided HOST buffers (pinned
- * for speed), sized from tsg_tiles_get_view; NULL skips an array.  Blocks until done.
+ * for speed), sized from tsg_tiles_get_view (val: nnz elements of the view's dtype); NULL skips
+ * an array.  Blocks until done.
  */
 TSG_API tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr,
                                   int32_t *tile_col, int64_t *tile_nnz, uint8_t *row_ptr,
-                                  uint16_t *mask, uint8_t *idx, double *val);
+                                  uint16_t *mask, uint8_t *idx, void *val);
 
 /* Release a handle (stream-ordered frees through its allocator).  NULL is a no-op. */
 TSG_API void tsg_tiles_destroy(tsg_tiles *T, void *stream);

@@ -41,6 +41,7 @@ _lib = None
 _i64p = np.ctypeslib.ndpointer(np.int64, flags="C")
 _i32p = np.ctypeslib.ndpointer(np.int32, flags="C")
 _f64p = np.ctypeslib.ndpointer(np.float64, flags="C")
+_f32p = np.ctypeslib.ndpointer(np.float32, flags="C")
 _u8p = np.ctypeslib.ndpointer(np.uint8, flags="C")
 _u16p = np.ctypeslib.ndpointer(np.uint16, flags="C")
 
@@ -55,6 +56,8 @@ def lib():
         L.orc_gustavson_rowcounts.argtypes = [i64, i64, _i64p, _i32p, _i64p, _i32p, C.c_void_p, i64, _i64p]
         L.orc_gustavson.argtypes = [i64, i64, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p, C.c_void_p, i64,
                                     _i64p, _i32p, _f64p, C.c_void_p, C.c_int]
+        L.orc_gustavson_f32.argtypes = [i64, i64, _i64p, _i32p, _f32p, _i64p, _i32p, _f32p, C.c_void_p, i64,
+                                         _i64p, _i32p, _f32p, C.c_void_p, C.c_int]
         L.orc_csr_to_tiles_count.argtypes = [i64, i64, _i64p, _i32p, _i64p]
         L.orc_csr_to_tiles_fill.argtypes = [i64, i64, _i64p, _i32p, _f64p, _i64p, _i32p, _i64p, _u8p, _u16p,
                                             _u8p, _f64p]
@@ -158,13 +161,19 @@ def transpose(A) -> OracleCSR:
     return OracleCSR(A.n, A.m, rpT, colT, valT)
 
 
-def spgemm(A, B, fma: bool = False, rows=None) -> OracleCSR:
-    """O1: C = A*B by Gustavson's row-row Algorithm 1.  ``rows`` selects a subset."""
+def spgemm(A, B, fma: bool = False, rows=None, prec: str = "f64") -> OracleCSR:
+    """O1: C = A*B by Gustavson's row-row Algorithm 1.  ``rows`` selects a subset.
+
+    prec="f32": the same loop in single precision (f3); values are taken as float32
+    (a float16 input is widened exactly), the result's val is float32, abs stays fp64."""
     if A.n != B.m:
         raise ValueError("shape mismatch")
+    if prec not in ("f64", "f32"):
+        raise ValueError("prec must be 'f64' or 'f32'")
     L = lib()
-    Arp, Aci, Av = _arr(A.rowptr, np.int64), _arr(A.col, np.int32), _arr(A.val, np.float64)
-    Brp, Bci, Bv = _arr(B.rowptr, np.int64), _arr(B.col, np.int32), _arr(B.val, np.float64)
+    vdt = np.float64 if prec == "f64" else np.float32
+    Arp, Aci, Av = _arr(A.rowptr, np.int64), _arr(A.col, np.int32), _arr(A.val, vdt)
+    Brp, Bci, Bv = _arr(B.rowptr, np.int64), _arr(B.col, np.int32), _arr(B.val, vdt)
     if rows is None:
         R, rp_ptr, nrows = A.m, None, 0
     else:
@@ -176,10 +185,11 @@ def spgemm(A, B, fma: bool = False, rows=None) -> OracleCSR:
     np.cumsum(rowlen[:R], out=rp[1:])
     nnz = int(rp[-1])
     col = np.zeros(max(nnz, 1), dtype=np.int32)
-    val = np.zeros(max(nnz, 1), dtype=np.float64)
+    val = np.zeros(max(nnz, 1), dtype=vdt)
     ab = np.zeros(max(nnz, 1), dtype=np.float64)
-    _chk(L.orc_gustavson(A.m, B.n, Arp, Aci, Av, Brp, Bci, Bv, rp_ptr, nrows, rp, col, val,
-                         ab.ctypes.data_as(C.c_void_p), int(fma)), "gustavson")
+    f = L.orc_gustavson if prec == "f64" else L.orc_gustavson_f32
+    _chk(f(A.m, B.n, Arp, Aci, Av, Brp, Bci, Bv, rp_ptr, nrows, rp, col, val, ab.ctypes.data_as(C.c_void_p),
+           int(fma)), "gustavson")
     return OracleCSR(R, B.n, rp, col[:nnz], val[:nnz], ab[:nnz])
 
 
@@ -268,9 +278,14 @@ def spmv(A, x) -> np.ndarray:
 DENSE_THRESHOLD = 192  # t_nnz = 192 for 16x16 tiles; dense iff nnz >= 192 (reading A7)
 
 
-def expected_tiles(A, B, fma: bool = False) -> OracleTiles:
-    """The exact tile-format C that TileSpGEMM must produce: O2(O1(A, B)) (reading A6)."""
-    return csr_to_tiles(spgemm(A, B, fma=fma))
+def expected_tiles(A, B, fma: bool = False, prec: str = "f64") -> OracleTiles:
+    """The exact tile-format C that TileSpGEMM must produce: O2(O1(A, B)) (reading A6).
+    prec="f32": O1 in single precision; the tiler moves the float32 values exactly (via fp64)."""
+    O = spgemm(A, B, fma=fma, prec=prec)
+    T = csr_to_tiles(O)
+    if prec == "f32":
+        T.val = T.val.astype(np.float32)
+    return T
 
 
 def diagnostics(A, B) -> dict:

@@ -137,6 +137,63 @@ int orc_gustavson(int64_t m, int64_t n, const int64_t *Arp, const int32_t *Aci, 
     return 0;
 }
 
+/* O1 in single precision (the paper's Section 4.7 setup computes with half
+ * inputs and single-precision output): the same Algorithm 1 loop with float
+ * accumulators; inputs are floats (a half input is widened to float exactly before the call).
+ * Cabs is the fp64 sum of |a*b| (exact products of floats). */
+int orc_gustavson_f32(int64_t m, int64_t n, const int64_t *Arp, const int32_t *Aci, const float *Aval,
+                      const int64_t *Brp, const int32_t *Bci, const float *Bval, const int64_t *rows,
+                      int64_t nrows, const int64_t *Crp, int32_t *Cci, float *Cval, double *Cabs,
+                      int fma_mode) {
+    if (m < 0 || n < 0) return -1;
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    int64_t *stamp = (int64_t *)malloc(sizeof(int64_t) * nn);
+    float *acc = (float *)malloc(sizeof(float) * nn);
+    double *acc_abs = (double *)malloc(sizeof(double) * nn);
+    int64_t *list = (int64_t *)malloc(sizeof(int64_t) * nn);
+    if (!stamp || !acc || !acc_abs || !list) {
+        free(stamp); free(acc); free(acc_abs); free(list);
+        return -2;
+    }
+    for (int64_t j = 0; j < n; j++) stamp[j] = -1;
+    int64_t R = rows ? nrows : m;
+    for (int64_t t = 0; t < R; t++) {
+        int64_t i = rows ? rows[t] : t;
+        int64_t len = 0;
+        for (int64_t p = Arp[i]; p < Arp[i + 1]; p++) {          /* line 4, ascending k */
+            int64_t k = Aci[p];
+            float a = Aval[p];
+            for (int64_t q = Brp[k]; q < Brp[k + 1]; q++) {      /* line 5 */
+                int64_t j = Bci[q];
+                float b = Bval[q];
+                float value = a * b;                             /* line 6 */
+                if (stamp[j] != t) {                             /* lines 7-9: insert */
+                    stamp[j] = t;
+                    list[len++] = j;
+                    acc[j] = value;
+                    acc_abs[j] = fabs((double)a * (double)b);
+                } else {                                         /* line 11: accumulate */
+                    acc[j] = fma_mode ? fmaf(a, b, acc[j]) : acc[j] + value;
+                    acc_abs[j] += fabs((double)a * (double)b);
+                }
+            }
+        }
+        if (Crp[t + 1] - Crp[t] != len) {
+            free(stamp); free(acc); free(acc_abs); free(list);
+            return -3;
+        }
+        qsort(list, (size_t)len, sizeof(int64_t), cmp_i64);
+        for (int64_t e = 0; e < len; e++) {
+            int64_t j = list[e];
+            Cci[Crp[t] + e] = (int32_t)j;
+            Cval[Crp[t] + e] = acc[j];
+            if (Cabs) Cabs[Crp[t] + e] = acc_abs[j];
+        }
+    }
+    free(stamp); free(acc); free(acc_abs); free(list);
+    return 0;
+}
+
 /* ------------------------------------------------------------------------------------------
  * O2: CSR -> sparse tiles, Section 3.2.
  *   tile_ptr[tm+1]   offsets of tiles per tile row

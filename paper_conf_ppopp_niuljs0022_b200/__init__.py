@@ -25,7 +25,11 @@ from ._lib import TILE, DENSE_NNZ, TsgError  # noqa: F401
 __all__ = ["Tiles", "csr_to_tiles", "spgemm", "tiles_to_csr", "slice_rows", "wrap", "TsgError",
            "kernel_launch_count", "workspace_release", "transpose"]
 
-_DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8)}
+_DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8),
+       "float32": ("<f4", 4), "float16": ("<f2", 2)}
+# tsg_dtype (include/tsg.h) <-> value type names
+DTYPES = {0: "float64", 1: "float32", 2: "float16"}
+_DTYPE_CODE = {v: k for k, v in DTYPES.items()}
 
 
 class _DeviceArray:
@@ -84,6 +88,7 @@ class Tiles:
     idx: object
     val: object
     stats: dict | None = None
+    dtype: str = "float64"
 
     @property
     def ptr(self) -> C.c_void_p:
@@ -101,15 +106,17 @@ class Tiles:
         P:2991-3057).  Tile format: tile_ptr 8(tm+1) + per tile 4 (col) + 8 (nnz offset) + 16
         (row_ptr) + 32 (mask) + per nonzero 1 (idx) + 8 (val); CSR: 8(m+1) row offsets (int64, reading
         A4) + per nonzero 4 (col) + 8 (val)."""
-        tile = 8 * (self.tile_m + 1) + 8 + 60 * self.num_tiles + 9 * self.nnz
-        csr = 8 * (self.m + 1) + 12 * self.nnz
+        vb = _DT[self.dtype][1]
+        tile = 8 * (self.tile_m + 1) + 8 + 60 * self.num_tiles + (1 + vb) * self.nnz
+        csr = 8 * (self.m + 1) + (4 + vb) * self.nnz
         return {"tile_bytes": tile, "csr_bytes": csr, "ratio": tile / csr if csr else float("nan")}
 
     def copy_to_host(self, out: dict | None = None, stream=None) -> dict:
         """Copy the seven arrays into host buffers (numpy or pinned torch CPU tensors) via the C ABI."""
         sizes = {"tile_ptr": (self.tile_m + 1, np.int64), "tile_col": (self.num_tiles, np.int32),
                  "tile_nnz": (self.num_tiles + 1, np.int64), "row_ptr": (16 * self.num_tiles, np.uint8),
-                 "mask": (16 * self.num_tiles, np.uint16), "idx": (self.nnz, np.uint8), "val": (self.nnz, np.float64)}
+                 "mask": (16 * self.num_tiles, np.uint16), "idx": (self.nnz, np.uint8),
+                 "val": (self.nnz, getattr(np, self.dtype))}
         if out is None:
             out = {k: np.empty(n, dt) for k, (n, dt) in sizes.items()}
         ptrs = []
@@ -135,8 +142,8 @@ def _from_handle(ptr: int, stats=None) -> Tiles:
     return Tiles(h, v.m, v.n, v.tile_m, v.tile_n, v.num_tiles, v.nnz,
                  t(v.tile_ptr, v.tile_m + 1, "int64"), t(v.tile_col, v.num_tiles, "int32"),
                  t(v.tile_nnz, v.num_tiles + 1, "int64"), t(v.row_ptr, 16 * v.num_tiles, "uint8"),
-                 t(v.mask, 16 * v.num_tiles, "uint16"), t(v.idx, v.nnz, "uint8"), t(v.val, v.nnz, "float64"),
-                 stats)
+                 t(v.mask, 16 * v.num_tiles, "uint16"), t(v.idx, v.nnz, "uint8"), t(v.val, v.nnz, DTYPES[v.dtype]),
+                 stats, DTYPES[v.dtype])
 
 
 def _dptr(x, dtype) -> C.c_void_p:
@@ -149,10 +156,11 @@ def _dptr(x, dtype) -> C.c_void_p:
 
 
 def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=None) -> Tiles:
-    """CSR -> sparse tiles on the GPU (tsg_csr_to_tiles).
+    """CSR -> sparse tiles on the GPU (tsg_csr_to_tiles_typed).
 
-    Device input: torch CUDA tensors (int64 row_ptr, int32 col_idx, float64 val).
+    Device input: torch CUDA tensors (int64 row_ptr, int32 col_idx, float64/float32/float16 val).
     Host input: numpy arrays or CPU torch tensors (pinned for speed) -- copied in by the library.
+    The value type is taken from ``val`` (f3: fp32 and fp16 variants).
     """
     torch = _torch()
     m, n = int(shape[0]), int(shape[1])
@@ -163,7 +171,10 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
     if host:
         flags |= _lib.INPUT_HOST
         arrs = []
-        for a, dt in ((row_ptr, np.int64), (col_idx, np.int32), (val, np.float64)):
+        vdt = str(val.dtype).replace("torch.", "") if isinstance(val, torch.Tensor) else np.asarray(val).dtype.name
+        if vdt not in _DTYPE_CODE:
+            vdt = "float64"
+        for a, dt in ((row_ptr, np.int64), (col_idx, np.int32), (val, getattr(np, vdt))):
             if isinstance(a, torch.Tensor):
                 a = a.contiguous()
                 arrs.append((a, C.c_void_p(a.data_ptr() if a.numel() else 0)))
@@ -171,13 +182,16 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
                 a = np.ascontiguousarray(a, dtype=dt)
                 arrs.append((a, C.c_void_p(a.ctypes.data if a.size else 0)))
         nnz = int(arrs[0][0][-1]) if m >= 0 and len(arrs[0][0]) else 0
-        rc = L.tsg_csr_to_tiles(m, n, nnz, arrs[0][1], arrs[1][1], arrs[2][1], flags, None,
-                                C.c_void_p(_stream_ptr(stream)), C.byref(out))
+        rc = L.tsg_csr_to_tiles_typed(m, n, nnz, arrs[0][1], arrs[1][1], arrs[2][1], _DTYPE_CODE[vdt], flags,
+                                      None, C.c_void_p(_stream_ptr(stream)), C.byref(out))
     else:
         nnz = int(col_idx.numel())
-        rc = L.tsg_csr_to_tiles(m, n, nnz, _dptr(row_ptr, torch.int64), _dptr(col_idx, torch.int32),
-                                _dptr(val, torch.float64), flags, None, C.c_void_p(_stream_ptr(stream)),
-                                C.byref(out))
+        vdt = str(val.dtype).replace("torch.", "")
+        if vdt not in _DTYPE_CODE:
+            raise TypeError(f"unsupported value type {val.dtype}")
+        rc = L.tsg_csr_to_tiles_typed(m, n, nnz, _dptr(row_ptr, torch.int64), _dptr(col_idx, torch.int32),
+                                      _dptr(val, val.dtype), _DTYPE_CODE[vdt], flags, None,
+                                      C.c_void_p(_stream_ptr(stream)), C.byref(out))
     _lib.check(rc)
     return _from_handle(out.value)
 
@@ -220,7 +234,7 @@ def transpose(T: Tiles, stream=None) -> Tiles:
 
 
 def tiles_to_csr(T: Tiles, stream=None):
-    """Sparse tiles -> CSR on the GPU; returns (row_ptr int64, col_idx int32, val float64) tensors."""
+    """Sparse tiles -> CSR on the GPU; returns (row_ptr int64, col_idx int32, val of T's dtype) tensors."""
     L = _lib.load()
     torch = _torch()
     rp, ci, v = C.c_void_p(), C.c_void_p(), C.c_void_p()
@@ -234,7 +248,7 @@ def tiles_to_csr(T: Tiles, stream=None):
             return torch.empty(0, dtype=getattr(torch, dt), device="cuda")
         return torch.as_tensor(_DeviceArray(p, count, dt, owner), device="cuda")
 
-    return t(rp.value, T.m + 1, "int64"), t(ci.value, nnz.value, "int32"), t(v.value, nnz.value, "float64")
+    return t(rp.value, T.m + 1, "int64"), t(ci.value, nnz.value, "int32"), t(v.value, nnz.value, T.dtype)
 
 
 class _CsrOwner:
@@ -269,8 +283,12 @@ def wrap(m: int, n: int, arrays: dict, keepalive=None) -> Tiles:
     v.tile_m, v.tile_n = (m + TILE - 1) // TILE, (n + TILE - 1) // TILE
     v.num_tiles = int(arrays["tile_col"].numel())
     v.nnz = int(arrays["val"].numel())
+    vdt = str(arrays["val"].dtype).replace("torch.", "")
+    if vdt not in _DTYPE_CODE:
+        raise TypeError(f"unsupported value type {arrays['val'].dtype}")
+    v.dtype = _DTYPE_CODE[vdt]
     for k, dt in (("tile_ptr", torch.int64), ("tile_col", torch.int32), ("tile_nnz", torch.int64),
-                  ("row_ptr", torch.uint8), ("mask", torch.uint16), ("idx", torch.uint8), ("val", torch.float64)):
+                  ("row_ptr", torch.uint8), ("mask", torch.uint16), ("idx", torch.uint8), ("val", arrays["val"].dtype)):
         setattr(v, k, _dptr(arrays[k], dt).value)
     out = C.c_void_p()
     _lib.check(_lib.load().tsg_tiles_wrap(C.byref(v), None, C.byref(out)))

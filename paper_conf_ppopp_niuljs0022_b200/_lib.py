@@ -42,7 +42,8 @@ class TilesView(C.Structure):
     _fields_ = [("m", C.c_int64), ("n", C.c_int64), ("tile_m", C.c_int64), ("tile_n", C.c_int64),
                 ("num_tiles", C.c_int64), ("nnz", C.c_int64),
                 ("tile_ptr", C.c_void_p), ("tile_col", C.c_void_p), ("tile_nnz", C.c_void_p),
-                ("row_ptr", C.c_void_p), ("mask", C.c_void_p), ("idx", C.c_void_p), ("val", C.c_void_p)]
+                ("row_ptr", C.c_void_p), ("mask", C.c_void_p), ("idx", C.c_void_p), ("val", C.c_void_p),
+                ("dtype", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -65,7 +66,7 @@ class Allocator(C.Structure):
 
 
 # every symbol the header declares (checked by tests/test_abi.py against include/tsg.h)
-SYMBOLS = ["tsg_csr_to_tiles", "tsg_spgemm", "tsg_tiles_to_csr", "tsg_tiles_get_view", "tsg_tiles_wrap",
+SYMBOLS = ["tsg_csr_to_tiles", "tsg_csr_to_tiles_typed", "tsg_spgemm", "tsg_tiles_to_csr", "tsg_tiles_get_view", "tsg_tiles_wrap",
            "tsg_tiles_slice_rows", "tsg_tiles_copy_to_host", "tsg_tiles_destroy", "tsg_free",
            "tsg_status_string", "tsg_last_error", "tsg_abi_version", "tsg_kernel_launch_count",
            "tsg_workspace_release", "tsg_tiles_transpose"]
@@ -86,6 +87,8 @@ def load():
     pp = C.POINTER(C.c_void_p)
     L.tsg_csr_to_tiles.restype = C.c_int
     L.tsg_csr_to_tiles.argtypes = [i64, i64, i64, vp, vp, vp, u32, vp, vp, pp]
+    L.tsg_csr_to_tiles_typed.restype = C.c_int
+    L.tsg_csr_to_tiles_typed.argtypes = [i64, i64, i64, vp, vp, vp, C.c_int32, u32, vp, vp, pp]
     L.tsg_spgemm.restype = C.c_int
     L.tsg_spgemm.argtypes = [vp, vp, u32, vp, vp, pp, C.POINTER(Stats)]
     L.tsg_tiles_to_csr.restype = C.c_int

@@ -185,8 +185,15 @@ int64_t tsg_kernel_launch_count(void) { return g_launches.load(); }
 tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *row_ptr,
                             const int32_t *col_idx, const double *val, uint32_t flags,
                             const tsg_allocator *al, void *stream, tsg_tiles **out) {
+    return tsg_csr_to_tiles_typed(m, n, nnz, row_ptr, col_idx, val, TSG_F64, flags, al, stream, out);
+}
+
+tsg_status tsg_csr_to_tiles_typed(int64_t m, int64_t n, int64_t nnz, const int64_t *row_ptr,
+                                  const int32_t *col_idx, const void *val, int32_t dtype, uint32_t flags,
+                                  const tsg_allocator *al, void *stream, tsg_tiles **out) {
     if (out) *out = nullptr;
     return guarded([&] {
+        TSG_REQUIRE(dtype_ok(dtype), TSG_ERR_INVALID_ARG, "unknown dtype");
         TSG_REQUIRE(out, TSG_ERR_INVALID_ARG, "out is NULL");
         TSG_REQUIRE(m >= 0 && n >= 0 && nnz >= 0, TSG_ERR_INVALID_ARG, "negative size");
         TSG_REQUIRE(row_ptr, TSG_ERR_INVALID_ARG, "row_ptr is NULL");
@@ -202,15 +209,15 @@ tsg_status tsg_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *ro
                 Buffers staging(A, s, true);
                 int64_t *drp = staging.get<int64_t>(m + 1);
                 int32_t *dci = staging.get<int32_t>(nnz);
-                double *dv = staging.get<double>(nnz);
+                void *dv = staging.get<uint8_t>((int64_t)dtype_size(dtype) * nnz);
                 TSG_CUDA(cudaMemcpyAsync(drp, row_ptr, sizeof(int64_t) * (m + 1), cudaMemcpyHostToDevice, s));
                 if (nnz) {
                     TSG_CUDA(cudaMemcpyAsync(dci, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, s));
-                    TSG_CUDA(cudaMemcpyAsync(dv, val, sizeof(double) * nnz, cudaMemcpyHostToDevice, s));
+                    TSG_CUDA(cudaMemcpyAsync(dv, val, dtype_size(dtype) * nnz, cudaMemcpyHostToDevice, s));
                 }
-                launch_csr_to_tiles(m, n, nnz, drp, dci, dv, flags & TSG_VALIDATE, A, s, T);
+                launch_csr_to_tiles(m, n, nnz, drp, dci, dv, dtype, flags & TSG_VALIDATE, A, s, T);
             } else {
-                launch_csr_to_tiles(m, n, nnz, row_ptr, col_idx, val, flags & TSG_VALIDATE, A, s, T);
+                launch_csr_to_tiles(m, n, nnz, row_ptr, col_idx, val, dtype, flags & TSG_VALIDATE, A, s, T);
             }
         } catch (...) {
             destroy_handle(T, s);
@@ -261,7 +268,7 @@ tsg_status tsg_tiles_transpose(const tsg_tiles *T, const tsg_allocator *al, void
 }
 
 tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *stream, int64_t **row_ptr,
-                            int32_t **col_idx, double **val, int64_t *nnz) {
+                            int32_t **col_idx, void **val, int64_t *nnz) {
     if (row_ptr) *row_ptr = nullptr;
     if (col_idx) *col_idx = nullptr;
     if (val) *val = nullptr;
@@ -272,7 +279,7 @@ tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al, void *s
         Buffers out(A, s);
         int64_t *rp = out.get<int64_t>(T->m + 1);
         int32_t *ci = out.get<int32_t>(T->nnz);
-        double *v = out.get<double>(T->nnz);
+        void *v = out.get<uint8_t>((int64_t)T->vsize() * T->nnz);
         launch_tiles_to_csr(T, rp, ci, v, s);
         out.take(rp);
         out.take(ci);
@@ -300,6 +307,7 @@ tsg_status tsg_tiles_get_view(const tsg_tiles *T, tsg_tiles_view *o) {
         o->mask = T->mask;
         o->idx = T->idx;
         o->val = T->val;
+        o->dtype = T->dtype;
     });
 }
 
@@ -311,7 +319,9 @@ tsg_status tsg_tiles_wrap(const tsg_tiles_view *v, const tsg_allocator *owner, t
         TSG_REQUIRE(v->tile_m == ceil_div(v->m, TILE) && v->tile_n == ceil_div(v->n, TILE), TSG_ERR_INVALID_ARG,
                     "tile_m/tile_n inconsistent with m/n");
         TSG_REQUIRE(v->tile_ptr && v->tile_nnz, TSG_ERR_INVALID_ARG, "tile_ptr/tile_nnz NULL");
+        TSG_REQUIRE(dtype_ok(v->dtype), TSG_ERR_INVALID_ARG, "unknown dtype");
         tsg_tiles *T = new tsg_tiles();
+        T->dtype = v->dtype;
         T->m = v->m;
         T->n = v->n;
         T->tm = v->tile_m;
@@ -324,13 +334,13 @@ tsg_status tsg_tiles_wrap(const tsg_tiles_view *v, const tsg_allocator *owner, t
         T->row_ptr = const_cast<uint8_t *>(v->row_ptr);
         T->mask = const_cast<uint16_t *>(v->mask);
         T->idx = const_cast<uint8_t *>(v->idx);
-        T->val = const_cast<double *>(v->val);
+        T->val = const_cast<void *>(v->val);
         if (owner) {
             T->al = Allocator::from(owner);
             TSG_REQUIRE(T->al.custom, TSG_ERR_INVALID_ARG, "owner allocator needs alloc and free");
             size_t b[7] = {sizeof(int64_t) * (size_t)(T->tm + 1), sizeof(int32_t) * (size_t)T->nt,
                            sizeof(int64_t) * (size_t)(T->nt + 1), (size_t)(16 * T->nt),
-                           sizeof(uint16_t) * (size_t)(16 * T->nt), (size_t)T->nnz, sizeof(double) * (size_t)T->nnz};
+                           sizeof(uint16_t) * (size_t)(16 * T->nt), (size_t)T->nnz, T->vsize() * (size_t)T->nnz};
             for (int i = 0; i < 7; i++) {
                 T->owns[i] = true;
                 T->bytes[i] = b[i];
@@ -373,7 +383,8 @@ tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t b, int64_t e, void *
         V->row_ptr = T->row_ptr + 16 * t0;
         V->mask = T->mask + 16 * t0;
         V->idx = T->idx + z0;
-        V->val = T->val + z0;
+        V->val = static_cast<uint8_t *>(T->val) + T->vsize() * (size_t)z0;
+        V->dtype = T->dtype;
         V->al = A;
         V->owns[0] = V->owns[2] = true;
         V->bytes[0] = buf.take(tp);
@@ -383,7 +394,7 @@ tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t b, int64_t e, void *
 }
 
 tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
-                                  int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, double *val) {
+                                  int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, void *val) {
     return guarded([&] {
         TSG_REQUIRE(T, TSG_ERR_INVALID_ARG, "NULL handle");
         cudaStream_t s = (cudaStream_t)stream;
@@ -396,7 +407,7 @@ tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *til
         cp(row_ptr, T->row_ptr, 16 * T->nt);
         cp(mask, T->mask, sizeof(uint16_t) * 16 * T->nt);
         cp(idx, T->idx, T->nnz);
-        cp(val, T->val, sizeof(double) * T->nnz);
+        cp(val, T->val, T->vsize() * T->nnz);
         TSG_CUDA(cudaStreamSynchronize(s));
     });
 }

@@ -85,12 +85,14 @@ __global__ void __launch_bounds__(256) k_c2t_count(int64_t m, int64_t tm, const 
 }
 
 // pass 2: emit the seven arrays
+// values are moved as raw words W of the value type's size (8/4/2 bytes): a permutation
+template <typename W>
 __global__ void __launch_bounds__(256) k_c2t_fill(int64_t m, int64_t tm, const int64_t *__restrict__ rp,
-                                                  const int32_t *__restrict__ ci, const double *__restrict__ v,
+                                                  const int32_t *__restrict__ ci, const W *__restrict__ v,
                                                   const int64_t *__restrict__ tile_ptr, int32_t *__restrict__ tile_col,
                                                   int64_t *__restrict__ tile_nnz, uint8_t *__restrict__ row_ptr,
                                                   uint16_t *__restrict__ mask, uint8_t *__restrict__ idx,
-                                                  double *__restrict__ val) {
+                                                  W *__restrict__ val) {
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t I = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     const bool active = I < tm;
@@ -140,12 +142,13 @@ __global__ void k_set_i64(int64_t *p, int64_t v) { *p = v; }
 
 // tiles -> CSR: lane r of a half owns global row 16I+r; row lengths are popcounts of the row's
 // masks across the tile row; the CSR row offsets follow from the tile row's nonzero base.
+template <typename W>
 __global__ void __launch_bounds__(256) k_t2c(int64_t m, int64_t tm, const int64_t *__restrict__ tile_ptr,
                                              const int32_t *__restrict__ tile_col, const int64_t *__restrict__ tile_nnz,
                                              const uint8_t *__restrict__ row_ptr, const uint16_t *__restrict__ mask,
-                                             const uint8_t *__restrict__ idx, const double *__restrict__ val,
+                                             const uint8_t *__restrict__ idx, const W *__restrict__ val,
                                              int64_t *__restrict__ out_rp, int32_t *__restrict__ out_ci,
-                                             double *__restrict__ out_v) {
+                                             W *__restrict__ out_v) {
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t I = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     const bool active = I < tm;
@@ -178,8 +181,8 @@ __global__ void __launch_bounds__(256) k_t2c(int64_t m, int64_t tm, const int64_
 
 }  // namespace
 
-void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, const int32_t *ci, const double *v,
-                         bool validate, const Allocator &al, cudaStream_t s, tsg_tiles *T) {
+void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, const int32_t *ci, const void *v,
+                         int32_t dtype, bool validate, const Allocator &al, cudaStream_t s, tsg_tiles *T) {
     Buffers tmp(al, s, true), out(al, s);
     const int64_t tm = ceil_div(m, TILE), tn = ceil_div(n, TILE);
     const unsigned grid = grid_for(ceil_div(tm, 2), 8);  // 8 warps x 2 tile rows per CTA
@@ -203,8 +206,20 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
     uint8_t *row_ptr = out.get<uint8_t>(16 * nt);
     uint16_t *mask = out.get<uint16_t>(16 * nt);
     uint8_t *idx = out.get<uint8_t>(nnz);
-    double *val = out.get<double>(nnz);
-    TSG_LAUNCH(k_c2t_fill, grid, 256, 0, s, m, tm, rp, ci, v, tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val);
+    void *val = out.get<uint8_t>((int64_t)dtype_size(dtype) * nnz);
+    switch (dtype_size(dtype)) {
+        case 8:
+            TSG_LAUNCH(k_c2t_fill<uint64_t>, grid, 256, 0, s, m, tm, rp, ci, (const uint64_t *)v, tile_ptr, tile_col,
+                       tile_nnz, row_ptr, mask, idx, (uint64_t *)val);
+            break;
+        case 4:
+            TSG_LAUNCH(k_c2t_fill<uint32_t>, grid, 256, 0, s, m, tm, rp, ci, (const uint32_t *)v, tile_ptr, tile_col,
+                       tile_nnz, row_ptr, mask, idx, (uint32_t *)val);
+            break;
+        default:
+            TSG_LAUNCH(k_c2t_fill<uint16_t>, grid, 256, 0, s, m, tm, rp, ci, (const uint16_t *)v, tile_ptr, tile_col,
+                       tile_nnz, row_ptr, mask, idx, (uint16_t *)val);
+    }
     TSG_LAUNCH(k_set_i64, 1, 1, 0, s, tile_nnz + nt, nnz);
     T->m = m;
     T->n = n;
@@ -212,6 +227,7 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
     T->tn = tn;
     T->nt = nt;
     T->nnz = nnz;
+    T->dtype = dtype;
     void *arr[7] = {tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val};
     T->tile_ptr = tile_ptr;
     T->tile_col = tile_col;
@@ -226,10 +242,21 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
     }
 }
 
-void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, double *v, cudaStream_t s) {
+void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, void *v, cudaStream_t s) {
     const unsigned grid = grid_for(ceil_div(T->tm, 2), 8);
-    TSG_LAUNCH(k_t2c, grid, 256, 0, s, T->m, T->tm, T->tile_ptr, T->tile_col, T->tile_nnz, T->row_ptr, T->mask,
-               T->idx, T->val, rp, ci, v);
+    switch (T->vsize()) {
+        case 8:
+            TSG_LAUNCH(k_t2c<uint64_t>, grid, 256, 0, s, T->m, T->tm, T->tile_ptr, T->tile_col, T->tile_nnz, T->row_ptr,
+                       T->mask, T->idx, (const uint64_t *)T->val, rp, ci, (uint64_t *)v);
+            break;
+        case 4:
+            TSG_LAUNCH(k_t2c<uint32_t>, grid, 256, 0, s, T->m, T->tm, T->tile_ptr, T->tile_col, T->tile_nnz, T->row_ptr,
+                       T->mask, T->idx, (const uint32_t *)T->val, rp, ci, (uint32_t *)v);
+            break;
+        default:
+            TSG_LAUNCH(k_t2c<uint16_t>, grid, 256, 0, s, T->m, T->tm, T->tile_ptr, T->tile_col, T->tile_nnz, T->row_ptr,
+                       T->mask, T->idx, (const uint16_t *)T->val, rp, ci, (uint16_t *)v);
+    }
     TSG_LAUNCH(k_set_i64, 1, 1, 0, s, rp + T->m, T->nnz);
 }
 

@@ -168,6 +168,11 @@ class Buffers {
 
 }  // namespace tsg
 
+namespace tsg {
+inline size_t dtype_size(int32_t d) { return d == TSG_F64 ? 8 : d == TSG_F32 ? 4 : 2; }
+inline bool dtype_ok(int32_t d) { return d == TSG_F64 || d == TSG_F32 || d == TSG_F16; }
+}  // namespace tsg
+
 // ------------------------------------------------------------------------------------------
 // the handle (opaque in the ABI)
 // ------------------------------------------------------------------------------------------
@@ -179,7 +184,9 @@ struct tsg_tiles {
     uint8_t *row_ptr = nullptr;
     uint16_t *mask = nullptr;
     uint8_t *idx = nullptr;
-    double *val = nullptr;
+    void *val = nullptr;
+    int32_t dtype = TSG_F64;  // tsg_dtype of val
+    size_t vsize() const { return tsg::dtype_size(dtype); }
     // ownership: which arrays this handle frees, their byte sizes, and through what
     tsg::Allocator al;
     bool owns[7] = {false, false, false, false, false, false, false};
@@ -208,9 +215,9 @@ int64_t call_launches();
 
 // kernels shared by the API translation units
 void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,
-                         const double *v, bool validate, const Allocator &al, cudaStream_t s,
+                         const void *v, int32_t dtype, bool validate, const Allocator &al, cudaStream_t s,
                          tsg_tiles *out);
-void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, double *v, cudaStream_t s);
+void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, void *v, cudaStream_t s);
 void launch_rebase(const int64_t *src, int64_t *dst, int64_t count, cudaStream_t s);
 void launch_transpose_tiles(const tsg_tiles *T, const Allocator &al, cudaStream_t s, tsg_tiles *O);
 void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Allocator &al,

@@ -90,7 +90,7 @@ struct StepParams {
     const uint16_t *mTA;      // transposed masks
     const uint16_t *colOccA;
     const uint8_t *ixA;
-    const double *vA;
+    const void *vA;           // values: dtype_in (double / float / half)
     // B
     const int64_t *tnzB;
     const uint8_t *rpB;
@@ -98,13 +98,14 @@ struct StepParams {
     const uint16_t *rowOccB;
     const uint16_t *mTB;      // transposed masks (column j of B_KJ: bit c <=> B(c,j) != 0)
     const uint8_t *ixB;
-    const double *vB;
+    const void *vB;
     // C
     int64_t *tnzC;   // step 2: per-tile nnz; step 3: offsets
     uint8_t *rpC;
     uint16_t *mC;
     uint8_t *ixC;
-    double *vC;
+    void *vC;              // values: double for F64 inputs, float for F32 and F16 inputs
+    int dtype_in;          // tsg_dtype of A and B
     const uint32_t *work;  // step-2 class split
     const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
     int dense_threshold;

@@ -47,9 +47,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     reset_call_launches();
     TSG_REQUIRE(A->nt < ((int64_t)1 << 31) && B->nt < ((int64_t)1 << 31), TSG_ERR_OVERFLOW, "input has >= 2^31 tiles");
     TSG_REQUIRE(A->tn == B->tm, TSG_ERR_SHAPE, "tile shapes disagree");
+    TSG_REQUIRE(A->dtype == B->dtype, TSG_ERR_INVALID_ARG, "A and B value types differ");
+    const int32_t dtC = A->dtype == TSG_F64 ? TSG_F64 : TSG_F32;  // F16 x F16 -> F32
     TSG_REQUIRE(((uintptr_t)A->mask & 15) == 0 && ((uintptr_t)B->mask & 15) == 0 && ((uintptr_t)A->row_ptr & 15) == 0 &&
-                    ((uintptr_t)B->row_ptr & 15) == 0 && ((uintptr_t)A->val & 7) == 0 && ((uintptr_t)B->val & 7) == 0,
-                TSG_ERR_INVALID_ARG, "mask and row_ptr arrays must be 16-byte aligned, val 8-byte aligned");
+                    ((uintptr_t)B->row_ptr & 15) == 0 && ((uintptr_t)A->val % A->vsize()) == 0 && ((uintptr_t)B->val % B->vsize()) == 0,
+                TSG_ERR_INVALID_ARG, "mask and row_ptr arrays must be 16-byte aligned, val aligned to its type");
     int TH = (int)((flags >> TSG_DENSE_THRESHOLD_SHIFT) & 0x1ffu);
     if (TH == 0) TH = TSG_DENSE_NNZ;
     Timer tm_;
@@ -185,6 +187,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.colOccA = colOccA;
     P.ixA = A->idx;
     P.vA = A->val;
+    P.dtype_in = A->dtype;
     P.tnzB = B->tile_nnz;
     P.rpB = B->row_ptr;
     P.mB = B->mask;
@@ -213,12 +216,12 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     R.rpA = A->row_ptr;
     R.mA = A->mask;
     R.colOccA = colOccA;
-    R.vA = A->val;
+    R.vA = static_cast<const double *>(A->val);
     R.tpB = B->tile_ptr;
     R.tnzB = B->tile_nnz;
     R.rpB = B->row_ptr;
     R.mB = B->mask;
-    R.vB = B->val;
+    R.vB = static_cast<const double *>(B->val);
     R.pairs = P1.pairs;
     R.pairBeg = pairBeg;
     R.pairCnt = pairCnt;
@@ -228,7 +231,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     R.mC = mask;
     R.dense_threshold = TH;
     R.cnt = cnt;
-    const bool rowk = (flags & TSG_STEP3_ROWS) != 0;
+    const bool rowk = (flags & TSG_STEP3_ROWS) != 0 && A->dtype == TSG_F64;  // the row kernel is fp64 only
     if (rowk) {
         R.rowAcc = tmp.get<int32_t>(tmA);
         R.skip = tmp.get<uint8_t>(ntC);
@@ -245,14 +248,14 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     }
     syncs++;
     uint8_t *idx = out.get<uint8_t>(nnzC);
-    double *val = out.get<double>(nnzC);
+    void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
     tm_.mark(5);
 
     // ---------------- a4: step 3
     P.ixC = idx;
     P.vC = val;
     R.ixC = idx;
-    R.vC = val;
+    R.vC = static_cast<double *>(val);
     if (rowk && hc2.n3rows > 0) launch_step3_rows(R, s);
     if (!rowk || hc2.n3fallback > 0) {
         P.skip = rowk ? R.skip : nullptr;
@@ -274,6 +277,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     C->mask = mask;
     C->idx = idx;
     C->val = val;
+    C->dtype = dtC;
     void *arr[7] = {tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val};
     for (int k = 0; k < 7; k++) {
         C->bytes[k] = out.take(arr[k]);

@@ -23,10 +23,20 @@
 // deterministic (readings A8/A16).
 #include <algorithm>
 
+#include <cuda_fp16.h>
+
 #include "tsg_kernels.cuh"
 
 namespace tsg {
 namespace {
+
+// ---- value types: TI = stored input type, TO = accumulator/output type
+// (double x double -> double, float x float -> float, half x half -> float)
+template <typename TO> __device__ __forceinline__ TO vcvt(double x) { return (TO)x; }
+template <typename TO> __device__ __forceinline__ TO vcvt(float x) { return (TO)x; }
+template <typename TO> __device__ __forceinline__ TO vcvt(__half x) { return (TO)__half2float(x); }
+__device__ __forceinline__ double vfma(double a, double b, double c) { return fma(a, b, c); }
+__device__ __forceinline__ float vfma(float a, float b, float c) { return fmaf(a, b, c); }
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int T2 = 256;    // step-2 CTA
@@ -212,8 +222,11 @@ __device__ __forceinline__ void cp_wait_all() {
 constexpr int TS = 256;  // small-class CTA
 constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <= 16)
 
+template <typename TI, typename TO>
 __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
     __shared__ uint8_t mapsm[TS / 32][SMAP];
+    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
+    TO *vC = static_cast<TO *>(P.vC);
     const int lane = threadIdx.x & 31;
     uint8_t *map = mapsm[threadIdx.x >> 5];
     const int64_t ngroups = (P.ntC + 31) / 32;
@@ -256,7 +269,7 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
                 const int k = q - (int)((rpw >> (8 * (r & 3))) & 0xffu);
                 const int j = (int)__fns((uint32_t)P.mC[t * TILE + r], 0, k + 1);
                 const uint32_t lowj = (1u << j) - 1u;
-                double acc = 0.0;
+                TO acc = 0;
                 // pair p's metadata is loaded while pair p-1 is being multiplied
                 uint64_t prn = pp[0];
                 int64_t pA = (int64_t)(prn >> 32), pB = (int64_t)(uint32_t)prn;
@@ -279,13 +292,13 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
                     while (x) {
                         const int c = __ffs(x) - 1;
                         x &= x - 1;
-                        const double a = P.vA[czA + __popc(cmA & ((1u << c) - 1u))];
-                        const double b = P.vB[czB + P.rpB[cB * TILE + c] + __popc((uint32_t)P.mB[cB * TILE + c] & lowj)];
-                        acc = fma(a, b, acc);
+                        const TO a = vcvt<TO>(vA[czA + __popc(cmA & ((1u << c) - 1u))]);
+                        const TO b = vcvt<TO>(vB[czB + P.rpB[cB * TILE + c] + __popc((uint32_t)P.mB[cB * TILE + c] & lowj)]);
+                        acc = vfma(a, b, acc);
                     }
                 }
                 P.ixC[o] = (uint8_t)((r << 4) | j);
-                P.vC[o] = acc;
+                vC[o] = acc;
             }
         }
         __syncwarp();
@@ -296,58 +309,59 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
 // with c in mask_A_i[r] & rowOcc(B_i): a = A_i(r,c) and B_i's row c (mask, first three values,
 // pointer to the rest).  Items come pair-ascending then c-ascending, so every C(r,j) receives its
 // products in ascending k.
+template <typename TI, typename TO>
 struct ItemStream {
     uint32_t rel;  // batch pairs that touch row r (mask_A_i[r] & rowOcc(B_i) != 0), not yet started
     int pi = 0;
     uint32_t mAr = 0, ma = 0;
-    const double *va = nullptr, *vbt = nullptr;
+    const TI *va = nullptr, *vbt = nullptr;
     // next item -> (a, b0..b2, mb, vb); false when the batch is exhausted
-    __device__ __forceinline__ bool fetch(const StepParams &P, const MedStage &S, int r, double &a, double &b0,
-                                          double &b1, double &b2, uint32_t &mb, const double *&vb) {
+    __device__ __forceinline__ bool fetch(const StepParams &P, const MedStage &S, int r, TO &a, TO &b0, TO &b1,
+                                          TO &b2, uint32_t &mb, const TI *&vb) {
         if (!ma) {
             if (!rel) return false;
             pi = __ffs(rel) - 1;
             rel &= rel - 1;
             mAr = S.mA[pi][r];
             ma = mAr & S.oB[pi];
-            va = P.vA + S.zA[pi] + S.rA[pi][r];
-            vbt = P.vB + S.zB[pi];
+            va = static_cast<const TI *>(P.vA) + S.zA[pi] + S.rA[pi][r];
+            vbt = static_cast<const TI *>(P.vB) + S.zB[pi];
         }
         const int c = __ffs(ma) - 1;
         ma &= ma - 1;
-        a = va[__popc(mAr & ((1u << c) - 1u))];
+        a = vcvt<TO>(va[__popc(mAr & ((1u << c) - 1u))]);
         mb = S.mB[pi][c];
         vb = vbt + S.rB[pi][c];
         const int n = __popc(mb);  // >= 1: row c of B_i is non-empty (rowOcc filter)
-        b0 = vb[0];
-        b1 = n > 1 ? vb[1] : 0.0;
-        b2 = n > 2 ? vb[2] : 0.0;
+        b0 = vcvt<TO>(vb[0]);
+        b1 = n > 1 ? vcvt<TO>(vb[1]) : (TO)0;
+        b2 = n > 2 ? vcvt<TO>(vb[2]) : (TO)0;
         return true;
     }
 };
 
 // acc[16 j] += a * B(c, j) over B's row c in ascending j; the first three slots are distinct, so
 // their loads, FMAs and stores are independent
-__device__ __forceinline__ void accumulate_row(double a, double b0, double b1, double b2, uint32_t mb,
-                                               const double *vb, double *acc) {
+template <typename TI, typename TO>
+__device__ __forceinline__ void accumulate_row(TO a, TO b0, TO b1, TO b2, uint32_t mb, const TI *vb, TO *acc) {
     const int j0 = __ffs(mb) - 1;
     uint32_t m = mb & (mb - 1);
     const int j1 = __ffs(m) - 1;
     m &= m - 1;
     const int j2 = __ffs(m) - 1;
     m &= m - 1;
-    double *p0 = acc + j0 * 16;
-    double *p1 = acc + (j1 >= 0 ? j1 : j0) * 16;
-    double *p2 = acc + (j2 >= 0 ? j2 : j0) * 16;
-    const double c0 = *p0, c1 = *p1, c2 = *p2;
-    *p0 = fma(a, b0, c0);
-    if (j1 >= 0) *p1 = fma(a, b1, c1);
-    if (j2 >= 0) *p2 = fma(a, b2, c2);
-    const double *q = vb + 3;
+    TO *p0 = acc + j0 * 16;
+    TO *p1 = acc + (j1 >= 0 ? j1 : j0) * 16;
+    TO *p2 = acc + (j2 >= 0 ? j2 : j0) * 16;
+    const TO c0 = *p0, c1 = *p1, c2 = *p2;
+    *p0 = vfma(a, b0, c0);
+    if (j1 >= 0) *p1 = vfma(a, b1, c1);
+    if (j2 >= 0) *p2 = vfma(a, b2, c2);
+    const TI *q = vb + 3;
     while (m) {
         const int j = __ffs(m) - 1;
         m &= m - 1;
-        acc[j * 16] = fma(a, *q++, acc[j * 16]);
+        acc[j * 16] = vfma(a, vcvt<TO>(*q++), acc[j * 16]);
     }
 }
 
@@ -382,7 +396,8 @@ struct MedMeta {
     }
 };
 
-__device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M, double *acc, MedStage &S, int r) {
+template <typename TI, typename TO>
+__device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M, TO *acc, MedStage &S, int r) {
     const uint32_t np = M.np, mCr = M.mCr;
     const uint64_t *pp = M.pp;
     {
@@ -390,7 +405,7 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
         while (m) {
             const int j = __ffs(m) - 1;
             m &= m - 1;
-            acc[j * 16] = 0.0;
+            acc[j * 16] = (TO)0;
         }
     }
     const uint32_t nbat = (np + BATCH3 - 1) / BATCH3;
@@ -414,12 +429,12 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
         __syncwarp();
         const int nb = np > bt * BATCH3 ? (int)min((uint32_t)BATCH3, np - bt * BATCH3) : 0;
         if (mCr) {
-            ItemStream it;
+            ItemStream<TI, TO> it;
             it.rel = 0;
             for (int i = 0; i < nb; i++) it.rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
-            double aX, bX0, bX1, bX2, aY, bY0, bY1, bY2;
+            TO aX, bX0, bX1, bX2, aY, bY0, bY1, bY2;
             uint32_t mX, mY;
-            const double *vX, *vY;
+            const TI *vX, *vY;
             bool hX = it.fetch(P, S, r, aX, bX0, bX1, bX2, mX, vX);
             while (hX) {
                 const bool hY = it.fetch(P, S, r, aY, bY0, bY1, bY2, mY, vY);
@@ -439,7 +454,7 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
             const int j = __ffs(m) - 1;
             m &= m - 1;
             P.ixC[ob + qq] = (uint8_t)((r << 4) | j);
-            P.vC[ob + qq] = acc[j * 16];
+            static_cast<TO *>(P.vC)[ob + qq] = acc[j * 16];
             qq++;
         }
     }
@@ -451,34 +466,57 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
 // mask_C at the end.  Structurally absent A entries are skipped; absent B entries
 // are staged as 0 so a finite a adds an exact +-0 (value unchanged); a non-finite a falls back to
 // mask-predicated FMAs so Inf*0 never appears.
+// eight consecutive accumulator-type values from shared memory (16-byte vector loads)
+__device__ __forceinline__ void lds8(const double *p, double (&b)[8]) {
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+        const double2 v = reinterpret_cast<const double2 *>(p)[k];
+        b[2 * k] = v.x;
+        b[2 * k + 1] = v.y;
+    }
+}
+__device__ __forceinline__ void lds8(const float *p, float (&b)[8]) {
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+        const float4 v = reinterpret_cast<const float4 *>(p)[k];
+        b[4 * k] = v.x;
+        b[4 * k + 1] = v.y;
+        b[4 * k + 2] = v.z;
+        b[4 * k + 3] = v.w;
+    }
+}
+
+template <typename TI, typename TO>
 __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigned char *wr, int lane) {
     constexpr int AP = 17;  // padded row pitch of the staged A tile (conflict-free column reads)
-    double *Ad = reinterpret_cast<double *>(wr);
-    double *Bd = Ad + TILE * AP;  // byte offset 2176: 16-byte aligned
+    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
+    TO *Ad = reinterpret_cast<TO *>(wr);
+    TO *Bd = reinterpret_cast<TO *>(wr + 2176);  // after 16 x 17 doubles: 16-byte aligned
     const int r = lane >> 1, h = lane & 1;
-    double acc[8];
+    TO acc[8];
 #pragma unroll
-    for (int j = 0; j < 8; j++) acc[j] = 0.0;
+    for (int j = 0; j < 8; j++) acc[j] = (TO)0;
     const uint64_t *pp = P.pairs + P.pairBeg[t];
     const uint32_t np = P.pairCnt[t];
     // A is read only at its structural positions (c in mask_A[r]), so it is never cleared; B is
-    // cleared per pair (four 16-byte stores per lane) and its nonzeros scattered over it
+    // cleared per pair (16-byte stores) and its nonzeros scattered over it
     for (uint32_t p = 0; p < np; p++) {
         const uint64_t pr = pp[p];
         const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
 #pragma unroll
-        for (int e = lane; e < TILE * TILE / 2; e += 32) reinterpret_cast<double2 *>(Bd)[e] = make_double2(0.0, 0.0);
+        for (int e = lane; e < TILE * TILE * (int)sizeof(TO) / 16; e += 32)
+            reinterpret_cast<uint4 *>(Bd)[e] = make_uint4(0u, 0u, 0u, 0u);
         __syncwarp();
         bool nf = false;
         for (int64_t e = P.tnzA[pA] + lane; e < P.tnzA[pA + 1]; e += 32) {
             const uint32_t ix = P.ixA[e];
-            const double v = P.vA[e];
+            const TO v = vcvt<TO>(vA[e]);
             nf |= !isfinite(v);
             Ad[(ix >> 4) * AP + (ix & 15)] = v;
         }
         for (int64_t e = P.tnzB[pB] + lane; e < P.tnzB[pB + 1]; e += 32) {
             const uint32_t ix = P.ixB[e];
-            Bd[(ix >> 4) * TILE + (ix & 15)] = P.vB[e];
+            Bd[(ix >> 4) * TILE + (ix & 15)] = vcvt<TO>(vB[e]);
         }
         const uint32_t mA = P.mA[pA * TILE + r];
         const bool anynf = __any_sync(FULL, nf);
@@ -487,25 +525,22 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
 #pragma unroll
             for (int c = 0; c < TILE; c++) {
                 if ((mA >> c) & 1u) {
-                    const double a = Ad[r * AP + c];
-                    const double2 *bp = reinterpret_cast<const double2 *>(Bd + c * TILE + 8 * h);
+                    const TO a = Ad[r * AP + c];
+                    TO b[8];
+                    lds8(Bd + c * TILE + 8 * h, b);
 #pragma unroll
-                    for (int jj = 0; jj < 4; jj++) {
-                        const double2 b2 = bp[jj];
-                        acc[2 * jj] = fma(a, b2.x, acc[2 * jj]);
-                        acc[2 * jj + 1] = fma(a, b2.y, acc[2 * jj + 1]);
-                    }
+                    for (int jj = 0; jj < 8; jj++) acc[jj] = vfma(a, b[jj], acc[jj]);
                 }
             }
         } else {
             const uint16_t *mbt = P.mB + pB * TILE;
             for (int c = 0; c < TILE; c++) {
                 if ((mA >> c) & 1u) {
-                    const double a = Ad[r * AP + c];
+                    const TO a = Ad[r * AP + c];
                     const uint32_t mb = (uint32_t)mbt[c] >> (8 * h);
 #pragma unroll
                     for (int jj = 0; jj < 8; jj++)
-                        if ((mb >> jj) & 1u) acc[jj] = fma(a, Bd[c * TILE + 8 * h + jj], acc[jj]);
+                        if ((mb >> jj) & 1u) acc[jj] = vfma(a, Bd[c * TILE + 8 * h + jj], acc[jj]);
                 }
             }
         }
@@ -519,12 +554,13 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
         if ((mC >> j) & 1u) {
             const int q = __popc(mC & ((1u << j) - 1u));
             P.ixC[ob + q] = (uint8_t)((r << 4) | j);
-            P.vC[ob + q] = acc[jj];
+            static_cast<TO *>(P.vC)[ob + q] = acc[jj];
         }
     }
     __syncwarp();
 }
 
+template <typename TI, typename TO>
 __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
     __shared__ MedStage med[T3 / 16];
@@ -542,7 +578,7 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         const unsigned dm = __ballot_sync(FULL, dense);
         unsigned mm = __ballot_sync(FULL, v) & ~sm & ~dm;
         // medium tiles: two at a time, a half warp each
-        double *acc = reinterpret_cast<double *>(wr) + half * (TILE * TILE) + r;
+        TO *acc = reinterpret_cast<TO *>(wr) + half * (TILE * TILE) + r;
         auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
             const int f0 = __ffs(mm) - 1;
             mm &= mm - 1;
@@ -556,7 +592,7 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
             for (;;) {
                 const bool more = mm != 0;  // warp-uniform
                 if (more) nxt.load(P, pop2(), g, r);
-                s3_medium(P, cur, acc, med[threadIdx.x >> 4], r);
+                s3_medium<TI, TO>(P, cur, acc, med[threadIdx.x >> 4], r);
                 if (!more) break;
                 cur = nxt;
             }
@@ -566,7 +602,7 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         while (dd) {
             const int f = __ffs(dd) - 1;
             dd &= dd - 1;
-            s3_dense(P, g * 32 + f, wr, lane);
+            s3_dense<TI, TO>(P, g * 32 + f, wr, lane);
         }
         const unsigned vm = __ballot_sync(FULL, v);
         if (lane == 0) {
@@ -590,10 +626,19 @@ void launch_step2(const StepParams &P, cudaStream_t s) {
     TSG_LAUNCH(k_s2, grid_groups(P.ntC, T2 / 32), T2, 0, s, P);
 }
 
+template <typename TI, typename TO>
+static void launch_step3_t(const StepParams &P, cudaStream_t s) {
+    if (P.small_max > 0) TSG_LAUNCH((k_s3_small<TI, TO>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
+    TSG_LAUNCH((k_s3<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
+}
+
 void launch_step3(const StepParams &P, cudaStream_t s) {
     if (P.ntC <= 0) return;
-    if (P.small_max > 0) TSG_LAUNCH(k_s3_small, grid_groups(P.ntC, TS / 32), TS, 0, s, P);
-    TSG_LAUNCH(k_s3, grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
+    switch (P.dtype_in) {
+        case TSG_F64: launch_step3_t<double, double>(P, s); break;
+        case TSG_F32: launch_step3_t<float, float>(P, s); break;
+        default: launch_step3_t<__half, float>(P, s);
+    }
 }
 
 }  // namespace tsg

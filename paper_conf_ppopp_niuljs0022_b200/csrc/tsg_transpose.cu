@@ -58,11 +58,12 @@ __global__ void k_tp_nnz(int64_t nt, const int64_t *__restrict__ perm, const int
 }
 
 // thread per tile of A^T: transpose source tile perm[d] (whose column masks are maskTs)
+template <typename W>  // raw value words (8/4/2 bytes): a permutation of T's values
 __global__ void k_tp_fill(int64_t nt, const int64_t *__restrict__ perm, const int64_t *__restrict__ tnz,
                           const uint16_t *__restrict__ mask, const uint16_t *__restrict__ maskTs,
-                          const double *__restrict__ val, const int64_t *__restrict__ tnzT,
+                          const W *__restrict__ val, const int64_t *__restrict__ tnzT,
                           uint8_t *__restrict__ rpT, uint16_t *__restrict__ maskT, uint8_t *__restrict__ idxT,
-                          double *__restrict__ valT) {
+                          W *__restrict__ valT) {
     const int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (d >= nt) return;
     const int64_t t = perm[d];
@@ -124,15 +125,27 @@ void launch_transpose_tiles(const tsg_tiles *T, const Allocator &al, cudaStream_
     uint8_t *rpT = out.get<uint8_t>(TILE * nt);
     uint16_t *maskT = out.get<uint16_t>(TILE * nt);
     uint8_t *idxT = out.get<uint8_t>(T->nnz);
-    double *valT = out.get<double>(T->nnz);
-    TSG_LAUNCH(k_tp_fill, grid_for(nt, 128), 128, 0, s, nt, perm, T->tile_nnz, T->mask, mTs, T->val, tnzT, rpT, maskT,
-               idxT, valT);
+    void *valT = out.get<uint8_t>((int64_t)T->vsize() * T->nnz);
+    switch (T->vsize()) {
+        case 8:
+            TSG_LAUNCH(k_tp_fill<uint64_t>, grid_for(nt, 128), 128, 0, s, nt, perm, T->tile_nnz, T->mask, mTs,
+                       (const uint64_t *)T->val, tnzT, rpT, maskT, idxT, (uint64_t *)valT);
+            break;
+        case 4:
+            TSG_LAUNCH(k_tp_fill<uint32_t>, grid_for(nt, 128), 128, 0, s, nt, perm, T->tile_nnz, T->mask, mTs,
+                       (const uint32_t *)T->val, tnzT, rpT, maskT, idxT, (uint32_t *)valT);
+            break;
+        default:
+            TSG_LAUNCH(k_tp_fill<uint16_t>, grid_for(nt, 128), 128, 0, s, nt, perm, T->tile_nnz, T->mask, mTs,
+                       (const uint16_t *)T->val, tnzT, rpT, maskT, idxT, (uint16_t *)valT);
+    }
     O->m = T->n;
     O->n = T->m;
     O->tm = tmT;
     O->tn = tnT;
     O->nt = nt;
     O->nnz = T->nnz;
+    O->dtype = T->dtype;
     O->tile_ptr = tpT;
     O->tile_col = tcolT;
     O->tile_nnz = tnzT;

@@ -60,18 +60,25 @@ def _wire(t):
 def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, group=None):
     """Broadcast the seven arrays of a tile matrix from ``src``; returns (meta, arrays) everywhere.
 
-    meta = (m, n, num_tiles, nnz).  On non-src ranks pass arrays=None, meta=None.
+    meta = (m, n, num_tiles, nnz) for fp64 values, or (m, n, num_tiles, nnz, dtype) with dtype a
+    torch value type (f3).  On non-src ranks pass arrays=None, meta=None; they receive the 4-tuple
+    for fp64 and the 5-tuple otherwise.
     """
     import torch
     import torch.distributed as dist
 
-    mt = torch.tensor(list(meta) if meta is not None else [0, 0, 0, 0], dtype=torch.int64, device=device)
+    codes = [torch.float64, torch.float32, torch.float16]
+    if meta is not None:
+        vals = list(meta[:4]) + [codes.index(meta[4]) if len(meta) > 4 else 0]
+    else:
+        vals = [0, 0, 0, 0, 0]
+    mt = torch.tensor(vals, dtype=torch.int64, device=device)
     dist.broadcast(mt, src, group=group)
-    m, n, nt, nnz = (int(x) for x in mt.tolist())
+    m, n, nt, nnz, dc = (int(x) for x in mt.tolist())
     tm = (m + TILE - 1) // TILE
     shapes = {"tile_ptr": (tm + 1, torch.int64), "tile_col": (nt, torch.int32), "tile_nnz": (nt + 1, torch.int64),
               "row_ptr": (16 * nt, torch.uint8), "mask": (32 * nt, torch.uint8), "idx": (nnz, torch.uint8),
-              "val": (nnz, torch.float64)}
+              "val": (nnz, codes[dc])}
     out = {}
     for k in ARRAYS:
         if arrays is not None:
@@ -81,7 +88,7 @@ def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, g
         if t.numel():
             dist.broadcast(t, src, group=group)
         out[k] = t.view(torch.uint16) if k == "mask" else t
-    return (m, n, nt, nnz), out
+    return ((m, n, nt, nnz) if dc == 0 else (m, n, nt, nnz, codes[dc])), out
 
 
 def allgatherv(t, group=None):

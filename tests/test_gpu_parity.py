@@ -393,3 +393,53 @@ def test_space_and_peak_memory_reporting(tsg):
         st = C.stats
         assert st["bytes_out"] >= C.space()["tile_bytes"]
         assert st["bytes_scratch"] > 0
+
+
+# ------------------------------------------------------------------------------------------
+# f3: precision variants (fp32, and the paper's half-in / single-out setup)
+# ------------------------------------------------------------------------------------------
+def _typed(A, np_dtype):
+    return gen.CSR(A.m, A.n, A.rowptr, A.col, A.val.astype(np_dtype), A.name)
+
+
+PREC_CASES = [("C1", gen.config("C1")), ("stencil27-10", gen.stencil27(10)),
+              ("strip-fem-8x30", gen.strip_fem(8, 30, 6)), ("rmat-12", gen.rmat(12)),
+              ("dense-64", gen.dense_block(64, 64)),
+              ("hub", gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004))]
+
+
+@pytest.mark.parametrize("np_dtype", [np.float32, np.float16], ids=["f32", "f16"])
+@pytest.mark.parametrize("name,A", PREC_CASES, ids=[c[0] for c in PREC_CASES])
+def test_precision_variants_match_oracle(tsg, name, A, np_dtype):
+    """Steps 1-2 are value-free; step 3 in fp32 (fp16 inputs widened exactly) sums in ascending k
+    with fmaf, so the result equals the oracle's single-precision fma loop bit for bit."""
+    At = _typed(A, np_dtype)
+    T = tiles_of(tsg, At)
+    assert T.dtype == np.dtype(np_dtype).name and T.val.dtype == getattr(__import__("torch"), T.dtype)
+    assert np.array_equal(T.val.cpu().numpy(), oracle.csr_to_tiles(A).val.astype(np_dtype))
+    for th in (None, 1):  # default classes, and every tile through the dense accumulator
+        C = tsg.spgemm(T, T, stats=True, dense_threshold=th)
+        assert C.dtype == "float32"
+        ref = oracle.expected_tiles(At, At, fma=True, prec="f32")
+        got = host(C)
+        assert_tiles_equal(got, ref, values=None)
+        assert got["val"].dtype == np.float32
+        assert bitwise_equal_values(got["val"].astype(np.float64), ref.val.astype(np.float64)), (name, th)
+    # the other entry points keep the value type
+    rp, ci, v = tsg.tiles_to_csr(C)
+    O = oracle.spgemm(At, At, fma=True, prec="f32")
+    assert v.dtype == __import__("torch").float32 and np.array_equal(v.cpu().numpy(), O.val)
+    TT = tsg.transpose(T)
+    assert TT.dtype == T.dtype
+    ref_t = oracle.csr_to_tiles(oracle.transpose(A))
+    assert np.array_equal(TT.val.cpu().numpy(), ref_t.val.astype(np_dtype))
+    h = T.copy_to_host()
+    assert h["val"].dtype == np.dtype(np_dtype) and np.array_equal(h["val"], T.val.cpu().numpy())
+
+
+def test_mixed_precision_inputs_rejected(tsg):
+    A = gen.config("C1")
+    T64, T32 = tiles_of(tsg, A), tiles_of(tsg, _typed(A, np.float32))
+    with pytest.raises(tsg.TsgError) as e:
+        tsg.spgemm(T64, T32)
+    assert e.value.name == "TSG_ERR_INVALID_ARG"

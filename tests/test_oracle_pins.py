@@ -373,3 +373,77 @@ def test_transpose_involution_and_product_rule():
     QT = oracle.transpose(Q)
     assert np.array_equal(Q.rowptr, QT.rowptr) and np.array_equal(Q.col, QT.col)
     assert np.allclose(Q.val, QT.val, rtol=0, atol=1e-12 * np.abs(Q.val).max())
+
+
+# ------------------------------------------------------------------------------------------
+# O1 in single precision (the paper's Section 4.7 half-in / single-out setup,
+# P:3143-3152)
+# ------------------------------------------------------------------------------------------
+def _with_values(A, vals):
+    return gen.CSR(A.m, A.n, A.rowptr, A.col, vals, A.name)
+
+
+def test_gustavson_f32_exact_on_small_integers():
+    """Integers with |sums| < 2^24 are exact in fp32: the f32 loop must equal the fp64 one."""
+    rng = np.random.default_rng(5)
+    for m, k, n in ((16, 16, 16), (40, 33, 27)):
+        A = gen.random_sparse(m, k, 0.3, seed=m + 1)
+        B = gen.random_sparse(k, n, 0.3, seed=n + 2)
+        A = _with_values(A, rng.integers(-8, 9, A.col.size).astype(np.float64))
+        B = _with_values(B, rng.integers(-8, 9, B.col.size).astype(np.float64))
+        for fma in (False, True):
+            C64 = oracle.spgemm(A, B, fma=fma)
+            C32 = oracle.spgemm(A, B, fma=fma, prec="f32")
+            assert C32.val.dtype == np.float32
+            assert np.array_equal(C32.rowptr, C64.rowptr) and np.array_equal(C32.col, C64.col)
+            assert np.array_equal(C32.val.astype(np.float64), C64.val)
+
+
+def test_gustavson_f32_within_rounding_bound():
+    """Random values: |c32 - c64| <= (k+1) * 2^-24 * sum|a*b| per entry (k = products of the
+    entry; standard recursive-summation bound with fp32 inputs rounded first), and the fp64
+    products of the fp32-rounded inputs bound the abs sums."""
+    A = gen.random_sparse(70, 60, 0.15, seed=3)
+    B = gen.random_sparse(60, 50, 0.15, seed=4)
+    A32 = _with_values(A, A.val.astype(np.float32).astype(np.float64))
+    B32 = _with_values(B, B.val.astype(np.float32).astype(np.float64))
+    ref = oracle.spgemm(A32, B32)  # exact-input fp64 reference
+    ones = oracle.spgemm(_with_values(A, np.ones_like(A.val)), _with_values(B, np.ones_like(B.val)))
+    k = ones.val  # products per entry
+    for fma in (False, True):
+        C32 = oracle.spgemm(A, B, fma=fma, prec="f32")
+        assert np.array_equal(C32.col, ref.col)
+        err = np.abs(C32.val.astype(np.float64) - ref.val)
+        assert np.all(err <= (k + 1) * 2.0 ** -24 * ref.abs + 1e-300)
+        assert np.allclose(C32.abs, ref.abs, rtol=1e-15, atol=0)
+
+
+def test_gustavson_f16_inputs_widen_exactly():
+    """Half inputs are widened to fp32 exactly: the f32 product of float16 values
+    equals the f32 product of the same values given as float32, and matches the dense fp64 product
+    of the half-rounded matrices within the fp32 bound."""
+    A = gen.random_sparse(33, 35, 0.2, seed=8)
+    B = gen.random_sparse(35, 31, 0.2, seed=9)
+    Ah, Bh = _with_values(A, A.val.astype(np.float16)), _with_values(B, B.val.astype(np.float16))
+    Af, Bf = _with_values(A, Ah.val.astype(np.float32)), _with_values(B, Bh.val.astype(np.float32))
+    Ch = oracle.spgemm(Ah, Bh, fma=True, prec="f32")
+    Cf = oracle.spgemm(Af, Bf, fma=True, prec="f32")
+    assert np.array_equal(Ch.val, Cf.val)
+    D = csr_dense(A.m, A.n, A.rowptr, A.col, Ah.val.astype(np.float64)) @ \
+        csr_dense(B.m, B.n, B.rowptr, B.col, Bh.val.astype(np.float64))
+    got = csr_dense(Ch.m, Ch.n, Ch.rowptr, Ch.col, Ch.val.astype(np.float64))
+    absd = np.abs(csr_dense(A.m, A.n, A.rowptr, A.col, Ah.val.astype(np.float64))) @ \
+        np.abs(csr_dense(B.m, B.n, B.rowptr, B.col, Bh.val.astype(np.float64)))
+    assert np.all(np.abs(got - D) <= (A.n + 1) * 2.0 ** -24 * absd + 1e-300)
+
+
+def test_gustavson_f32_accumulates_in_single_precision():
+    """Closed form: products 1, 2^-24, 2^-24 summed in ascending k.  In fp32 each 1 + 2^-24 is a
+    tie and rounds to even (1.0), so the result is exactly 1.0; in fp64 it is 1 + 2^-23.  A loop
+    that accumulated in fp64 and rounded once would give 1 + 2^-23 (the next float above 1)."""
+    e = 2.0 ** -12
+    A = gen.from_coo(1, 3, [0, 0, 0], [0, 1, 2], [1.0, e, e])
+    B = gen.from_coo(3, 1, [0, 1, 2], [0, 0, 0], [1.0, e, e])
+    for fma in (False, True):
+        assert oracle.spgemm(A, B, fma=fma, prec="f32").val.tolist() == [1.0]
+        assert oracle.spgemm(A, B, fma=fma).val.tolist() == [1.0 + 2.0 ** -23]
