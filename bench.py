@@ -31,7 +31,8 @@ sys.path.insert(0, ROOT)
 METRIC = "fp64 C=A^2 GFLOPS (2×products/time) at 1/2/4/8 B200; % HBM roofline"
 UNIT = "GFLOPS"
 L2_BYTES = 126 * 2 ** 20
-ROW_BLOCKS = {"C5": 4}  # tile-row blocks per step on one GPU (C5's C is ~144 GB in tile form)
+ROW_BLOCKS = {"C5": 4}
+VDT = {"f64": np.float64, "f32": np.float32, "f16": np.float16}  # tile-row blocks per step on one GPU (C5's C is ~144 GB in tile form)
 
 
 def peaks():
@@ -42,9 +43,9 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def tile_bytes(tm, ntiles, nnz):
-    """S(M) = 8(tm+1) + 60*tiles + 9*nnz."""
-    return 8 * (tm + 1) + 60 * ntiles + 9 * nnz
+def tile_bytes(tm, ntiles, nnz, vbytes=8):
+    """S(M) = 8(tm+1) + 60*tiles + (1 + value bytes)*nnz  (9*nnz for fp64)."""
+    return 8 * (tm + 1) + 60 * ntiles + (1 + vbytes) * nnz
 
 
 class ClockSampler:
@@ -103,7 +104,7 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None):
+def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str = "f64"):
     """The oracle as it stands (single thread) on a bounded row sample of A*B (B = A by default)."""
     import oracle
 
@@ -113,7 +114,7 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None):
     # calibrate on a small row block, then size the sample to ~budget_s seconds
     probe = np.arange(0, min(m, 256), dtype=np.int64)
     t0 = time.perf_counter()
-    oracle.spgemm(A, B, rows=probe)
+    oracle.spgemm(A, B, rows=probe, prec=prec)
     dt = max(time.perf_counter() - t0, 1e-4)
     rows_per_s = len(probe) / dt
     R = int(min(m, max(len(probe), rows_per_s * budget_s)))
@@ -123,7 +124,7 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None):
     sub = gen_row_block(A, R)
     prods = oracle.products(sub, B)
     t0 = time.perf_counter()
-    C = oracle.spgemm(A, B, rows=rows)
+    C = oracle.spgemm(A, B, rows=rows, prec=prec)
     el = time.perf_counter() - t0
     return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
@@ -144,20 +145,24 @@ def run_reference(args):
     from workloads import gen
 
     A = gen.config(args.config)
+    if args.dtype != "f64":
+        A = gen.CSR(A.m, A.n, A.rowptr, A.col, A.val.astype(VDT[args.dtype]), A.name)
+    prec = "f64" if args.dtype == "f64" else "f32"
     B = _csr_transpose(A) if args.aat else A
     for _ in range(args.warmup):
-        oracle_baseline(A, budget_s=2.0, B=B)
+        oracle_baseline(A, budget_s=2.0, B=B, prec=prec)
     vals, secs, prods = [], 0.0, 0
     last = None
     for _ in range(args.steps):
-        last = oracle_baseline(A, budget_s=args.ref_step_s, B=B)
+        last = oracle_baseline(A, budget_s=args.ref_step_s, B=B, prec=prec)
         vals.append(last["value"])
         secs += last["seconds"]
         prods += last["products"]
     value = 2.0 * prods / secs / 1e9
     line = {"impl": "reference", "metric": _metric(args), "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": {"f64": "f64", "f32": "f32", "f16": "f16 in, f32 accumulate/out"}[args.dtype], "data": "synthetic",
             "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}" + (", C = A*A^T" if args.aat else ""),
                        "n": A.m, "nnz_a": A.nnz},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": last["sample"]},
@@ -182,6 +187,9 @@ def main():
     ap.add_argument("--aat", action="store_true",
                     help="C = A * A^T (the paper's second workload, SURVEY f1); A^T is formed once with "
                          "tsg_tiles_transpose outside the timed region, like the CSR->tile conversion")
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32", "f16"],
+                    help="value type (SURVEY f3): f64 (BASELINE's metric), f32, or f16 inputs with f32 "
+                         "accumulation/output (the paper's Section 4.7 setup, P:3143-3152)")
     ap.add_argument("--row-blocks", type=int, default=0,
                     help="compute each rank's C in this many tile-row blocks, one after the other (0 = "
                          "config default: C5 needs 4 on one GPU, its C alone is ~144 GB in tile form)")
@@ -208,6 +216,10 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     A = gen.config(args.config)
+    if args.dtype != "f64":
+        A = gen.CSR(A.m, A.n, A.rowptr, A.col, A.val.astype(VDT[args.dtype]), A.name)
+    vb = np.dtype(VDT[args.dtype]).itemsize  # value bytes of A and B
+    cb = 8 if args.dtype == "f64" else 4     # value bytes of C
     stream = torch.cuda.current_stream()
     T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.col).to(dev),
                          torch.from_numpy(A.val).to(dev), (A.m, A.n))
@@ -293,11 +305,12 @@ def main():
     nnzC, ntC = stats_last["nnz_c"], stats_last["tiles_c"]
     steps_ms = {"step1": float(np.mean(s1_ms)), "step2": float(np.mean(s2_ms)), "step3": float(np.mean(s3_ms))}
     alloc_ms = float(np.mean(sa_ms))
-    alg = {  # algorithmic bytes per launch of each step's kernels (DESIGN.md §6)
-        # (B is read once per row block)
+    alg = {  # algorithmic bytes per launch of each step's kernels (DESIGN.md §5)
+        # (B is read once per row block; value bytes vb for A and B, cb for C)
         "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + K * (6 * Bt.num_tiles + 8 * (Bt.tile_m + 1)) + 12 * ntC,
         "step2": 32 * (Ashard.num_tiles + K * Bt.num_tiles) + 60 * ntC,
-        "step3": 9 * (Ashard.nnz + K * Bt.nnz + nnzC) + 48 * (Ashard.num_tiles + K * Bt.num_tiles) + 56 * ntC,
+        "step3": (1 + vb) * (Ashard.nnz + K * Bt.nnz) + (1 + cb) * nnzC + 48 * (Ashard.num_tiles + K * Bt.num_tiles)
+                 + 56 * ntC,
     }
     dom = max(steps_ms, key=steps_ms.get)
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
@@ -305,8 +318,8 @@ def main():
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(dom)
-    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz) + K * tile_bytes(Bt.tile_m, Bt.num_tiles, Bt.nnz) + \
-        tile_bytes(Ashard.tile_m, ntC, nnzC)
+    bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz, vb) + \
+        K * tile_bytes(Bt.tile_m, Bt.num_tiles, Bt.nnz, vb) + tile_bytes(Ashard.tile_m, ntC, nnzC, cb)
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",
             "frac": achieved / bw, "traffic": traffic, "algorithmic_bytes": alg[dom], "peak_source": bw_src,
             "kernel_ms": steps_ms[dom]}
@@ -327,7 +340,7 @@ def main():
             dts = {k: _host_dtype(v) for k, v in Cx.arrays().items()}
             del Cx
         bufs = {k: torch.empty(n, dtype=dts[k], pin_memory=True) for k, n in sizes.items()}
-        bi = h_rp.numel() * 8 + h_ci.numel() * 4 + h_v.numel() * 8
+        bi = h_rp.numel() * 8 + h_ci.numel() * 4 + h_v.numel() * vb
         torch.cuda.synchronize()
         e2e_ms = []
         for _ in range(args.e2e_steps):
@@ -359,13 +372,14 @@ def main():
         return 0
     cpu = None
     if not args.no_cpu_baseline and not args.profile and world == 1:
-        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr)
+        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr, prec="f64" if args.dtype == "f64" else "f32")
         cpu.pop("seconds", None)
         cpu.pop("products", None)
     clocks = clk.summary() if not args.profile else None
     line = {
         "metric": _metric(args), "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": {"f64": "f64", "f32": "f32", "f16": "f16 in, f32 accumulate/out"}[args.dtype],
         "data": "synthetic",
         "config": {"workload": f"{args.config} {gen.CONFIGS[args.config][0]}" + (", C = A*A^T" if args.aat else ""),
                    "n": A.m, "nnz_a": A.nnz,
@@ -392,7 +406,8 @@ def main():
 
 
 def _metric(args):
-    return METRIC.replace("C=A^2", "C=A*A^T") if args.aat else METRIC
+    m = METRIC.replace("C=A^2", "C=A*A^T") if args.aat else METRIC
+    return m.replace("fp64", {"f64": "fp64", "f32": "fp32", "f16": "fp16-in/fp32-out"}[args.dtype])
 
 
 def _csr_transpose(A):
