@@ -48,6 +48,7 @@ struct S1Params {
     const int32_t *rowJhi;
     const uint8_t *rowClass;
     int64_t tnB;       // tile columns of B (the merge packs a tile column into 27 bits)
+    int sort_only;     // TSG_STEP1_SORT_ONLY: wide rows use the global radix sort, not the bitmap rank
     uint64_t *pairs;   // [Utot]  (posA << 32) | posB, at costOff[a0] + i
     int32_t *tJ;       // [Utot]  C tile column of rank r, at costOff[a0] + r
     uint32_t *tStart;  // [Utot]  first pair (row-relative)

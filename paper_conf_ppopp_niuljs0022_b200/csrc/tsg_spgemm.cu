@@ -137,6 +137,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.rowJhi = rowJhi;
     P1.rowClass = rowClass;
     P1.tnB = B->tn;
+    P1.sort_only = (flags & TSG_STEP1_SORT_ONLY) ? 1 : 0;
     P1.pairs = tmp.get<uint64_t>(Utot);
     P1.tJ = tmp.get<int32_t>(Utot);
     P1.tStart = tmp.get<uint32_t>(Utot);

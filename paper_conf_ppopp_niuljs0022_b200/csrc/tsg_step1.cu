@@ -580,6 +580,160 @@ __global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) {
                                       32);
 }
 
+// ------------------------------------------------------------------------------------------
+// a1 (rank): tile rows too wide for the warp merge and the shared-memory sort (R-MAT hubs, up to
+// ~10^6 candidates).  One CTA per row, no sort: the row's tile columns J that have a product are
+// marked in a shared-memory bitmap over the row's J window; a C tile's rank in the row is the
+// number of marked columns before it (per-word popcount prefix).  Pairs are counted per rank,
+// offsets scanned, and scattered with per-tile cursors; each C tile's (short) pair list is then
+// insertion-sorted by A tile position, i.e. ascending K (reading A8).  Three passes over the
+// candidates (expand once into global scratch, count, scatter) instead of a multi-pass radix sort.
+// ------------------------------------------------------------------------------------------
+constexpr int RANK_T = 512;
+constexpr int RANK_NW = RANK_T / 32;
+
+__device__ __forceinline__ int64_t block_excl_scan64(int64_t v, int64_t *total, int64_t *sm /* RANK_NW+1 */) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int64_t incl = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const int64_t o = __shfl_up_sync(FULL, incl, d);
+        if (lane >= d) incl += o;
+    }
+    if (lane == 31) sm[w] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int64_t acc = 0;
+        for (int k = 0; k < RANK_NW; k++) {
+            const int64_t x = sm[k];
+            sm[k] = acc;
+            acc += x;
+        }
+        sm[RANK_NW] = acc;
+    }
+    __syncthreads();
+    const int64_t res = sm[w] + incl - v;
+    *total = sm[RANK_NW];
+    __syncthreads();
+    return res;
+}
+
+__global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
+    extern __shared__ uint32_t bm[];  // [wwords] bitmap, then [wwords] exclusive popcount prefix
+    uint32_t *pre = bm + wwords;
+    __shared__ int64_t sm[RANK_NW + 1];
+    const int64_t I = P.bigList[blockIdx.x];
+    const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
+    const int nA = (int)(a1 - a0);
+    const int64_t base = P.costOff[a0];
+    const int64_t U = P.costOff[a1] - base;
+    const int32_t jlo = P.rowJlo[I];
+    const int64_t o = P.bigOff[I];
+    uint32_t *sJ = reinterpret_cast<uint32_t *>(P.bigKeysA + o);  // J - jlo, or ~0u without product
+    uint32_t *sPos = P.bigPosB + o;
+    uint32_t *sK = P.bigKpos + o;
+    for (int w = threadIdx.x; w < wwords; w += RANK_T) bm[w] = 0;
+    __syncthreads();
+    // pass 1: expand (load-balanced over the row's candidates), mark the bitmap
+    for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
+        const int64_t target = base + u;
+        int lo = 0, hi = nA - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (P.costOff[a0 + mid] <= target) lo = mid;
+            else hi = mid - 1;
+        }
+        const int64_t t = a0 + lo;
+        const int64_t s = target - P.costOff[t];
+        const int64_t st = P.startA[t];
+        uint32_t posB;
+        bool valid;
+        if (st < 0) {
+            posB = P.list[-st - 1 + s];
+            valid = true;
+        } else {
+            posB = (uint32_t)(st + s);
+            valid = (P.rowOccB[posB] & P.colOccA[t]) != 0;
+        }
+        const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : ~0u;
+        sJ[u] = jr;
+        sPos[u] = posB;
+        sK[u] = (uint32_t)lo;
+        if (valid) atomicOr(&bm[jr >> 5], 1u << (jr & 31));
+    }
+    __syncthreads();
+    // ranks: exclusive popcount prefix over the bitmap words (blocked ownership)
+    const int per = (wwords + RANK_T - 1) / RANK_T;
+    const int w0 = min(wwords, (int)threadIdx.x * per), w1 = min(wwords, w0 + per);
+    int64_t cntw = 0;
+    for (int w = w0; w < w1; w++) cntw += __popc(bm[w]);
+    int64_t nC;
+    int64_t run = block_excl_scan64(cntw, &nC, sm);
+    for (int w = w0; w < w1; w++) {
+        pre[w] = (uint32_t)run;
+        run += __popc(bm[w]);
+    }
+    for (int64_t r = threadIdx.x; r < nC; r += RANK_T) {
+        P.tCnt[base + r] = 0;
+        P.tWork[base + r] = 0;
+    }
+    __syncthreads();
+    // pass 2: pairs per C tile (and its tile column)
+    for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
+        const uint32_t jr = sJ[u];
+        if (jr == ~0u) continue;
+        const uint32_t rank = pre[jr >> 5] + __popc(bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
+        atomicAdd(&P.tCnt[base + rank], 1u);
+        P.tJ[base + rank] = jlo + (int32_t)jr;
+    }
+    __syncthreads();
+    // pair offsets of the C tiles (row-relative), blocked scan over the nC counts
+    const int64_t perC = (nC + RANK_T - 1) / RANK_T;
+    const int64_t c0 = min(nC, (int64_t)threadIdx.x * perC), c1 = min(nC, c0 + perC);
+    int64_t cs = 0;
+    for (int64_t r = c0; r < c1; r++) cs += P.tCnt[base + r];
+    int64_t npairs;
+    int64_t runc = block_excl_scan64(cs, &npairs, sm);
+    for (int64_t r = c0; r < c1; r++) {
+        P.tStart[base + r] = (uint32_t)runc;
+        runc += P.tCnt[base + r];
+    }
+    __syncthreads();
+    // pass 3: scatter the pairs with per-tile cursors (tWork is the cursor until pass 4)
+    for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
+        const uint32_t jr = sJ[u];
+        if (jr == ~0u) continue;
+        const uint32_t rank = pre[jr >> 5] + __popc(bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
+        const uint32_t slot = P.tStart[base + rank] + atomicAdd(&P.tWork[base + rank], 1u);
+        P.pairs[base + slot] = ((uint64_t)(a0 + sK[u]) << 32) | sPos[u];
+    }
+    __syncthreads();
+    // pass 4: each C tile's pairs in ascending A tile position (= ascending K), work estimate
+    for (int64_t r = threadIdx.x; r < nC; r += RANK_T) {
+        uint64_t *pp = P.pairs + base + P.tStart[base + r];
+        const uint32_t n = P.tCnt[base + r];
+        for (uint32_t i = 1; i < n; i++) {
+            const uint64_t x = pp[i];
+            uint32_t k = i;
+            while (k > 0 && pp[k - 1] > x) {
+                pp[k] = pp[k - 1];
+                k--;
+            }
+            pp[k] = x;
+        }
+        uint32_t wk = 0;
+        for (uint32_t i = 0; i < n; i++) {
+            const uint64_t x = pp[i];
+            wk += __popc((uint32_t)P.colOccA[(int64_t)(x >> 32)] & (uint32_t)P.rowOccB[(uint32_t)x]);
+        }
+        P.tWork[base + r] = wk;
+    }
+    if (threadIdx.x == 0) {
+        P.nC[I] = nC;
+        atomicAdd(&P.cnt->pairs, (u64c)npairs);
+    }
+}
+
 // transposed tile masks: maskT[c] bit r <=> nonzero (r,c)  (used by the item-driven paths)
 __global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ maskT) {
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -672,7 +826,17 @@ void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t
         TSG_CUDA(cudaFuncSetAttribute(k_row_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         TSG_LAUNCH(k_row_small, (unsigned)tm, ROW_T, smem, s, P, tm, cap);
     }
-    if (nbig > 0) TSG_LAUNCH(k_row_big, (unsigned)nbig, ROW_T, 0, s, P);
+    if (nbig > 0) {
+        // bitmap over the J window (<= tile columns of B) in shared memory, else the global sort
+        const int64_t wwords = (P.tnB + 31) / 32;
+        const size_t smem = (size_t)wwords * 8;
+        if (!P.sort_only && smem <= 200 * 1024) {
+            TSG_CUDA(cudaFuncSetAttribute(k_row_rank, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            TSG_LAUNCH(k_row_rank, (unsigned)nbig, RANK_T, smem, s, P, (int)wwords);
+        } else {
+            TSG_LAUNCH(k_row_big, (unsigned)nbig, ROW_T, 0, s, P);
+        }
+    }
 }
 
 

@@ -122,6 +122,8 @@ def pair_cases():
     c.append(("dense-64", D, D))
     c.append(("hub", gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004),
               gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)))
+    W = gen.hub(8192, hub_rows=(0, 5000), hub_cols=(), density=0.002)
+    c.append(("hub-wide", W, W))  # hub tile rows of ~10^5 candidates: the bitmap-rank step 1
     c.append(("identity", gen.identity(300, 3.0), gen.random_sparse(300, 300, 0.02, 9)))
     c.append(("perm", gen.permutation(257, 1), gen.permutation(257, 2)))
     return c
@@ -166,7 +168,8 @@ def _abs_csr(A, B):
                                   dict(sort_only=True, list_always=True), dict(sort_only=True, scan_only=True)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
-    for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12)):
+    for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12),
+              gen.hub(8192, hub_rows=(0, 5000), hub_cols=(), density=0.002)):
         T = tiles_of(tsg, A)
         base = host(tsg.spgemm(T, T))
         alt = host(tsg.spgemm(T, T, **opts))
