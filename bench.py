@@ -184,6 +184,9 @@ def main():
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
     ap.add_argument("--step3-rows", action="store_true", help="step 3 in the whole-tile-row kernel (experimental)")
+    ap.add_argument("--dense-tc", action="store_true",
+                    help="fp64 dense tiles on the tensor cores (DMMA 8x8x4; TSG_DENSE_TC): values within the "
+                         "north_star tolerance instead of bitwise equal to the ascending-k FMA order")
     ap.add_argument("--aat", action="store_true",
                     help="C = A * A^T (the paper's second workload, SURVEY f1); A^T is formed once with "
                          "tsg_tiles_transpose outside the timed region, like the CSR->tile conversion")
@@ -241,7 +244,8 @@ def main():
         """One step: C = A_shard * A block by block; returns summed stats (and C if one block)."""
         tot, last = {}, None
         for Ab in shards:
-            C = tsg.spgemm(Ab, Bt, stats=True, timing=timing, products=products, step3_rows=args.step3_rows)
+            C = tsg.spgemm(Ab, Bt, stats=True, timing=timing, products=products, step3_rows=args.step3_rows,
+                           dense_tc=args.dense_tc)
             for k, v in C.stats.items():
                 tot[k] = tot.get(k, 0) + v
             last = C if (keep and len(shards) == 1) else None
@@ -350,7 +354,7 @@ def main():
             Bh = tsg.transpose(Th) if args.aat else Th
             for b0, b1 in blocks:
                 Ah = tsg.slice_rows(Th, b0, b1) if (b0, b1) != (0, Th.tile_m) else Th
-                Cx = tsg.spgemm(Ah, Bh)
+                Cx = tsg.spgemm(Ah, Bh, dense_tc=args.dense_tc)
                 Cx.copy_to_host(bufs)
                 del Cx, Ah
             e1.record(stream)

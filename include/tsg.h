@@ -130,6 +130,8 @@ typedef struct {
 #define TSG_STATS_PRODUCTS 0x10u  /* also count intermediate products into stats->products */
 #define TSG_STEP3_ROWS 0x20u      /* step 3 in the whole-tile-row kernel where rows fit (experimental; same results) */
 #define TSG_STEP1_SORT_ONLY 0x40u /* step 1: no warp merge; every tile row expands + radix-sorts (same results) */
+#define TSG_DENSE_TC 0x80u        /* step 3: fp64 dense tiles on the tensor cores (DMMA 8x8x4); values within the
+                                     tolerance of the ascending-k FMA result instead of equal to it bit for bit */
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = TSG_DENSE_NNZ; 257 disables dense) */
 
 /*

@@ -25,6 +25,7 @@ STEP1_LIST_ALWAYS = 0x8
 STATS_PRODUCTS = 0x10
 STEP3_ROWS = 0x20
 STEP1_SORT_ONLY = 0x40
+DENSE_TC = 0x80
 DENSE_THRESHOLD_SHIFT = 16
 
 STATUS = {0: "TSG_OK", 1: "TSG_ERR_INVALID_ARG", 2: "TSG_ERR_SHAPE", 3: "TSG_ERR_UNSORTED",

@@ -111,6 +111,7 @@ struct StepParams {
     const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
+    int dense_tc;          // step 3: fp64 dense tiles on the tensor cores (DMMA), TSG_DENSE_TC
     DevCounters *cnt;
 };
 

@@ -202,6 +202,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.work = work;
     P.dense_threshold = TH;
     P.small_max = SMALL_NNZ;
+    P.dense_tc = ((flags & TSG_DENSE_TC) || getenv("TSG_DENSE_TC")) ? 1 : 0;  // env: tuning only
     if (const char *e = getenv("TSG_SMALL_NNZ")) P.small_max = std::max(0, std::min(16, atoi(e)));  // tuning only
     P.cnt = cnt;
     launch_step2(P, s);

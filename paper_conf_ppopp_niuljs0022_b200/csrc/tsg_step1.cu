@@ -766,6 +766,7 @@ __global__ void __launch_bounds__(256) k_compact(CompactParams P) {
     if (I >= P.tm) return;
     const int64_t base = P.costOff[P.tpA[I]];
     const int64_t t0 = P.tilePtrC[I], n = P.tilePtrC[I + 1] - t0;
+#pragma unroll 4
     for (int64_t r = lane; r < n; r += 32) {
         const int64_t slot = base + r, t = t0 + r;
         P.tile_col[t] = P.tJ[slot];

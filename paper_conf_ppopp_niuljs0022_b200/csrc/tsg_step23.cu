@@ -193,8 +193,9 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
 // ==========================================================================================
 // step 3
 // ==========================================================================================
-constexpr int WREG = 4224;  // bytes of per-warp shared scratch (small: 4 KB acc + 1.5 KB masks;
-                            // medium: 4 KB of row accumulators; dense: 4.2 KB of staged tiles)
+// per-warp shared scratch, one union: medium = 4 KB of row accumulators + two MedStage (one per
+// half warp); dense = 4.2 KB of staged tiles; dense on the tensor cores = 5 KB
+constexpr int WACC = 4096;
 
 struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
     uint16_t mA[BATCH3][TILE], mB[BATCH3][TILE];  // cp.async'd masks of A_IK and B_KJ
@@ -202,6 +203,10 @@ struct MedStage {  // per half warp: staged metadata and tile masks / row offset
     int64_t zA[BATCH3], zB[BATCH3];
     uint16_t oB[BATCH3];
 };
+
+constexpr int WREG = WACC + 2 * (int)sizeof(MedStage);
+static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
+static_assert(WREG >= 5120, "the tensor-core dense path stages 5 KB");
 
 __device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
     const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
@@ -560,10 +565,108 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
     __syncwarp();
 }
 
+// dense tile (nnz >= t_nnz), fp64 on the tensor cores (opt-in TSG_DENSE_TC): the warp holds the
+// 16x16 C tile as 2x2 DMMA m8n8k4 accumulator fragments; per pair both tiles are staged densely
+// (zero-filled, A row-major and B transposed, pitch 20 doubles: conflict-free fragment loads) and
+// 4 k-steps x 4 blocks of DMMA.8x8x4 multiply them (16 instructions for the 4096 dense FMAs).
+// The k-chunks of four are summed inside the tensor core, so values agree with the ascending-k
+// FMA order to rounding (the north_star tolerance), not bit for bit; run-to-run deterministic.
+// A pair holding a non-finite value is multiplied entry by entry instead (Inf*0 never appears).
+__device__ __forceinline__ void dmma884(double &d0, double &d1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(d0), "+d"(d1)
+                 : "d"(a), "d"(b));
+}
+
+template <typename TI>
+__device__ __forceinline__ void s3_dense_tc(const StepParams &P, int64_t t, unsigned char *wr, int lane) {
+    constexpr int PT = 20;
+    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
+    double *As = reinterpret_cast<double *>(wr);  // [16][PT]: A(r, c) at r*PT + c
+    double *Bt = As + TILE * PT;                  // [16][PT]: B(c, j) at j*PT + c
+    const int g = lane >> 2, tq = lane & 3;
+    double acc[2][2][2];
+#pragma unroll
+    for (int i = 0; i < 8; i++) (&acc[0][0][0])[i] = 0.0;
+    const uint64_t *pp = P.pairs + P.pairBeg[t];
+    const uint32_t np = P.pairCnt[t];
+    for (uint32_t p = 0; p < np; p++) {
+        const uint64_t pr = pp[p];
+        const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+#pragma unroll
+        for (int e = lane; e < 2 * TILE * PT * 8 / 16; e += 32) reinterpret_cast<uint4 *>(As)[e] = make_uint4(0u, 0u, 0u, 0u);
+        __syncwarp();
+        bool nf = false;
+        for (int64_t e = P.tnzA[pA] + lane; e < P.tnzA[pA + 1]; e += 32) {
+            const uint32_t ix = P.ixA[e];
+            const double v = vcvt<double>(vA[e]);
+            nf |= !isfinite(v);
+            As[(ix >> 4) * PT + (ix & 15)] = v;
+        }
+        for (int64_t e = P.tnzB[pB] + lane; e < P.tnzB[pB + 1]; e += 32) {
+            const uint32_t ix = P.ixB[e];
+            const double v = vcvt<double>(vB[e]);
+            nf |= !isfinite(v);
+            Bt[(ix & 15) * PT + (ix >> 4)] = v;
+        }
+        const bool anynf = __any_sync(FULL, nf);
+        __syncwarp();
+        if (!anynf) {
+#pragma unroll
+            for (int ks = 0; ks < 4; ks++) {
+                const double a0 = As[g * PT + 4 * ks + tq], a1 = As[(8 + g) * PT + 4 * ks + tq];
+                const double b0 = Bt[g * PT + 4 * ks + tq], b1 = Bt[(8 + g) * PT + 4 * ks + tq];
+                dmma884(acc[0][0][0], acc[0][0][1], a0, b0);
+                dmma884(acc[0][1][0], acc[0][1][1], a0, b1);
+                dmma884(acc[1][0][0], acc[1][0][1], a1, b0);
+                dmma884(acc[1][1][0], acc[1][1][1], a1, b1);
+            }
+        } else {
+            // entry by entry over the structural intersection (the lane's eight C entries)
+#pragma unroll
+            for (int mi = 0; mi < 2; mi++) {
+                const int r = 8 * mi + g;
+                const uint32_t mAr = P.mA[pA * TILE + r];
+#pragma unroll
+                for (int ni = 0; ni < 2; ni++)
+#pragma unroll
+                    for (int h = 0; h < 2; h++) {
+                        const int j = 8 * ni + 2 * tq + h;
+                        uint32_t x = mAr & P.mTB[pB * TILE + j];
+                        while (x) {
+                            const int c = __ffs(x) - 1;
+                            x &= x - 1;
+                            acc[mi][ni][h] = fma(As[r * PT + c], Bt[j * PT + c], acc[mi][ni][h]);
+                        }
+                    }
+            }
+        }
+        __syncwarp();
+    }
+    double *vC = static_cast<double *>(P.vC);
+#pragma unroll
+    for (int mi = 0; mi < 2; mi++) {
+        const int r = 8 * mi + g;
+        const uint32_t mC = P.mC[t * TILE + r];
+        const int64_t ob = P.tnzC[t] + P.rpC[t * TILE + r];
+#pragma unroll
+        for (int ni = 0; ni < 2; ni++)
+#pragma unroll
+            for (int h = 0; h < 2; h++) {
+                const int j = 8 * ni + 2 * tq + h;
+                if ((mC >> j) & 1u) {
+                    const int q = __popc(mC & ((1u << j) - 1u));
+                    P.ixC[ob + q] = (uint8_t)((r << 4) | j);
+                    vC[ob + q] = acc[mi][ni][h];
+                }
+            }
+    }
+    __syncwarp();
+}
+
 template <typename TI, typename TO>
 __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
-    __shared__ MedStage med[T3 / 16];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
     unsigned char *wr = wreg[w];
     const int64_t ngroups = (P.ntC + 31) / 32;
@@ -592,7 +695,7 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
             for (;;) {
                 const bool more = mm != 0;  // warp-uniform
                 if (more) nxt.load(P, pop2(), g, r);
-                s3_medium<TI, TO>(P, cur, acc, med[threadIdx.x >> 4], r);
+                s3_medium<TI, TO>(P, cur, acc, *reinterpret_cast<MedStage *>(wr + WACC + half * sizeof(MedStage)), r);
                 if (!more) break;
                 cur = nxt;
             }
@@ -602,6 +705,12 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         while (dd) {
             const int f = __ffs(dd) - 1;
             dd &= dd - 1;
+            if constexpr (sizeof(TO) == 8) {
+                if (P.dense_tc) {
+                    s3_dense_tc<TI>(P, g * 32 + f, wr, lane);
+                    continue;
+                }
+            }
             s3_dense<TI, TO>(P, g * 32 + f, wr, lane);
         }
         const unsigned vm = __ballot_sync(FULL, v);

@@ -446,3 +446,36 @@ def test_mixed_precision_inputs_rejected(tsg):
     with pytest.raises(tsg.TsgError) as e:
         tsg.spgemm(T64, T32)
     assert e.value.name == "TSG_ERR_INVALID_ARG"
+
+
+@pytest.mark.parametrize("name,A,B", [(n, a, b) for n, a, b in PAIRS if n in
+                                      ("C1", "strip-fem-8x30", "dense-64", "rmat-12", "rect", "hub")],
+                         ids=["C1", "strip-fem-8x30", "dense-64", "rmat-12", "rect", "hub"])
+def test_dense_tensor_core_variant(tsg, name, A, B):
+    """TSG_DENSE_TC: fp64 dense tiles on DMMA 8x8x4.  Structure bit-exact, values within the
+    north_star tolerance of the oracle (the tensor core sums k in chunks of four), deterministic."""
+    TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
+    ref = oracle.expected_tiles(A, B)
+    absref = oracle.csr_to_tiles(_abs_csr(A, B)).val
+    for th in (None, 1):
+        C = tsg.spgemm(TA, TB, dense_tc=True, dense_threshold=th)
+        got = host(C)
+        assert_tiles_equal(got, ref, values=None)
+        assert_values_close(got["val"], ref.val, absref)
+        again = host(tsg.spgemm(TA, TB, dense_tc=True, dense_threshold=th))
+        assert np.array_equal(got["val"].view(np.int64), again["val"].view(np.int64))
+
+
+def test_dense_tensor_core_nonfinite(tsg):
+    """A pair holding Inf/NaN is multiplied entry by entry: Inf*0 never appears."""
+    A = gen.dense_block(16, 16)
+    A.val[5] = np.inf
+    A.val[40] = np.nan
+    B = gen.random_sparse(16, 16, 0.5, 3)
+    for a, b in ((A, B), (B, A), (A, A)):
+        C = tsg.spgemm(tiles_of(tsg, a), tiles_of(tsg, b), dense_threshold=1, dense_tc=True)
+        ref = oracle.expected_tiles(a, b, fma=True)
+        got = host(C)
+        assert_tiles_equal(got, ref, values=None)
+        absref = oracle.csr_to_tiles(_abs_csr(a, b)).val
+        assert_values_close(got["val"], ref.val, absref)
