@@ -205,6 +205,7 @@ struct MedStage {  // per half warp: staged metadata and tile masks / row offset
 };
 
 constexpr int WREG = WACC + 2 * (int)sizeof(MedStage);
+static_assert(BATCH3 == 16 && BATCH == 16, "staging lane r of a half warp stages pair r of the batch");
 static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
 static_assert(WREG >= 5120, "the tensor-core dense path stages 5 KB");
 

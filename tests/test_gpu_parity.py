@@ -347,6 +347,45 @@ def test_full_size_sampled_rows(tsg, cfg):
         assert bitwise_equal_values(cv[b:e].cpu().numpy(), sub.val[s0:s1]), i
 
 
+@pytest.mark.slow
+def test_full_size_c5_row_block(tsg):
+    """C5 (R-MAT scale 22) in bench.py's launch configuration on one GPU: C is computed in four
+    tile-row blocks cut at equal product shares (its C is ~144 GB in tile form).  The first block
+    is checked: products against the oracle's count, size-independent properties, and sampled rows
+    of the block one by one against the oracle."""
+    import torch
+
+    from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
+
+    A = gen.config("C5")
+    T = tiles_of(tsg, A)
+    cuts = tdist.partition_tile_rows(A, A, 4)
+    b0, b1 = int(cuts[0]), int(cuts[1])
+    Ab = tsg.slice_rows(T, b0, b1)
+    C = tsg.spgemm(Ab, T, stats=True, products=True)
+    r0, r1 = 16 * b0, min(A.m, 16 * b1)
+    assert C.stats["products"] == oracle.products(gen.row_block(A, r0, r1), A)
+    pop = torch.zeros((), dtype=torch.int64, device=C.mask.device)
+    CH = 1 << 24
+    for t0 in range(0, C.num_tiles, CH):
+        m = C.mask[16 * t0:16 * min(C.num_tiles, t0 + CH)].view(torch.int16).to(torch.int32) & 0xFFFF
+        for b in range(16):
+            pop += ((m >> b) & 1).sum()
+        del m
+    assert int(pop) == C.nnz
+    assert bool((C.tile_nnz[1:] > C.tile_nnz[:-1]).all())
+    rng = np.random.default_rng(5)
+    rows = np.unique(np.concatenate([[r0, r1 - 1], rng.integers(r0, r1, 200)]))
+    sub = oracle.spgemm(A, A, fma=True, rows=rows)
+    crp, cci, cv = tsg.tiles_to_csr(C)
+    crp_h = crp.cpu().numpy()
+    for t, i in enumerate(rows):
+        b, e = int(crp_h[i - r0]), int(crp_h[i - r0 + 1])
+        s0, s1 = int(sub.rowptr[t]), int(sub.rowptr[t + 1])
+        assert np.array_equal(cci[b:e].cpu().numpy(), sub.col[s0:s1]), i
+        assert bitwise_equal_values(cv[b:e].cpu().numpy(), sub.val[s0:s1]), i
+
+
 # ------------------------------------------------------------------------------------------
 # SURVEY §8(f) f1: tile transpose and C = A * A^T (the paper's second workload, P:335-340)
 # ------------------------------------------------------------------------------------------
