@@ -54,6 +54,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
                 TSG_ERR_INVALID_ARG, "mask and row_ptr arrays must be 16-byte aligned, val aligned to its type");
     int TH = (int)((flags >> TSG_DENSE_THRESHOLD_SHIFT) & 0x1ffu);
     if (TH == 0) TH = TSG_DENSE_NNZ;
+    if (const char *e = getenv("TSG_DENSE_THRESHOLD")) TH = std::max(1, std::min(257, atoi(e)));  // tuning only
     Timer tm_;
     tm_.init((flags & TSG_STATS_TIMING) && st, s);
     tm_.mark(0);
@@ -71,8 +72,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
     uint16_t *mTA = tmp.get<uint16_t>(TILE * ntA);
     launch_transpose(A->mask, ntA, mTA, s);
-    uint16_t *mTB = mTA;  // A^2 (and any call with B's masks == A's): one transpose serves both
-    if (B->mask != A->mask) {
+    uint16_t *mTB = mTA;  // A^2 (B's tiles are A's tiles): one transpose serves both.  A row slice
+                          // of B shares B's mask pointer but not its tile count: transpose B then.
+    if (B->mask != A->mask || B->nt != A->nt) {
         mTB = tmp.get<uint16_t>(TILE * B->nt);
         launch_transpose(B->mask, B->nt, mTB, s);
     }

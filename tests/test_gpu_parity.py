@@ -274,13 +274,14 @@ def test_slice_rows_and_wrap(tsg):
     A = gen.rmat(11)
     T = tiles_of(tsg, A)
     full = oracle.spgemm(A, A, fma=True)
-    b, e = 17, 60
-    V = tsg.slice_rows(T, b, e)
-    CV = tsg.spgemm(V, T)
-    rows = np.arange(16 * b, 16 * e)
-    sub = oracle.spgemm(A, A, fma=True, rows=rows)
-    ref = oracle.csr_to_tiles(gen.CSR(len(rows), A.n, sub.rowptr, sub.col, sub.val))
-    assert_tiles_equal(host(CV), ref)
+    # (0, 40): a prefix slice shares B's array pointers but not its tile count (rank 0 / block 0)
+    for b, e in ((17, 60), (0, 40), (0, T.tile_m)):
+        V = tsg.slice_rows(T, b, e)
+        CV = tsg.spgemm(V, T)
+        rows = np.arange(16 * b, 16 * e)
+        sub = oracle.spgemm(A, A, fma=True, rows=rows)
+        ref = oracle.csr_to_tiles(gen.CSR(len(rows), A.n, sub.rowptr, sub.col, sub.val))
+        assert_tiles_equal(host(CV), ref)
     W = tsg.wrap(A.m, A.n, T.arrays(), keepalive=T)
     CW = tsg.spgemm(W, W)
     assert_tiles_equal(host(CW), oracle.csr_to_tiles(gen.CSR(full.m, full.n, full.rowptr, full.col, full.val)))
