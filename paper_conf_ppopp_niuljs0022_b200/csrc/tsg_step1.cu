@@ -414,13 +414,10 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
     constexpr uint32_t JM = (1u << 27) - 1u;  // tile column bits (n < 2^31); bits 27..31: work
     __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
     __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
-    __shared__ int64_t sSt[MERGE_W][32];
-    __shared__ uint32_t sOff[MERGE_W][33], sCo[MERGE_W][32], sCnt[MERGE_W][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
     if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
     const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
-    const int nA = (int)(a1 - a0);
     const int64_t base = P.costOff[a0];
     const int64_t U = P.costOff[a1] - base;
     const int64_t t = a0 + lane;
@@ -438,48 +435,23 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
     const unsigned lt = (1u << lane) - 1u;
     MergeOut out;
     if (U <= MERGE_CAP && P.tnB < (int64_t)JM) {
-        // stage: the candidates that have products (reading B3), compacted per lane segment in
-        // order: tile column + work in the top bits, and the candidate's index k in its segment
-        // (16 bits; the B tile position is st + k, or list[st + k] in list mode).  The rank inside
-        // a segment comes from a ballot over the lanes of the same segment plus its count so far.
-        sOff[w][lane] = t < a1 ? (uint32_t)off : (uint32_t)U;
-        sSt[w][lane] = isl ? -st - 1 : st;
-        sCo[w][lane] = co;
-        sCnt[w][lane] = 0;
-        __syncwarp();
-        for (int u0 = 0; u0 < (int)U; u0 += 32) {
-            const int u = u0 + lane;
-            const bool in = u < (int)U;
-            int lo = 0, k = 0;
-            uint32_t val = 0;
-            bool ok = false;
-            if (in) {
-                int hi = nA - 1;
-                while (lo < hi) {
-                    const int mid = (lo + hi + 1) >> 1;
-                    if ((int)sOff[w][mid] <= u) lo = mid;
-                    else hi = mid - 1;
-                }
-                const int64_t sl = sSt[w][lo];
-                k = u - (int)sOff[w][lo];
-                const bool il = sl < 0;
-                const uint32_t pos = il ? P.list[-sl - 1 + k] : (uint32_t)(sl + k);
-                const uint32_t wk = il ? 1u : (uint32_t)__popc(sCo[w][lo] & (uint32_t)P.rowOccB[pos]);
-                ok = wk != 0;
-                val = (uint32_t)P.tcB[pos] | (wk << 27);
+        // stage: each lane walks its own candidate list (a B tile row, or a B row list: no search
+        // for the owner) and keeps, in order, those with a product (reading B3): tile column +
+        // work in the top bits, and the candidate's index k (16 bits; the B tile position is
+        // st + k, or list[st + k] in list mode).  Four candidates per lane in flight.
+        int64_t cntv = 0;
+#pragma unroll 4
+        for (int64_t k = 0; k < len; k++) {
+            const uint32_t pos = isl ? P.list[st + k] : (uint32_t)(st + k);
+            const uint32_t wk = isl ? 1u : (uint32_t)__popc(co & (uint32_t)P.rowOccB[pos]);
+            if (wk) {
+                sJ[w][off + cntv] = (uint32_t)P.tcB[pos] | (wk << 27);
+                sK[w][off + cntv] = (uint16_t)k;
+                cntv++;
             }
-            const unsigned peers = __match_any_sync(FULL, in ? lo : -1);
-            const unsigned vb = __ballot_sync(FULL, ok) & peers;
-            if (ok) {
-                const int d = (int)sOff[w][lo] + (int)sCnt[w][lo] + __popc(vb & lt);
-                sJ[w][d] = val;
-                sK[w][d] = (uint16_t)k;
-            }
-            __syncwarp();
-            if (in && lane == 31 - __clz(peers)) sCnt[w][lo] += (uint32_t)__popc(vb);
-            __syncwarp();
         }
-        const int64_t vlen = t < a1 ? (int64_t)sCnt[w][lane] : 0;
+        __syncwarp();
+        const int64_t vlen = cntv;
         const uint32_t *mj = &sJ[w][off];
         int64_t s = 0;
         uint32_t hv = vlen > 0 ? mj[0] : INF;
