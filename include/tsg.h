@@ -132,6 +132,8 @@ typedef struct {
 #define TSG_STEP1_SORT_ONLY 0x40u /* step 1: no warp merge; every tile row expands + radix-sorts (same results) */
 #define TSG_DENSE_TC 0x80u        /* step 3: fp64 dense tiles on the tensor cores (DMMA 8x8x4); values within the
                                      tolerance of the ascending-k FMA result instead of equal to it bit for bit */
+#define TSG_SMALL_STAGE_ON 0x100u  /* step 3 small tiles: stage B row metadata by cp.async (default: iff nnz(B) < 4 tiles(B)) */
+#define TSG_SMALL_STAGE_OFF 0x200u /* step 3 small tiles: plain dependent loads (same results either way) */
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = TSG_DENSE_NNZ; 257 disables dense) */
 
 /*

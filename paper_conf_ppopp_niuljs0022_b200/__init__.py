@@ -198,7 +198,8 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
 
 def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, products: bool = False,
            scan_only: bool = False, list_always: bool = False, dense_threshold: int | None = None,
-           step3_rows: bool = False, sort_only: bool = False, dense_tc: bool = False, stream=None) -> Tiles:
+           step3_rows: bool = False, sort_only: bool = False, dense_tc: bool = False, small_stage: bool | None = None,
+           stream=None) -> Tiles:
     """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3)."""
     L = _lib.load()
     flags = 0
@@ -216,6 +217,8 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
         flags |= _lib.STEP1_SORT_ONLY
     if dense_tc:
         flags |= _lib.DENSE_TC
+    if small_stage is not None:
+        flags |= _lib.SMALL_STAGE_ON if small_stage else _lib.SMALL_STAGE_OFF
     if dense_threshold is not None:
         if not 1 <= dense_threshold <= 257:
             raise ValueError("dense_threshold must be in [1, 257]")

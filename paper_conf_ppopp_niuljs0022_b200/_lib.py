@@ -26,6 +26,8 @@ STATS_PRODUCTS = 0x10
 STEP3_ROWS = 0x20
 STEP1_SORT_ONLY = 0x40
 DENSE_TC = 0x80
+SMALL_STAGE_ON = 0x100
+SMALL_STAGE_OFF = 0x200
 DENSE_THRESHOLD_SHIFT = 16
 
 STATUS = {0: "TSG_OK", 1: "TSG_ERR_INVALID_ARG", 2: "TSG_ERR_SHAPE", 3: "TSG_ERR_UNSORTED",

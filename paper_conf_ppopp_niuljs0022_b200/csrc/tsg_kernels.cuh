@@ -25,6 +25,7 @@ struct DevCounters {
     u64c n3fallback;   // C tiles left to the per-tile kernel of step 3
     u64c next3;        // work counter of the step-3 row kernel
     u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
+    u64c n2dense;      // C tiles with nnz >= t_nnz (step 2 counts them; step 3 launches the dense kernel iff > 0)
 };
 
 constexpr int ROW_T = 256;        // threads of a step-1 row CTA
@@ -112,6 +113,7 @@ struct StepParams {
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     int dense_tc;          // step 3: fp64 dense tiles on the tensor cores (DMMA), TSG_DENSE_TC
+    int small_stage;       // step 3: k_s3_small stages B row metadata with cp.async (hypersparse B)
     DevCounters *cnt;
 };
 
@@ -171,7 +173,7 @@ void launch_compact(const CompactParams &P, cudaStream_t s);
 
 // launchers (tsg_step23.cu)
 void launch_step2(const StepParams &P, cudaStream_t s);
-void launch_step3(const StepParams &P, cudaStream_t s);
+void launch_step3(const StepParams &P, bool any_dense, cudaStream_t s);
 // launchers (tsg_step3row.cu)
 void launch_step3_class(const RowParams &R, cudaStream_t s);
 void launch_step3_rows(const RowParams &R, cudaStream_t s);

@@ -205,6 +205,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.dense_threshold = TH;
     P.small_max = SMALL_NNZ;
     P.dense_tc = ((flags & TSG_DENSE_TC) || getenv("TSG_DENSE_TC")) ? 1 : 0;  // env: tuning only
+    // small-tile B staging pays where B's tile metadata misses in cache: hypersparse tiles
+    // (fewer than 4 nonzeros per B tile on average, e.g. R-MAT); flags force either way
+    P.small_stage = (flags & TSG_SMALL_STAGE_ON) ? 1 : (flags & TSG_SMALL_STAGE_OFF) ? 0 : (B->nnz < 4 * B->nt);
     if (const char *e = getenv("TSG_SMALL_NNZ")) P.small_max = std::max(0, std::min(16, atoi(e)));  // tuning only
     P.cnt = cnt;
     launch_step2(P, s);
@@ -263,7 +266,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     if (rowk && hc2.n3rows > 0) launch_step3_rows(R, s);
     if (!rowk || hc2.n3fallback > 0) {
         P.skip = rowk ? R.skip : nullptr;
-        launch_step3(P, s);
+        launch_step3(P, hc2.n2dense > 0, s);
     }
     tm_.mark(6);
 

@@ -44,6 +44,26 @@ constexpr int T3 = 128;    // step-3 CTA (4 warps; 5.5 KB of shared memory per w
 constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
 constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
 
+// The selected lanes of a warp (sel) in ascending order of their key (ties by lane): lane k gets
+// the lane index of the k-th selected lane (-1 past the end).  Used to pair tiles of similar work
+// onto the two half warps (a half warp that finishes early idles until its partner is done).
+__device__ __forceinline__ int order_by_key(bool sel, uint32_t key, int lane, uint8_t *slots) {
+    const uint32_t k = sel ? key : 0xffffffffu;
+    int rank = 0;
+#pragma unroll 8
+    for (int o = 0; o < 32; o++) {
+        const uint32_t w = __shfl_sync(FULL, k, o);
+        rank += (w < k) || (w == k && o < lane);
+    }
+    __syncwarp();
+    if (sel) slots[rank] = (uint8_t)lane;
+    __syncwarp();
+    const int nsel = __popc(__ballot_sync(FULL, sel));
+    const int mine = lane < nsel ? (int)slots[lane] : -1;
+    __syncwarp();
+    return mine;
+}
+
 // ==========================================================================================
 // step 2
 // ==========================================================================================
@@ -57,7 +77,7 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
     __shared__ uint32_t wsm[8 * T2L];
     uint32_t *w = wsm + threadIdx.x;
     const int64_t stride = (int64_t)gridDim.x * T2L;
-    u64c nl = 0;
+    u64c nl = 0, nd = 0;
     for (int64_t t = (int64_t)blockIdx.x * T2L + threadIdx.x; t < P.ntC; t += stride) {
         if (P.work[t] > (uint32_t)LIGHT_WORK) continue;
         nl++;
@@ -107,9 +127,12 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
         dm[1] = make_uint4(m[4], m[5], m[6], m[7]);
         *reinterpret_cast<uint4 *>(P.rpC + t * TILE) = make_uint4(rp[0], rp[1], rp[2], rp[3]);
         P.tnzC[t] = total;
+        nd += total >= P.dense_threshold;
     }
     for (int o = 16; o > 0; o >>= 1) nl += __shfl_xor_sync(FULL, nl, o);
     if ((threadIdx.x & 31) == 0 && nl) atomicAdd(&P.cnt->n2light, nl);
+    for (int o = 16; o > 0; o >>= 1) nd += __shfl_xor_sync(FULL, nd, o);
+    if ((threadIdx.x & 31) == 0 && nd) atomicAdd(&P.cnt->n2dense, nd);
 }
 
 __device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
@@ -120,6 +143,7 @@ __device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
 __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
+    __shared__ uint8_t sOrd[T2 / 32][32];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
     const int64_t ngroups = (P.ntC + 31) / 32;
     const int64_t gstride = (int64_t)gridDim.x * (T2 / 32);
@@ -127,15 +151,14 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC;
         const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;  // k_s2_light's class
-        unsigned hm = __ballot_sync(FULL, v && !light);
-        // heavy tiles: two at a time, a half warp each, lane r owns row r; per batch of 16 pairs
-        // lane i stages pair i's A and B masks (4 x 16-byte cp.async, all in flight at once)
-        while (hm) {
-            const int f0 = __ffs(hm) - 1;
-            hm &= hm - 1;
-            const int f1 = hm ? __ffs(hm) - 1 : -1;
-            if (hm) hm &= hm - 1;
-            const int mine = half ? f1 : f0;
+        const bool heavy = v && !light;
+        const int nh = __popc(__ballot_sync(FULL, heavy));
+        // heavy tiles in ascending work, two at a time (similar work per half warp), lane r owns
+        // row r; per batch of 16 pairs lane i stages pair i's A and B masks (4 x 16-byte
+        // cp.async, all in flight at once)
+        const int ord = order_by_key(heavy, heavy ? P.work[t] : 0u, lane, sOrd[threadIdx.x >> 5]);
+        for (int k = 0; k < nh; k += 2) {
+            const int mine = __shfl_sync(FULL, ord, k + half);
             const bool hv = mine >= 0;
             const int64_t th = g * 32 + (hv ? mine : 0);
             uint32_t acc = 0, np = 0;
@@ -184,6 +207,8 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
                 P.rpC[th * TILE + r] = (uint8_t)(incl - cnt);
                 if (r == 0) P.tnzC[th] = tot;
             }
+            const unsigned dn = __ballot_sync(FULL, hv && r == 0 && tot >= P.dense_threshold);
+            if (lane == 0 && dn) atomicAdd(&P.cnt->n2dense, (u64c)__popc(dn));
         }
         const unsigned lm = __ballot_sync(FULL, light), vm = __ballot_sync(FULL, v);
         if (lane == 0 && vm != lm) atomicAdd(&P.cnt->n2heavy, (u64c)(__popc(vm) - __popc(lm)));
@@ -228,9 +253,15 @@ __device__ __forceinline__ void cp_wait_all() {
 constexpr int TS = 256;  // small-class CTA
 constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <= 16)
 
-template <typename TI, typename TO>
+// STAGE (hypersparse inputs, where B's tile metadata misses in cache): a lane-private double buffer
+// of the B tile's row offsets and row masks of the next pair ([buffer][chunk: row_ptr, mask rows
+// 0-7, mask rows 8-15][thread], 16 bytes each) is filled by cp.async one pair ahead, so a
+// product's B address needs a shared load instead of a dependent global one.  On cache-friendly
+// inputs (stencils: B's metadata hits L1) the staging is pure overhead and STAGE is off.
+template <typename TI, typename TO, bool STAGE>
 __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
     __shared__ uint8_t mapsm[TS / 32][SMAP];
+    __shared__ __align__(16) uint4 stg[STAGE ? 2 : 1][3][STAGE ? TS : 1];
     const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
     TO *vC = static_cast<TO *>(P.vC);
     const int lane = threadIdx.x & 31;
@@ -276,6 +307,7 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
                 const int j = (int)__fns((uint32_t)P.mC[t * TILE + r], 0, k + 1);
                 const uint32_t lowj = (1u << j) - 1u;
                 TO acc = 0;
+                if constexpr (!STAGE) {
                 // pair p's metadata is loaded while pair p-1 is being multiplied
                 uint64_t prn = pp[0];
                 int64_t pA = (int64_t)(prn >> 32), pB = (int64_t)(uint32_t)prn;
@@ -302,6 +334,73 @@ __global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
                         const TO b = vcvt<TO>(vB[czB + P.rpB[cB * TILE + c] + __popc((uint32_t)P.mB[cB * TILE + c] & lowj)]);
                         acc = vfma(a, b, acc);
                     }
+                }
+                } else {
+                // three-stage pipeline over the tile's pairs: pair p+2's row masks are loaded,
+                // pair p+1's B row offsets and masks are staged (cp.async, only if the pair meets
+                // this entry: mask_A[r] & colmask_B[j] != 0), pair p is multiplied
+                const uint8_t *sb0 = reinterpret_cast<const uint8_t *>(&stg[0][0][threadIdx.x]);
+                constexpr int BUFB = 3 * TS * 16, CHB = TS * 16;  // buffer / chunk strides in bytes
+                auto stage = [&](int bf, int64_t b) {
+                    cp16(&stg[bf][0][threadIdx.x], P.rpB + b * TILE);
+                    cp16(&stg[bf][1][threadIdx.x], P.mB + b * TILE);
+                    cp16(&stg[bf][2][threadIdx.x], P.mB + b * TILE + 8);
+                };
+                uint64_t prn = pp[0];
+                int64_t pB = (int64_t)(uint32_t)prn, pA = (int64_t)(prn >> 32);
+                uint32_t mAr = P.mA[pA * TILE + r];
+                uint32_t x = mAr & P.mTB[pB * TILE + j];
+                int64_t zA = P.tnzA[pA] + P.rpA[pA * TILE + r], zB = P.tnzB[pB];
+                if (x) stage(0, pB);
+                asm volatile("cp.async.commit_group;\n" ::: "memory");
+                // pair p+1: masks in flight
+                uint32_t mAn = 0, mTn = 0;
+                int64_t zAn = 0, zBn = 0, pBn = 0;
+                if (np > 1) {
+                    prn = pp[1];
+                    pA = (int64_t)(prn >> 32);
+                    pBn = (int64_t)(uint32_t)prn;
+                    mAn = P.mA[pA * TILE + r];
+                    mTn = P.mTB[pBn * TILE + j];
+                    zAn = P.tnzA[pA] + P.rpA[pA * TILE + r];
+                    zBn = P.tnzB[pBn];
+                    if (np > 2) prn = pp[2];
+                }
+                for (uint32_t p = 0; p < np; p++) {
+                    const int64_t czA = zA, czB = zB;
+                    const uint32_t cx = x, cmA = mAr;
+                    const int buf = p & 1;
+                    if (p + 1 < np) {
+                        // pair p+1 becomes the staged pair; pair p+2's masks are loaded
+                        mAr = mAn;
+                        x = mAn & mTn;
+                        zA = zAn;
+                        zB = zBn;
+                        if (x) stage(buf ^ 1, pBn);
+                        if (p + 2 < np) {
+                            pA = (int64_t)(prn >> 32);
+                            pBn = (int64_t)(uint32_t)prn;
+                            mAn = P.mA[pA * TILE + r];
+                            mTn = P.mTB[pBn * TILE + j];
+                            zAn = P.tnzA[pA] + P.rpA[pA * TILE + r];
+                            zBn = P.tnzB[pBn];
+                            if (p + 3 < np) prn = pp[p + 3];
+                        }
+                    }
+                    asm volatile("cp.async.commit_group;\ncp.async.wait_group 1;\n" ::: "memory");
+                    const uint8_t *sb = sb0 + buf * BUFB;
+                    uint32_t xx = cx;
+                    while (xx) {
+                        const int c = __ffs(xx) - 1;
+                        xx &= xx - 1;
+                        const TO a = vcvt<TO>(vA[czA + __popc(cmA & ((1u << c) - 1u))]);
+                        const uint32_t rb = sb[c];
+                        const uint32_t mb = *reinterpret_cast<const uint16_t *>(sb + CHB * (1 + (c >> 3)) + 2 * (c & 7));
+                        const TO b = vcvt<TO>(vB[czB + rb + __popc(mb & lowj)]);
+                        acc = vfma(a, b, acc);
+                    }
+                }
+                asm volatile("cp.async.wait_group 0;\n" ::: "memory");
                 }
                 P.ixC[o] = (uint8_t)((r << 4) | j);
                 vC[o] = acc;
@@ -402,42 +501,59 @@ struct MedMeta {
     }
 };
 
+// 16x16 bit-matrix transpose across the 16 lanes of a half warp: lane i holds row i (bit c =
+// M[i][c]); afterwards lane c holds column c (bit i = M[i][c]).  Four butterfly stages.
+__device__ __forceinline__ uint32_t bit_transpose16(uint32_t v, int r) {
+#pragma unroll
+    for (int s = 8; s > 0; s >>= 1) {
+        const uint32_t m = s == 8 ? 0x00ffu : s == 4 ? 0x0f0fu : s == 2 ? 0x3333u : 0x5555u;
+        const uint32_t x = __shfl_xor_sync(FULL, v, s);
+        v = (r & s) ? ((v & ~m & 0xffffu) | ((x >> s) & m)) : ((v & m) | ((x << s) & ~m & 0xffffu));
+    }
+    return v;
+}
+
 template <typename TI, typename TO>
 __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M, TO *acc, MedStage &S, int r) {
     const uint32_t np = M.np, mCr = M.mCr;
     const uint64_t *pp = M.pp;
-    {
-        uint32_t m = mCr;
-        while (m) {
-            const int j = __ffs(m) - 1;
-            m &= m - 1;
-            acc[j * 16] = (TO)0;
-        }
-    }
     const uint32_t nbat = (np + BATCH3 - 1) / BATCH3;
     const uint32_t nbw = max(nbat, __shfl_xor_sync(FULL, nbat, 16));
     for (uint32_t bt = 0; bt < nbw; bt++) {
         const uint32_t q = bt * BATCH3 + r;
+        // lane r stages pair q of the batch and finds the rows of its A tile that meet a non-empty
+        // row of its B tile (bit r' <=> mask_A[r'] & rowOcc(B) != 0); a bit transpose then gives
+        // every lane the batch pairs that touch its own row
+        uint32_t rows = 0;
         if (q < np) {
             const uint64_t pr = bt == 0 ? M.pr : pp[q];
             const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-            cp16(&S.mA[r][0], P.mA + pA * TILE);
-            cp16(&S.mA[r][8], P.mA + pA * TILE + 8);
+            const uint4 *ga = reinterpret_cast<const uint4 *>(P.mA + pA * TILE);
+            const uint4 a0 = ga[0], a1 = ga[1];
             cp16(&S.mB[r][0], P.mB + pB * TILE);
             cp16(&S.mB[r][8], P.mB + pB * TILE + 8);
             cp16(&S.rA[r][0], P.rpA + pA * TILE);
             cp16(&S.rB[r][0], P.rpB + pB * TILE);
             S.zA[r] = P.tnzA[pA];
             S.zB[r] = P.tnzB[pB];
-            S.oB[r] = P.rowOccB[pB];
+            const uint32_t ob = P.rowOccB[pB];
+            S.oB[r] = (uint16_t)ob;
+            reinterpret_cast<uint4 *>(&S.mA[r][0])[0] = a0;
+            reinterpret_cast<uint4 *>(&S.mA[r][0])[1] = a1;
+            const uint32_t ob2 = ob * 0x10001u;
+            const uint32_t w[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+#pragma unroll
+            for (int k = 0; k < 8; k++) {
+                const uint32_t h = __vcmpne2(w[k] & ob2, 0u);
+                rows |= ((h & 1u) << (2 * k)) | (((h >> 16) & 1u) << (2 * k + 1));
+            }
         }
+        const uint32_t rel = bit_transpose16(rows, r);
         cp_wait_all();
         __syncwarp();
-        const int nb = np > bt * BATCH3 ? (int)min((uint32_t)BATCH3, np - bt * BATCH3) : 0;
-        if (mCr) {
+        if (rel) {
             ItemStream<TI, TO> it;
-            it.rel = 0;
-            for (int i = 0; i < nb; i++) it.rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
+            it.rel = rel;
             TO aX, bX0, bX1, bX2, aY, bY0, bY1, bY2;
             uint32_t mX, mY;
             const TI *vX, *vY;
@@ -452,16 +568,19 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
         }
         __syncwarp();
     }
+    // compaction through mask_C[r]; every slot the tile touched is in mask_C[r] and is reset to
+    // zero for the next tile (the accumulator is cleared once per warp at kernel start)
     if (mCr) {
-        const int64_t ob = M.ob;
+        uint8_t *px = P.ixC + M.ob;
+        TO *pv = static_cast<TO *>(P.vC) + M.ob;
         uint32_t m = mCr;
-        int qq = 0;
         while (m) {
             const int j = __ffs(m) - 1;
             m &= m - 1;
-            P.ixC[ob + qq] = (uint8_t)((r << 4) | j);
-            static_cast<TO *>(P.vC)[ob + qq] = acc[j * 16];
-            qq++;
+            TO *sl = acc + j * 16;
+            *px++ = (uint8_t)((r << 4) | j);
+            *pv++ = *sl;
+            *sl = (TO)0;
         }
     }
     __syncwarp();
@@ -665,10 +784,53 @@ __device__ __forceinline__ void s3_dense_tc(const StepParams &P, int64_t t, unsi
     __syncwarp();
 }
 
+// medium tiles: warps take groups of 32 consecutive C tiles; the group's medium tiles go two at a
+// time, a half warp each.  Register- and shared-memory-lean (no dense code): 7 CTAs per SM.
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
+__global__ void __launch_bounds__(T3, 7) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
+    __shared__ uint8_t sOrd[T3 / 32][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
+    unsigned char *wr = wreg[w];
+    TO *acc = reinterpret_cast<TO *>(wr) + half * (TILE * TILE) + r;
+#pragma unroll
+    for (int j = 0; j < TILE; j++) acc[j * 16] = (TO)0;
+    const int64_t ngroups = (P.ntC + 31) / 32;
+    const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
+    for (int64_t g = (int64_t)blockIdx.x * (T3 / 32) + w; g < ngroups; g += gstride) {
+        const int64_t t = g * 32 + lane;
+        const bool v = t < P.ntC && !(P.skip && P.skip[t]);
+        const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
+        const bool med = v && nz < P.dense_threshold && nz > P.small_max;
+        const int nm = __popc(__ballot_sync(FULL, med));
+        if (lane == 0 && nm) atomicAdd(&P.cnt->n3medium, (u64c)nm);
+        if (nm) {
+            // the group's medium tiles in ascending work, two at a time (one per half warp)
+            const int ord = order_by_key(med, med ? P.work[t] : 0u, lane, sOrd[w]);
+            int k = 0;
+            auto pop2 = [&]() {
+                const int f = __shfl_sync(FULL, ord, k + half);
+                k += 2;
+                return f;
+            };
+            MedMeta cur, nxt;
+            cur.load(P, pop2(), g, r);
+            for (;;) {
+                const bool more = k < nm;  // warp-uniform
+                if (more) nxt.load(P, pop2(), g, r);
+                s3_medium<TI, TO>(P, cur, acc, *reinterpret_cast<MedStage *>(wr + WACC + half * sizeof(MedStage)), r);
+                if (!more) break;
+                cur = nxt;
+            }
+        }
+    }
+}
+
+// dense tiles (nnz >= t_nnz): the whole warp each; launched only when step 2 counted any
+template <typename TI, typename TO>
+__global__ void __launch_bounds__(T3, 4) k_s3_dense(StepParams P) {
+    __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     unsigned char *wr = wreg[w];
     const int64_t ngroups = (P.ntC + 31) / 32;
     const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
@@ -676,32 +838,8 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC && !(P.skip && P.skip[t]);
         const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
-        const bool dense = v && nz >= P.dense_threshold;
-        const bool small = v && !dense && nz <= P.small_max;  // k_s3_small's class
-        const unsigned sm = __ballot_sync(FULL, small);
-        const unsigned dm = __ballot_sync(FULL, dense);
-        unsigned mm = __ballot_sync(FULL, v) & ~sm & ~dm;
-        // medium tiles: two at a time, a half warp each
-        TO *acc = reinterpret_cast<TO *>(wr) + half * (TILE * TILE) + r;
-        auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
-            const int f0 = __ffs(mm) - 1;
-            mm &= mm - 1;
-            const int f1 = mm ? __ffs(mm) - 1 : -1;
-            if (mm) mm &= mm - 1;
-            return half ? f1 : f0;
-        };
-        if (mm) {
-            MedMeta cur, nxt;
-            cur.load(P, pop2(), g, r);
-            for (;;) {
-                const bool more = mm != 0;  // warp-uniform
-                if (more) nxt.load(P, pop2(), g, r);
-                s3_medium<TI, TO>(P, cur, acc, *reinterpret_cast<MedStage *>(wr + WACC + half * sizeof(MedStage)), r);
-                if (!more) break;
-                cur = nxt;
-            }
-        }
-        // dense tiles: the whole warp each
+        const unsigned dm = __ballot_sync(FULL, v && nz >= P.dense_threshold);
+        if (lane == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
         unsigned dd = dm;
         while (dd) {
             const int f = __ffs(dd) - 1;
@@ -713,11 +851,6 @@ __global__ void __launch_bounds__(T3, 6) k_s3(StepParams P) {
                 }
             }
             s3_dense<TI, TO>(P, g * 32 + f, wr, lane);
-        }
-        const unsigned vm = __ballot_sync(FULL, v);
-        if (lane == 0) {
-            atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
-            atomicAdd(&P.cnt->n3medium, (u64c)(__popc(vm) - __popc(sm) - __popc(dm)));
         }
     }
 }
@@ -737,17 +870,23 @@ void launch_step2(const StepParams &P, cudaStream_t s) {
 }
 
 template <typename TI, typename TO>
-static void launch_step3_t(const StepParams &P, cudaStream_t s) {
-    if (P.small_max > 0) TSG_LAUNCH((k_s3_small<TI, TO>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
+static void launch_step3_t(const StepParams &P, bool any_dense, cudaStream_t s) {
+    if (P.small_max > 0) {
+        if (P.small_stage)
+            TSG_LAUNCH((k_s3_small<TI, TO, true>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
+        else
+            TSG_LAUNCH((k_s3_small<TI, TO, false>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
+    }
     TSG_LAUNCH((k_s3<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
+    if (any_dense) TSG_LAUNCH((k_s3_dense<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
 }
 
-void launch_step3(const StepParams &P, cudaStream_t s) {
+void launch_step3(const StepParams &P, bool any_dense, cudaStream_t s) {
     if (P.ntC <= 0) return;
     switch (P.dtype_in) {
-        case TSG_F64: launch_step3_t<double, double>(P, s); break;
-        case TSG_F32: launch_step3_t<float, float>(P, s); break;
-        default: launch_step3_t<__half, float>(P, s);
+        case TSG_F64: launch_step3_t<double, double>(P, any_dense, s); break;
+        case TSG_F32: launch_step3_t<float, float>(P, any_dense, s); break;
+        default: launch_step3_t<__half, float>(P, any_dense, s);
     }
 }
 

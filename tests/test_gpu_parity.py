@@ -165,7 +165,8 @@ def _abs_csr(A, B):
 @pytest.mark.parametrize("opts", [dict(scan_only=True), dict(list_always=True), dict(dense_threshold=1),
                                   dict(dense_threshold=257), dict(dense_threshold=100), dict(step3_rows=True),
                                   dict(step3_rows=True, dense_threshold=1), dict(sort_only=True),
-                                  dict(sort_only=True, list_always=True), dict(sort_only=True, scan_only=True)])
+                                  dict(sort_only=True, list_always=True), dict(sort_only=True, scan_only=True),
+                                  dict(small_stage=True), dict(small_stage=False)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
     for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12),
