@@ -44,26 +44,6 @@ constexpr int T3 = 128;    // step-3 CTA (4 warps; 5.5 KB of shared memory per w
 constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
 constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
 
-// The selected lanes of a warp (sel) in ascending order of their key (ties by lane): lane k gets
-// the lane index of the k-th selected lane (-1 past the end).  Used to pair tiles of similar work
-// onto the two half warps (a half warp that finishes early idles until its partner is done).
-__device__ __forceinline__ int order_by_key(bool sel, uint32_t key, int lane, uint8_t *slots) {
-    const uint32_t k = sel ? key : 0xffffffffu;
-    int rank = 0;
-#pragma unroll 8
-    for (int o = 0; o < 32; o++) {
-        const uint32_t w = __shfl_sync(FULL, k, o);
-        rank += (w < k) || (w == k && o < lane);
-    }
-    __syncwarp();
-    if (sel) slots[rank] = (uint8_t)lane;
-    __syncwarp();
-    const int nsel = __popc(__ballot_sync(FULL, sel));
-    const int mine = lane < nsel ? (int)slots[lane] : -1;
-    __syncwarp();
-    return mine;
-}
-
 // ==========================================================================================
 // step 2
 // ==========================================================================================
@@ -143,7 +123,6 @@ __device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
 __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
-    __shared__ uint8_t sOrd[T2 / 32][32];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
     const int64_t ngroups = (P.ntC + 31) / 32;
     const int64_t gstride = (int64_t)gridDim.x * (T2 / 32);
@@ -151,14 +130,15 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC;
         const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;  // k_s2_light's class
-        const bool heavy = v && !light;
-        const int nh = __popc(__ballot_sync(FULL, heavy));
-        // heavy tiles in ascending work, two at a time (similar work per half warp), lane r owns
-        // row r; per batch of 16 pairs lane i stages pair i's A and B masks (4 x 16-byte
-        // cp.async, all in flight at once)
-        const int ord = order_by_key(heavy, heavy ? P.work[t] : 0u, lane, sOrd[threadIdx.x >> 5]);
-        for (int k = 0; k < nh; k += 2) {
-            const int mine = __shfl_sync(FULL, ord, k + half);
+        unsigned hm = __ballot_sync(FULL, v && !light);
+        // heavy tiles: two at a time, a half warp each, lane r owns row r; per batch of 16 pairs
+        // lane i stages pair i's A and B masks (4 x 16-byte cp.async, all in flight at once)
+        while (hm) {
+            const int f0 = __ffs(hm) - 1;
+            hm &= hm - 1;
+            const int f1 = hm ? __ffs(hm) - 1 : -1;
+            if (hm) hm &= hm - 1;
+            const int mine = half ? f1 : f0;
             const bool hv = mine >= 0;
             const int64_t th = g * 32 + (hv ? mine : 0);
             uint32_t acc = 0, np = 0;
@@ -789,7 +769,6 @@ __device__ __forceinline__ void s3_dense_tc(const StepParams &P, int64_t t, unsi
 template <typename TI, typename TO>
 __global__ void __launch_bounds__(T3, 7) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
-    __shared__ uint8_t sOrd[T3 / 32][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
     unsigned char *wr = wreg[w];
     TO *acc = reinterpret_cast<TO *>(wr) + half * (TILE * TILE) + r;
@@ -802,21 +781,20 @@ __global__ void __launch_bounds__(T3, 7) k_s3(StepParams P) {
         const bool v = t < P.ntC && !(P.skip && P.skip[t]);
         const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
         const bool med = v && nz < P.dense_threshold && nz > P.small_max;
-        const int nm = __popc(__ballot_sync(FULL, med));
-        if (lane == 0 && nm) atomicAdd(&P.cnt->n3medium, (u64c)nm);
-        if (nm) {
-            // the group's medium tiles in ascending work, two at a time (one per half warp)
-            const int ord = order_by_key(med, med ? P.work[t] : 0u, lane, sOrd[w]);
-            int k = 0;
-            auto pop2 = [&]() {
-                const int f = __shfl_sync(FULL, ord, k + half);
-                k += 2;
-                return f;
-            };
+        unsigned mm = __ballot_sync(FULL, med);
+        if (lane == 0 && mm) atomicAdd(&P.cnt->n3medium, (u64c)__popc(mm));
+        auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
+            const int f0 = __ffs(mm) - 1;
+            mm &= mm - 1;
+            const int f1 = mm ? __ffs(mm) - 1 : -1;
+            if (mm) mm &= mm - 1;
+            return half ? f1 : f0;
+        };
+        if (mm) {
             MedMeta cur, nxt;
             cur.load(P, pop2(), g, r);
             for (;;) {
-                const bool more = k < nm;  // warp-uniform
+                const bool more = mm != 0;  // warp-uniform
                 if (more) nxt.load(P, pop2(), g, r);
                 s3_medium<TI, TO>(P, cur, acc, *reinterpret_cast<MedStage *>(wr + WACC + half * sizeof(MedStage)), r);
                 if (!more) break;
