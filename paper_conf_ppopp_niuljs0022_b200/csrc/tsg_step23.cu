@@ -44,6 +44,31 @@ constexpr int T3 = 128;    // step-3 CTA (4 warps; 5.5 KB of shared memory per w
 constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
 constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
 
+// 16x16 bit-matrix transpose across the 16 lanes of a half warp: lane i holds row i (bit c =
+// M[i][c]); afterwards lane c holds column c (bit i = M[i][c]).  Four butterfly stages.
+__device__ __forceinline__ uint32_t bit_transpose16(uint32_t v, int r) {
+#pragma unroll
+    for (int s = 8; s > 0; s >>= 1) {
+        const uint32_t m = s == 8 ? 0x00ffu : s == 4 ? 0x0f0fu : s == 2 ? 0x3333u : 0x5555u;
+        const uint32_t x = __shfl_xor_sync(FULL, v, s);
+        v = (r & s) ? ((v & ~m & 0xffffu) | ((x >> s) & m)) : ((v & m) | ((x << s) & ~m & 0xffffu));
+    }
+    return v;
+}
+
+// rows r of a 16x16 tile (mask words w[0..7], two rows per word) with mask[r] & occ != 0, as bits
+__device__ __forceinline__ uint32_t rows_meeting(const uint4 &a0, const uint4 &a1, uint32_t occ) {
+    const uint32_t o2 = occ * 0x10001u;
+    const uint32_t w[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+    uint32_t rows = 0;
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+        const uint32_t h = __vcmpne2(w[k] & o2, 0u);
+        rows |= ((h & 1u) << (2 * k)) | (((h >> 16) & 1u) << (2 * k + 1));
+    }
+    return rows;
+}
+
 // ==========================================================================================
 // step 2
 // ==========================================================================================
@@ -481,18 +506,6 @@ struct MedMeta {
     }
 };
 
-// 16x16 bit-matrix transpose across the 16 lanes of a half warp: lane i holds row i (bit c =
-// M[i][c]); afterwards lane c holds column c (bit i = M[i][c]).  Four butterfly stages.
-__device__ __forceinline__ uint32_t bit_transpose16(uint32_t v, int r) {
-#pragma unroll
-    for (int s = 8; s > 0; s >>= 1) {
-        const uint32_t m = s == 8 ? 0x00ffu : s == 4 ? 0x0f0fu : s == 2 ? 0x3333u : 0x5555u;
-        const uint32_t x = __shfl_xor_sync(FULL, v, s);
-        v = (r & s) ? ((v & ~m & 0xffffu) | ((x >> s) & m)) : ((v & m) | ((x << s) & ~m & 0xffffu));
-    }
-    return v;
-}
-
 template <typename TI, typename TO>
 __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M, TO *acc, MedStage &S, int r) {
     const uint32_t np = M.np, mCr = M.mCr;
@@ -508,8 +521,13 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
         if (q < np) {
             const uint64_t pr = bt == 0 ? M.pr : pp[q];
             const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+#ifdef TSG_MED_REL_LOOP
+            cp16(&S.mA[r][0], P.mA + pA * TILE);
+            cp16(&S.mA[r][8], P.mA + pA * TILE + 8);
+#else
             const uint4 *ga = reinterpret_cast<const uint4 *>(P.mA + pA * TILE);
             const uint4 a0 = ga[0], a1 = ga[1];
+#endif
             cp16(&S.mB[r][0], P.mB + pB * TILE);
             cp16(&S.mB[r][8], P.mB + pB * TILE + 8);
             cp16(&S.rA[r][0], P.rpA + pA * TILE);
@@ -518,19 +536,25 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
             S.zB[r] = P.tnzB[pB];
             const uint32_t ob = P.rowOccB[pB];
             S.oB[r] = (uint16_t)ob;
+#ifndef TSG_MED_REL_LOOP
             reinterpret_cast<uint4 *>(&S.mA[r][0])[0] = a0;
             reinterpret_cast<uint4 *>(&S.mA[r][0])[1] = a1;
-            const uint32_t ob2 = ob * 0x10001u;
-            const uint32_t w[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-#pragma unroll
-            for (int k = 0; k < 8; k++) {
-                const uint32_t h = __vcmpne2(w[k] & ob2, 0u);
-                rows |= ((h & 1u) << (2 * k)) | (((h >> 16) & 1u) << (2 * k + 1));
-            }
+            rows = rows_meeting(a0, a1, ob);
+#endif
         }
+#ifndef TSG_MED_REL_LOOP
         const uint32_t rel = bit_transpose16(rows, r);
         cp_wait_all();
         __syncwarp();
+#else
+        cp_wait_all();
+        __syncwarp();
+        uint32_t rel = 0;
+        {
+            const int nb = np > bt * BATCH3 ? (int)min((uint32_t)BATCH3, np - bt * BATCH3) : 0;
+            for (int i = 0; i < nb; i++) rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
+        }
+#endif
         if (rel) {
             ItemStream<TI, TO> it;
             it.rel = rel;
@@ -767,7 +791,10 @@ __device__ __forceinline__ void s3_dense_tc(const StepParams &P, int64_t t, unsi
 // medium tiles: warps take groups of 32 consecutive C tiles; the group's medium tiles go two at a
 // time, a half warp each.  Register- and shared-memory-lean (no dense code): 7 CTAs per SM.
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(T3, 7) k_s3(StepParams P) {
+#ifndef TSG_MED_MINB
+#define TSG_MED_MINB 7
+#endif
+__global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
     unsigned char *wr = wreg[w];
