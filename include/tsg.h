@@ -230,6 +230,17 @@ TSG_API tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int6
                                   int32_t *tile_col, int64_t *tile_nnz, uint8_t *row_ptr,
                                   uint16_t *mask, uint8_t *idx, void *val);
 
+/*
+ * tsg_tiles_copy_to_host_async -- the same copies, stream-ordered and non-blocking: the host
+ * buffers hold the result once `stream` has passed the call (the caller synchronizes, e.g. on an
+ * event), and T must stay alive until then.  Lets a caller overlap the copy of one result with
+ * the computation of the next (row blocks on two streams).  Host buffers should be pinned
+ * (pageable memory makes the copies synchronous).
+ */
+TSG_API tsg_status tsg_tiles_copy_to_host_async(const tsg_tiles *T, void *stream, int64_t *tile_ptr,
+                                        int32_t *tile_col, int64_t *tile_nnz, uint8_t *row_ptr,
+                                        uint16_t *mask, uint8_t *idx, void *val);
+
 /* Release a handle (stream-ordered frees through its allocator).  NULL is a no-op. */
 TSG_API void tsg_tiles_destroy(tsg_tiles *T, void *stream);
 

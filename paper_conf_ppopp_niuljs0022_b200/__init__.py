@@ -111,8 +111,10 @@ class Tiles:
         csr = 8 * (self.m + 1) + (4 + vb) * self.nnz
         return {"tile_bytes": tile, "csr_bytes": csr, "ratio": tile / csr if csr else float("nan")}
 
-    def copy_to_host(self, out: dict | None = None, stream=None) -> dict:
-        """Copy the seven arrays into host buffers (numpy or pinned torch CPU tensors) via the C ABI."""
+    def copy_to_host(self, out: dict | None = None, stream=None, blocking: bool = True) -> dict:
+        """Copy the seven arrays into host buffers (numpy or pinned torch CPU tensors) via the C ABI.
+        ``blocking=False``: stream-ordered (tsg_tiles_copy_to_host_async); the buffers are valid once
+        ``stream`` has passed the copy, and this matrix must stay alive until then."""
         sizes = {"tile_ptr": (self.tile_m + 1, np.int64), "tile_col": (self.num_tiles, np.int32),
                  "tile_nnz": (self.num_tiles + 1, np.int64), "row_ptr": (16 * self.num_tiles, np.uint8),
                  "mask": (16 * self.num_tiles, np.uint16), "idx": (self.nnz, np.uint8),
@@ -123,7 +125,9 @@ class Tiles:
         for k in sizes:
             a = out[k]
             ptrs.append(C.c_void_p(a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data))
-        _lib.check(_lib.load().tsg_tiles_copy_to_host(self.ptr, C.c_void_p(_stream_ptr(stream)), *ptrs))
+        L = _lib.load()
+        fn = L.tsg_tiles_copy_to_host if blocking else L.tsg_tiles_copy_to_host_async
+        _lib.check(fn(self.ptr, C.c_void_p(_stream_ptr(stream)), *ptrs))
         return out
 
 

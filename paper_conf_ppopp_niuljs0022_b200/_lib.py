@@ -70,7 +70,7 @@ class Allocator(C.Structure):
 
 # every symbol the header declares (checked by tests/test_abi.py against include/tsg.h)
 SYMBOLS = ["tsg_csr_to_tiles", "tsg_csr_to_tiles_typed", "tsg_spgemm", "tsg_tiles_to_csr", "tsg_tiles_get_view", "tsg_tiles_wrap",
-           "tsg_tiles_slice_rows", "tsg_tiles_copy_to_host", "tsg_tiles_destroy", "tsg_free",
+           "tsg_tiles_slice_rows", "tsg_tiles_copy_to_host", "tsg_tiles_copy_to_host_async", "tsg_tiles_destroy", "tsg_free",
            "tsg_status_string", "tsg_last_error", "tsg_abi_version", "tsg_kernel_launch_count",
            "tsg_workspace_release", "tsg_tiles_transpose"]
 
@@ -104,6 +104,8 @@ def load():
     L.tsg_tiles_slice_rows.argtypes = [vp, i64, i64, vp, pp]
     L.tsg_tiles_copy_to_host.restype = C.c_int
     L.tsg_tiles_copy_to_host.argtypes = [vp, vp, vp, vp, vp, vp, vp, vp, vp]
+    L.tsg_tiles_copy_to_host_async.restype = C.c_int
+    L.tsg_tiles_copy_to_host_async.argtypes = [vp, vp, vp, vp, vp, vp, vp, vp, vp]
     L.tsg_tiles_destroy.restype = None
     L.tsg_tiles_destroy.argtypes = [vp, vp]
     L.tsg_free.restype = None

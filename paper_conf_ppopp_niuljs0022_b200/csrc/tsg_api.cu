@@ -393,8 +393,9 @@ tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t b, int64_t e, void *
     });
 }
 
-tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
-                                  int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, void *val) {
+static tsg_status copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
+                               int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, void *val,
+                               bool blocking) {
     return guarded([&] {
         TSG_REQUIRE(T, TSG_ERR_INVALID_ARG, "NULL handle");
         cudaStream_t s = (cudaStream_t)stream;
@@ -408,8 +409,19 @@ tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *til
         cp(mask, T->mask, sizeof(uint16_t) * 16 * T->nt);
         cp(idx, T->idx, T->nnz);
         cp(val, T->val, T->vsize() * T->nnz);
-        TSG_CUDA(cudaStreamSynchronize(s));
+        if (blocking) TSG_CUDA(cudaStreamSynchronize(s));
     });
+}
+
+tsg_status tsg_tiles_copy_to_host(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
+                                  int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx, void *val) {
+    return copy_to_host(T, stream, tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val, true);
+}
+
+tsg_status tsg_tiles_copy_to_host_async(const tsg_tiles *T, void *stream, int64_t *tile_ptr, int32_t *tile_col,
+                                        int64_t *tile_nnz, uint8_t *row_ptr, uint16_t *mask, uint8_t *idx,
+                                        void *val) {
+    return copy_to_host(T, stream, tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val, false);
 }
 
 void tsg_tiles_destroy(tsg_tiles *T, void *stream) { destroy_handle(T, (cudaStream_t)stream); }
