@@ -173,7 +173,7 @@ void launch_compact(const CompactParams &P, cudaStream_t s);
 
 // launchers (tsg_step23.cu)
 void launch_step2(const StepParams &P, cudaStream_t s);
-void launch_step3(const StepParams &P, bool any_dense, cudaStream_t s);
+void launch_step3(const StepParams &P, int64_t n_dense, cudaStream_t s);
 // launchers (tsg_step3row.cu)
 void launch_step3_class(const RowParams &R, cudaStream_t s);
 void launch_step3_rows(const RowParams &R, cudaStream_t s);

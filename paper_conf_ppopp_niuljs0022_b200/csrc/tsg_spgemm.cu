@@ -266,7 +266,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     if (rowk && hc2.n3rows > 0) launch_step3_rows(R, s);
     if (!rowk || hc2.n3fallback > 0) {
         P.skip = rowk ? R.skip : nullptr;
-        launch_step3(P, hc2.n2dense > 0, s);
+        launch_step3(P, (int64_t)hc2.n2dense, s);
     }
     tm_.mark(6);
 

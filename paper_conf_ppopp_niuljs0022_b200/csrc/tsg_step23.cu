@@ -263,8 +263,11 @@ constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <=
 // 0-7, mask rows 8-15][thread], 16 bytes each) is filled by cp.async one pair ahead, so a
 // product's B address needs a shared load instead of a dependent global one.  On cache-friendly
 // inputs (stencils: B's metadata hits L1) the staging is pure overhead and STAGE is off.
+#ifndef TSG_SMALL_MINB
+#define TSG_SMALL_MINB 5
+#endif
 template <typename TI, typename TO, bool STAGE>
-__global__ void __launch_bounds__(TS, 5) k_s3_small(StepParams P) {
+__global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
     __shared__ uint8_t mapsm[TS / 32][SMAP];
     __shared__ __align__(16) uint4 stg[STAGE ? 2 : 1][3][STAGE ? TS : 1];
     const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
@@ -832,23 +835,33 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
 }
 
 // dense tiles (nnz >= t_nnz): the whole warp each; launched only when step 2 counted any
+#ifndef TSG_DENSE_MINB
+#define TSG_DENSE_MINB 4
+#endif
+constexpr int DREG = 5120;  // per-warp staging of the dense paths (fp64: 16x17 + 16x16 doubles; DMMA: 2 x 16x20)
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(T3, 4) k_s3_dense(StepParams P) {
-    __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
+__global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, int split) {
+    __shared__ __align__(16) unsigned char wreg[T3 / 32][DREG];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     unsigned char *wr = wreg[w];
-    const int64_t ngroups = (P.ntC + 31) / 32;
+    // `split` warps share a group of 32 C tiles, warp `part` taking every split-th dense tile of
+    // it: dense tiles cluster (FEM strips), and a group's dense tiles done by one warp one after
+    // the other would make the kernel a chain of serial per-pair latencies
+    const int64_t nunits = (P.ntC + 31) / 32 * split;
     const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
-    for (int64_t g = (int64_t)blockIdx.x * (T3 / 32) + w; g < ngroups; g += gstride) {
+    for (int64_t u = (int64_t)blockIdx.x * (T3 / 32) + w; u < nunits; u += gstride) {
+        const int64_t g = u / split;
+        const int part = (int)(u - g * split);
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC && !(P.skip && P.skip[t]);
         const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
         const unsigned dm = __ballot_sync(FULL, v && nz >= P.dense_threshold);
-        if (lane == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
+        if (lane == 0 && part == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
         unsigned dd = dm;
-        while (dd) {
+        for (int k = 0; dd; k++) {
             const int f = __ffs(dd) - 1;
             dd &= dd - 1;
+            if (k % split != part) continue;
             if constexpr (sizeof(TO) == 8) {
                 if (P.dense_tc) {
                     s3_dense_tc<TI>(P, g * 32 + f, wr, lane);
@@ -875,7 +888,7 @@ void launch_step2(const StepParams &P, cudaStream_t s) {
 }
 
 template <typename TI, typename TO>
-static void launch_step3_t(const StepParams &P, bool any_dense, cudaStream_t s) {
+static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s) {
     if (P.small_max > 0) {
         if (P.small_stage)
             TSG_LAUNCH((k_s3_small<TI, TO, true>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
@@ -883,15 +896,21 @@ static void launch_step3_t(const StepParams &P, bool any_dense, cudaStream_t s) 
             TSG_LAUNCH((k_s3_small<TI, TO, false>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
     }
     TSG_LAUNCH((k_s3<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
-    if (any_dense) TSG_LAUNCH((k_s3_dense<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
+    if (n_dense > 0) {
+        // dense tiles per group of 32: spread a group over up to 8 warps when dense tiles are common
+        const int64_t groups = (P.ntC + 31) / 32;
+        const int split = (int)std::max<int64_t>(1, std::min<int64_t>(8, 32 * n_dense / (groups * 4)));
+        const int64_t ctas = std::min<int64_t>(ceil_div(groups * split, T3 / 32), 148LL * 32);
+        TSG_LAUNCH((k_s3_dense<TI, TO>), (unsigned)std::max<int64_t>(ctas, 1), T3, 0, s, P, split);
+    }
 }
 
-void launch_step3(const StepParams &P, bool any_dense, cudaStream_t s) {
+void launch_step3(const StepParams &P, int64_t n_dense, cudaStream_t s) {
     if (P.ntC <= 0) return;
     switch (P.dtype_in) {
-        case TSG_F64: launch_step3_t<double, double>(P, any_dense, s); break;
-        case TSG_F32: launch_step3_t<float, float>(P, any_dense, s); break;
-        default: launch_step3_t<__half, float>(P, any_dense, s);
+        case TSG_F64: launch_step3_t<double, double>(P, n_dense, s); break;
+        case TSG_F32: launch_step3_t<float, float>(P, n_dense, s); break;
+        default: launch_step3_t<__half, float>(P, n_dense, s);
     }
 }
 
