@@ -858,10 +858,10 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
         const unsigned dm = __ballot_sync(FULL, v && nz >= P.dense_threshold);
         if (lane == 0 && part == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
         unsigned dd = dm;
-        for (int k = 0; dd; k++) {
+        for (int k = 0; dd; k = k + 1 == split ? 0 : k + 1) {
             const int f = __ffs(dd) - 1;
             dd &= dd - 1;
-            if (k % split != part) continue;
+            if (k != part) continue;
             if constexpr (sizeof(TO) == 8) {
                 if (P.dense_tc) {
                     s3_dense_tc<TI>(P, g * 32 + f, wr, lane);
