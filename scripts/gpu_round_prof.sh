@@ -11,7 +11,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
 done
 timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_s3|k_s2|k_row_merge" -s 0 -c 5 \
   -o gpurun_out/prof_${TAG}_C2 python bench.py --config C2 --profile --steps 1 --warmup 0 > /dev/null 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_s3" -s 0 -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_s3" -s 0 -c 3 \
   -o gpurun_out/prof_${TAG}_C3 python bench.py --config C3 --profile --steps 1 --warmup 0 > /dev/null 2>&1
 for d in f32 f16; do for c in C2 C3; do
 timeout 300 python bench.py --config $c --dtype $d --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/qb_${TAG}_${d}_$c.json 2>/dev/null
