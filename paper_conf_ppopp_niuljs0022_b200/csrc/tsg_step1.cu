@@ -707,25 +707,48 @@ __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
 }
 
 // transposed tile masks: maskT[c] bit r <=> nonzero (r,c)  (used by the item-driven paths)
+// 8x8 bit-matrix transpose in a 64-bit word (byte i = row i, bit j = column j), three masked
+// delta swaps
+__device__ __forceinline__ uint64_t transpose8(uint64_t x) {
+    uint64_t t;
+    t = (x ^ (x >> 7)) & 0x00AA00AA00AA00AAull;
+    x = x ^ t ^ (t << 7);
+    t = (x ^ (x >> 14)) & 0x0000CCCC0000CCCCull;
+    x = x ^ t ^ (t << 14);
+    t = (x ^ (x >> 28)) & 0x00000000F0F0F0F0ull;
+    x = x ^ t ^ (t << 28);
+    return x;
+}
+
+// transposed masks (maskT[c] bit r <=> mask[r] bit c): the 16x16 tile as four 8x8 blocks,
+// gathered with byte permutes, transposed in 64-bit words and scattered back
 __global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ maskT) {
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nt) return;
     const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
-    uint4 a = __ldg(p), b = __ldg(p + 1);
-    uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
-    uint32_t col[TILE];
+    const uint4 a = __ldg(p), b = __ldg(p + 1);
+    const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};  // w[k] = row 2k | row 2k+1 << 16
+    uint64_t y[2][2];  // y[rb][cb] = transpose of rows 8rb..8rb+7 x columns 8cb..8cb+7
 #pragma unroll
-    for (int c = 0; c < TILE; c++) col[c] = 0;
+    for (int rb = 0; rb < 2; rb++)
 #pragma unroll
-    for (int r = 0; r < TILE; r++) {
-        uint32_t m = (w[r >> 1] >> (16 * (r & 1))) & 0xffffu;
+        for (int cb = 0; cb < 2; cb++) {
+            const uint32_t sel = cb | (2 + cb) << 4 | (4 + cb) << 8 | (6 + cb) << 12;
+            const uint32_t lo = __byte_perm(w[4 * rb], w[4 * rb + 1], sel);
+            const uint32_t hi = __byte_perm(w[4 * rb + 2], w[4 * rb + 3], sel);
+            y[rb][cb] = transpose8((uint64_t)lo | (uint64_t)hi << 32);
+        }
+    uint32_t o[8];  // o[m] = column 2m | column 2m+1 << 16, column c = byte c%8 of y[0][c/8] | of y[1][c/8] << 8
 #pragma unroll
-        for (int c = 0; c < TILE; c++) col[c] |= ((m >> c) & 1u) << r;
+    for (int m = 0; m < 8; m++) {
+        const int c = 2 * m, cb = c >> 3, k = c & 7, kk = k & 3;
+        const uint32_t h0 = k >= 4 ? (uint32_t)(y[0][cb] >> 32) : (uint32_t)y[0][cb];
+        const uint32_t h1 = k >= 4 ? (uint32_t)(y[1][cb] >> 32) : (uint32_t)y[1][cb];
+        o[m] = __byte_perm(h0, h1, kk | (4 + kk) << 4 | (kk + 1) << 8 | (5 + kk) << 12);
     }
-    uint4 *o = reinterpret_cast<uint4 *>(maskT + t * TILE);
-    o[0] = make_uint4(col[0] | col[1] << 16, col[2] | col[3] << 16, col[4] | col[5] << 16, col[6] | col[7] << 16);
-    o[1] = make_uint4(col[8] | col[9] << 16, col[10] | col[11] << 16, col[12] | col[13] << 16,
-                      col[14] | col[15] << 16);
+    uint4 *q = reinterpret_cast<uint4 *>(maskT + t * TILE);
+    q[0] = make_uint4(o[0], o[1], o[2], o[3]);
+    q[1] = make_uint4(o[4], o[5], o[6], o[7]);
 }
 
 // ------------------------------------------------------------------------------------------

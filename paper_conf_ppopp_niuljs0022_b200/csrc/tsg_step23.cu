@@ -558,48 +558,6 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
             for (int i = 0; i < nb; i++) rel |= (S.mA[i][r] & S.oB[i]) ? (1u << i) : 0u;
         }
 #endif
-#ifdef TSG_MED_SPAN
-        // span form: per pair, lane r walks B's entries from row min(c) to row max(c) of
-        // mask_A[r] & rowOcc(B) in storage order (row c ascending, then j: ascending k per slot),
-        // skipping rows outside the set; j comes from B's idx byte, a from A's row r by rank
-        if (rel) {
-            const TI *vAb = static_cast<const TI *>(P.vA), *vBb = static_cast<const TI *>(P.vB);
-            uint32_t rl = rel;
-            while (rl) {
-                const int pi = __ffs(rl) - 1;
-                rl &= rl - 1;
-                const uint32_t mAr = S.mA[pi][r];
-                const uint32_t ma = mAr & S.oB[pi];
-                const TI *va = vAb + S.zA[pi] + S.rA[pi][r];
-                const int64_t zB = S.zB[pi];
-                const int cmin = __ffs(ma) - 1, cmax = 31 - __clz(ma);
-                int e = S.rB[pi][cmin];
-                const int eend = S.rB[pi][cmax] + __popc((uint32_t)S.mB[pi][cmax]);
-                const TI *vb = vBb + zB;
-                const uint8_t *ib = P.ixB + zB;
-                const int na = __popc(mAr);
-                const TO a0 = vcvt<TO>(va[0]);
-                const TO a1 = na > 1 ? vcvt<TO>(va[1]) : (TO)0;
-                const TO a2 = na > 2 ? vcvt<TO>(va[2]) : (TO)0;
-                int curc = -1;
-                TO a = (TO)0;
-#pragma unroll 2
-                for (; e < eend; e++) {
-                    const uint32_t ix = ib[e];
-                    const int c = (int)(ix >> 4);
-                    const TO b = vcvt<TO>(vb[e]);
-                    if (!((ma >> c) & 1u)) continue;
-                    if (c != curc) {
-                        curc = c;
-                        const int k = __popc(mAr & ((1u << c) - 1u));
-                        a = k == 0 ? a0 : k == 1 ? a1 : k == 2 ? a2 : vcvt<TO>(va[k]);
-                    }
-                    TO *sl = acc + (ix & 15u) * 16;
-                    *sl = vfma(a, b, *sl);
-                }
-            }
-        }
-#else
         if (rel) {
             ItemStream<TI, TO> it;
             it.rel = rel;
@@ -615,7 +573,6 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
                 accumulate_row(aY, bY0, bY1, bY2, mY, vY, acc);
             }
         }
-#endif
         __syncwarp();
     }
     // compaction through mask_C[r]; every slot the tile touched is in mask_C[r] and is reset to
