@@ -110,6 +110,9 @@ struct StepParams {
     int dtype_in;          // tsg_dtype of A and B
     const uint32_t *work;  // step-2 class split
     const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
+    // step-3 classes per group of 32 C tiles (bit i = tile 32g+i), written by step 2: medium / dense
+    // tiles among the light tiles (k_s2_light) and among the heavy tiles (k_s2)
+    uint32_t *medL, *medH, *denL, *denH;
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     int dense_tc;          // step 3: fp64 dense tiles on the tensor cores (DMMA), TSG_DENSE_TC

@@ -202,6 +202,13 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P.rpC = row_ptr;
     P.mC = mask;
     P.work = work;
+    {
+        const int64_t ng = (ntC + 31) / 32;
+        P.medL = tmp.get<uint32_t>(ng);
+        P.medH = tmp.get<uint32_t>(ng);
+        P.denL = tmp.get<uint32_t>(ng);
+        P.denH = tmp.get<uint32_t>(ng);
+    }
     P.dense_threshold = TH;
     P.small_max = SMALL_NNZ;
     P.dense_tc = ((flags & TSG_DENSE_TC) || getenv("TSG_DENSE_TC")) ? 1 : 0;  // env: tuning only

@@ -82,9 +82,13 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
     __shared__ uint32_t wsm[8 * T2L];
     uint32_t *w = wsm + threadIdx.x;
     const int64_t stride = (int64_t)gridDim.x * T2L;
+    const int lane = threadIdx.x & 31;
     u64c nl = 0, nd = 0;
-    for (int64_t t = (int64_t)blockIdx.x * T2L + threadIdx.x; t < P.ntC; t += stride) {
-        if (P.work[t] > (uint32_t)LIGHT_WORK) continue;
+    // warp-uniform loop: the 32 lanes of a warp hold the 32 tiles of one group
+    for (int64_t t0 = (int64_t)blockIdx.x * T2L + (threadIdx.x & ~31); t0 < P.ntC; t0 += stride) {
+        const int64_t t = t0 + lane;
+        int total = -1;
+        if (t < P.ntC && P.work[t] <= (uint32_t)LIGHT_WORK) {
         nl++;
 #pragma unroll
         for (int q = 0; q < 8; q++) w[q * T2L] = 0;
@@ -119,7 +123,7 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
         }
         uint32_t m[8];
         uint32_t rp[4] = {0, 0, 0, 0};
-        int total = 0;
+        total = 0;
 #pragma unroll
         for (int q = 0; q < 8; q++) m[q] = w[q * T2L];
 #pragma unroll
@@ -133,6 +137,14 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
         *reinterpret_cast<uint4 *>(P.rpC + t * TILE) = make_uint4(rp[0], rp[1], rp[2], rp[3]);
         P.tnzC[t] = total;
         nd += total >= P.dense_threshold;
+        }
+        // step-3 classes of the group's light tiles (medium / dense bit masks; heavy tiles: k_s2)
+        const unsigned mm = __ballot_sync(FULL, total > P.small_max && total < P.dense_threshold);
+        const unsigned dn = __ballot_sync(FULL, total >= P.dense_threshold);
+        if (lane == 0) {
+            P.medL[t0 >> 5] = mm;
+            P.denL[t0 >> 5] = dn;
+        }
     }
     for (int o = 16; o > 0; o >>= 1) nl += __shfl_xor_sync(FULL, nl, o);
     if ((threadIdx.x & 31) == 0 && nl) atomicAdd(&P.cnt->n2light, nl);
@@ -156,6 +168,7 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
         const bool v = t < P.ntC;
         const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;  // k_s2_light's class
         unsigned hm = __ballot_sync(FULL, v && !light);
+        unsigned medH = 0, denH = 0;  // step-3 classes of the group's heavy tiles
         // heavy tiles: two at a time, a half warp each, lane r owns row r; per batch of 16 pairs
         // lane i stages pair i's A and B masks (4 x 16-byte cp.async, all in flight at once)
         while (hm) {
@@ -213,7 +226,14 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
                 if (r == 0) P.tnzC[th] = tot;
             }
             const unsigned dn = __ballot_sync(FULL, hv && r == 0 && tot >= P.dense_threshold);
+            const unsigned md = __ballot_sync(FULL, hv && r == 0 && tot > P.small_max && tot < P.dense_threshold);
             if (lane == 0 && dn) atomicAdd(&P.cnt->n2dense, (u64c)__popc(dn));
+            denH |= ((dn & 1u) ? 1u << f0 : 0u) | ((dn >> 16) & 1u ? 1u << f1 : 0u);
+            medH |= ((md & 1u) ? 1u << f0 : 0u) | ((md >> 16) & 1u ? 1u << f1 : 0u);
+        }
+        if (lane == 0) {
+            P.medH[g] = medH;
+            P.denH[g] = denH;
         }
         const unsigned lm = __ballot_sync(FULL, light), vm = __ballot_sync(FULL, v);
         if (lane == 0 && vm != lm) atomicAdd(&P.cnt->n2heavy, (u64c)(__popc(vm) - __popc(lm)));
@@ -807,11 +827,9 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
     const int64_t ngroups = (P.ntC + 31) / 32;
     const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
     for (int64_t g = (int64_t)blockIdx.x * (T3 / 32) + w; g < ngroups; g += gstride) {
-        const int64_t t = g * 32 + lane;
-        const bool v = t < P.ntC && !(P.skip && P.skip[t]);
-        const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
-        const bool med = v && nz < P.dense_threshold && nz > P.small_max;
-        unsigned mm = __ballot_sync(FULL, med);
+        unsigned mm = P.medL[g] | P.medH[g];  // the group's medium tiles (step 2 classified them)
+        if (!mm) continue;                    // warp-uniform
+        if (P.skip) mm &= ~__ballot_sync(FULL, g * 32 + lane < P.ntC && P.skip[g * 32 + lane]);
         if (lane == 0 && mm) atomicAdd(&P.cnt->n3medium, (u64c)__popc(mm));
         auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
             const int f0 = __ffs(mm) - 1;
@@ -852,10 +870,9 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
     for (int64_t u = (int64_t)blockIdx.x * (T3 / 32) + w; u < nunits; u += gstride) {
         const int64_t g = u / split;
         const int part = (int)(u - g * split);
-        const int64_t t = g * 32 + lane;
-        const bool v = t < P.ntC && !(P.skip && P.skip[t]);
-        const int nz = v ? (int)(P.tnzC[t + 1] - P.tnzC[t]) : 0;
-        const unsigned dm = __ballot_sync(FULL, v && nz >= P.dense_threshold);
+        unsigned dm = P.denL[g] | P.denH[g];  // the group's dense tiles (step 2 classified them)
+        if (!dm) continue;                    // warp-uniform
+        if (P.skip) dm &= ~__ballot_sync(FULL, g * 32 + lane < P.ntC && P.skip[g * 32 + lane]);
         if (lane == 0 && part == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
         unsigned dd = dm;
         for (int k = 0; dd; k = k + 1 == split ? 0 : k + 1) {
