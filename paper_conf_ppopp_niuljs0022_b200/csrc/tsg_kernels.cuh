@@ -26,6 +26,7 @@ struct DevCounters {
     u64c next3;        // work counter of the step-3 row kernel
     u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
     u64c n2dense;      // C tiles with nnz >= t_nnz (step 2 counts them; step 3 launches the dense kernel iff > 0)
+    u64c q[5][16];     // work-queue counters of the step-2/3 kernels, one 128-byte line each
 };
 
 constexpr int ROW_T = 256;        // threads of a step-1 row CTA
@@ -113,6 +114,7 @@ struct StepParams {
     // step-3 classes per group of 32 C tiles (bit i = tile 32g+i), written by step 2: medium / dense
     // tiles among the light tiles (k_s2_light) and among the heavy tiles (k_s2)
     uint32_t *medL, *medH, *denL, *denH;
+    int qchunk[5];         // work-queue units per request (k_s2_light, k_s2, k_s3_small, k_s3, k_s3_dense)
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     int dense_tc;          // step 3: fp64 dense tiles on the tensor cores (DMMA), TSG_DENSE_TC

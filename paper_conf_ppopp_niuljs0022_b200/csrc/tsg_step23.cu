@@ -22,6 +22,9 @@
 // (pairs ascending K, then c ascending), so no atomics are needed and results are bitwise
 // deterministic (readings A8/A16).
 #include <algorithm>
+#include <cstdlib>
+#include <map>
+#include <mutex>
 
 #include <cuda_fp16.h>
 
@@ -69,6 +72,43 @@ __device__ __forceinline__ uint32_t rows_meeting(const uint4 &a0, const uint4 &a
     return rows;
 }
 
+// Dynamic work distribution for the step-2/3 kernels: warps take the next `chunk` units (groups
+// of 32 C tiles) from a per-kernel counter, so the warps running at any moment work on
+// neighbouring C tiles (their pairs' A and B tiles stay in L2) and a warp that drew light groups
+// takes more.  The next chunk is requested one chunk ahead, so the atomic's latency overlaps the
+// current work; `chunk` (host-chosen, about 16 requests per warp) keeps the counter cold.
+struct WorkQueue {
+    unsigned long long *ctr;
+    int64_t n;
+    int chunk;          // 0: static grid-stride distribution (unit = first, first + stride, ...)
+    long long nxt = 0;  // lane 0: first unit of the next chunk
+    int64_t cur = 0, end = 0, stride = 0;
+    __device__ WorkQueue(unsigned long long *c, int64_t units, int ch, int lane, int warps_per_cta)
+        : ctr(c), n(units), chunk(ch) {
+        if (ch == 0) {
+            cur = (int64_t)blockIdx.x * warps_per_cta + (threadIdx.x >> 5);
+            stride = (int64_t)gridDim.x * warps_per_cta;
+        } else if (lane == 0) {
+            nxt = (long long)atomicAdd(ctr, (unsigned long long)ch);
+        }
+    }
+    __device__ __forceinline__ bool next(int64_t &u, int lane) {
+        if (chunk == 0) {
+            u = cur;
+            cur += stride;
+            return u < n;
+        }
+        if (cur >= end) {
+            cur = (int64_t)__shfl_sync(FULL, nxt, 0);
+            if (cur >= n) return false;
+            end = min(cur + (int64_t)chunk, n);
+            if (lane == 0) nxt = (long long)atomicAdd(ctr, (unsigned long long)chunk);
+        }
+        u = cur++;
+        return true;
+    }
+};
+
 // ==========================================================================================
 // step 2
 // ==========================================================================================
@@ -81,11 +121,12 @@ constexpr int T2L = 256;
 __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
     __shared__ uint32_t wsm[8 * T2L];
     uint32_t *w = wsm + threadIdx.x;
-    const int64_t stride = (int64_t)gridDim.x * T2L;
     const int lane = threadIdx.x & 31;
     u64c nl = 0, nd = 0;
-    // warp-uniform loop: the 32 lanes of a warp hold the 32 tiles of one group
-    for (int64_t t0 = (int64_t)blockIdx.x * T2L + (threadIdx.x & ~31); t0 < P.ntC; t0 += stride) {
+    // the 32 lanes of a warp hold the 32 tiles of one group
+    WorkQueue wq(&P.cnt->q[0][0], (P.ntC + 31) / 32, P.qchunk[0], lane, T2L / 32);
+    for (int64_t gq; wq.next(gq, lane);) {
+        const int64_t t0 = gq * 32;
         const int64_t t = t0 + lane;
         int total = -1;
         if (t < P.ntC && P.work[t] <= (uint32_t)LIGHT_WORK) {
@@ -162,8 +203,8 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     __shared__ uint16_t sOB[T2 / 16][BATCH];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
     const int64_t ngroups = (P.ntC + 31) / 32;
-    const int64_t gstride = (int64_t)gridDim.x * (T2 / 32);
-    for (int64_t g = (int64_t)blockIdx.x * (T2 / 32) + (threadIdx.x >> 5); g < ngroups; g += gstride) {
+    WorkQueue wq(&P.cnt->q[1][0], ngroups, P.qchunk[1], lane, T2 / 32);
+    for (int64_t g; wq.next(g, lane);) {
         const int64_t t = g * 32 + lane;
         const bool v = t < P.ntC;
         const bool light = v && P.work[t] <= (uint32_t)LIGHT_WORK;  // k_s2_light's class
@@ -295,8 +336,8 @@ __global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
     const int lane = threadIdx.x & 31;
     uint8_t *map = mapsm[threadIdx.x >> 5];
     const int64_t ngroups = (P.ntC + 31) / 32;
-    const int64_t gstride = (int64_t)gridDim.x * (TS / 32);
-    for (int64_t g = (int64_t)blockIdx.x * (TS / 32) + (threadIdx.x >> 5); g < ngroups; g += gstride) {
+    WorkQueue wq(&P.cnt->q[2][0], ngroups, P.qchunk[2], lane, TS / 32);
+    for (int64_t g; wq.next(g, lane);) {
         const int64_t tl = g * 32 + lane;
         const bool v = tl < P.ntC && !(P.skip && P.skip[tl]);
         const int nz = v ? (int)(P.tnzC[tl + 1] - P.tnzC[tl]) : 0;
@@ -825,8 +866,8 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
 #pragma unroll
     for (int j = 0; j < TILE; j++) acc[j * 16] = (TO)0;
     const int64_t ngroups = (P.ntC + 31) / 32;
-    const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
-    for (int64_t g = (int64_t)blockIdx.x * (T3 / 32) + w; g < ngroups; g += gstride) {
+    WorkQueue wq(&P.cnt->q[3][0], ngroups, P.qchunk[3], lane, T3 / 32);
+    for (int64_t g; wq.next(g, lane);) {
         unsigned mm = P.medL[g] | P.medH[g];  // the group's medium tiles (step 2 classified them)
         if (!mm) continue;                    // warp-uniform
         if (P.skip) mm &= ~__ballot_sync(FULL, g * 32 + lane < P.ntC && P.skip[g * 32 + lane]);
@@ -866,8 +907,8 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
     // it: dense tiles cluster (FEM strips), and a group's dense tiles done by one warp one after
     // the other would make the kernel a chain of serial per-pair latencies
     const int64_t nunits = (P.ntC + 31) / 32 * split;
-    const int64_t gstride = (int64_t)gridDim.x * (T3 / 32);
-    for (int64_t u = (int64_t)blockIdx.x * (T3 / 32) + w; u < nunits; u += gstride) {
+    WorkQueue wq(&P.cnt->q[4][0], nunits, P.qchunk[4], lane, T3 / 32);
+    for (int64_t u; wq.next(u, lane);) {
         const int64_t g = u / split;
         const int part = (int)(u - g * split);
         unsigned dm = P.denL[g] | P.denH[g];  // the group's dense tiles (step 2 classified them)
@@ -890,35 +931,84 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
     }
 }
 
-unsigned grid_groups(int64_t ntC, int warps_per_cta) {
-    const int64_t groups = (ntC + 31) / 32;
-    const int64_t g = std::min<int64_t>(ceil_div(std::max<int64_t>(groups, 1), warps_per_cta), 148LL * 32);
-    return (unsigned)std::max<int64_t>(g, 1);
+// Launch shape of a step-2/3 kernel over `units` work units (groups of 32 C tiles), `wpc` warps
+// per CTA.  Many units per warp: a persistent grid (the CTAs resident at once: SM count x
+// occupancy) with the work queue, so the warps running at any moment work on neighbouring C tiles
+// (the A and B tiles their pairs read stay in L2) and the load balances; `chunk` units per
+// request grows with the units per warp (C2: 1, R-MAT: 4-8) so the counter stays cold.  Few
+// units per warp (C3), and dense tiles: static grid-stride over up to 32 CTAs per SM (measured
+// faster there).
+struct Shape {
+    unsigned grid;
+    int chunk;
+};
+template <typename K>
+Shape step_shape(K kernel, int threads, int64_t units, int64_t min_per_warp = 4) {
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, int> cache;  // (kernel, device) -> resident CTAs per GPU
+    const int wpc = threads / 32;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int resident;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find({(const void *)kernel, dev});
+        if (it == cache.end()) {
+            int nsm = 148, occ = 1;
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, 0);
+            it = cache.emplace(std::make_pair((const void *)kernel, dev), nsm * std::max(occ, 1)).first;
+        }
+        resident = it->second;
+    }
+    units = std::max<int64_t>(units, 1);
+    const int64_t per_warp = units / ((int64_t)resident * wpc);
+    int64_t chunk = per_warp >= min_per_warp ? std::max<int64_t>(1, std::min<int64_t>(8, per_warp / 256)) : 0;
+    if (const char *e = getenv("TSG_QUEUE_CHUNK")) chunk = atoi(e);  // tuning only (0 = static)
+    if (chunk <= 0) return {(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, wpc), 148LL * 32)), 0};
+    return {(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, wpc), resident)), (int)chunk};
 }
 
 }  // namespace
 
 void launch_step2(const StepParams &P, cudaStream_t s) {
     if (P.ntC <= 0) return;
-    TSG_LAUNCH(k_s2_light, (unsigned)std::min<int64_t>(ceil_div(P.ntC, T2L), 148LL * 8 * 4), T2L, 0, s, P);
-    TSG_LAUNCH(k_s2, grid_groups(P.ntC, T2 / 32), T2, 0, s, P);
+    const int64_t groups = (P.ntC + 31) / 32;
+    StepParams Q = P;
+    const Shape sl = step_shape(k_s2_light, T2L, groups), sh = step_shape(k_s2, T2, groups);
+    Q.qchunk[0] = sl.chunk;
+    Q.qchunk[1] = sh.chunk;
+    TSG_LAUNCH(k_s2_light, sl.grid, T2L, 0, s, Q);
+    TSG_LAUNCH(k_s2, sh.grid, T2, 0, s, Q);
 }
 
 template <typename TI, typename TO>
 static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s) {
+    const int64_t groups = (P.ntC + 31) / 32;
+    StepParams Q = P;
     if (P.small_max > 0) {
-        if (P.small_stage)
-            TSG_LAUNCH((k_s3_small<TI, TO, true>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
-        else
-            TSG_LAUNCH((k_s3_small<TI, TO, false>), grid_groups(P.ntC, TS / 32), TS, 0, s, P);
+        if (P.small_stage) {
+            const Shape sp = step_shape(k_s3_small<TI, TO, true>, TS, groups);
+            Q.qchunk[2] = sp.chunk;
+            TSG_LAUNCH((k_s3_small<TI, TO, true>), sp.grid, TS, 0, s, Q);
+        } else {
+            const Shape sp = step_shape(k_s3_small<TI, TO, false>, TS, groups);
+            Q.qchunk[2] = sp.chunk;
+            TSG_LAUNCH((k_s3_small<TI, TO, false>), sp.grid, TS, 0, s, Q);
+        }
     }
-    TSG_LAUNCH((k_s3<TI, TO>), grid_groups(P.ntC, T3 / 32), T3, 0, s, P);
+    {
+        const Shape sp = step_shape(k_s3<TI, TO>, T3, groups);
+        Q.qchunk[3] = sp.chunk;
+        TSG_LAUNCH((k_s3<TI, TO>), sp.grid, T3, 0, s, Q);
+    }
     if (n_dense > 0) {
         // dense tiles per group of 32: spread a group over up to 8 warps when dense tiles are common
-        const int64_t groups = (P.ntC + 31) / 32;
         const int split = (int)std::max<int64_t>(1, std::min<int64_t>(8, 32 * n_dense / (groups * 4)));
-        const int64_t ctas = std::min<int64_t>(ceil_div(groups * split, T3 / 32), 148LL * 32);
-        TSG_LAUNCH((k_s3_dense<TI, TO>), (unsigned)std::max<int64_t>(ctas, 1), T3, 0, s, P, split);
+        // (dense tiles: static distribution, measured faster on C3)
+        const Shape sp = step_shape(k_s3_dense<TI, TO>, T3, groups * split, INT64_MAX);
+        Q.qchunk[4] = sp.chunk;
+        TSG_LAUNCH((k_s3_dense<TI, TO>), sp.grid, T3, 0, s, Q, split);
     }
 }
 
