@@ -1,9 +1,12 @@
 // tsg_scan.cu -- device exclusive prefix sum with int64 output (the "device prefix-sum
 // allocation" between the steps: tile offsets, nonzero offsets).
 //
-// Three phases per level: (1) each 1024-thread CTA reduces 8192 inputs to one sum, (2) the sums
-// are scanned (recursively, same code), (3) each CTA rescans its 8192 inputs and adds its base.
-// HBM traffic: 2 reads + 1 write of the input; used on arrays of at most a few hundred M entries.
+// Single pass (chained scan with decoupled look-back): each 1024-thread CTA takes the next 8192
+// inputs in launch order (ticket counter), publishes its sum, finds its prefix from the closest
+// predecessors' published sums / inclusive prefixes (warp-parallel look-back, 32 predecessors per
+// round), publishes its inclusive prefix and writes its outputs.  HBM traffic: 1 read + 1 write;
+// one memset + one launch per scan.  In place (in == out) is allowed: a CTA reads all its inputs
+// before writing.
 #include "tsg_internal.cuh"
 
 namespace tsg {
@@ -44,33 +47,62 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *total) {
     return base + incl - v;
 }
 
-template <typename Tin>
-__global__ void __launch_bounds__(SCAN_T) k_scan_reduce(const Tin *__restrict__ in, int64_t n,
-                                                        int64_t *__restrict__ sums) {
-    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_IPT;
-    int64_t s = 0;
-#pragma unroll
-    for (int i = 0; i < SCAN_IPT; i++)
-        if (base + i < n) s += (int64_t)in[base + i];
-    int64_t total;
-    block_excl_scan(s, &total);
-    if (threadIdx.x == 0) sums[blockIdx.x] = total;
+// tile status word: flag in the top 2 bits (0 = not ready, 1 = aggregate, 2 = inclusive prefix),
+// value in the low 62 bits (all scanned quantities are counts < 2^62)
+constexpr uint64_t ST_AGG = 1ull << 62, ST_PRE = 2ull << 62, ST_VAL = (1ull << 62) - 1;
+
+__device__ __forceinline__ uint64_t ld_status(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_status(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 template <typename Tin>
-__global__ void __launch_bounds__(SCAN_T) k_scan_down(const Tin *in, int64_t n, int64_t *out,
-                                                      const int64_t *__restrict__ block_base) {
-    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_IPT;
+__global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n, int64_t *out, uint64_t *status,
+                                                      unsigned long long *ticket) {
+    __shared__ int64_t s_bid, s_base;
+    if (threadIdx.x == 0) s_bid = (int64_t)atomicAdd(ticket, 1ull);
+    __syncthreads();
+    const int64_t b = s_bid;
+    const int64_t base = b * SCAN_TILE + (int64_t)threadIdx.x * SCAN_IPT;
     int64_t v[SCAN_IPT];
-    int64_t s = 0;
+    int64_t sum = 0;
 #pragma unroll
     for (int i = 0; i < SCAN_IPT; i++) {
         v[i] = (base + i < n) ? (int64_t)in[base + i] : 0;
-        s += v[i];
+        sum += v[i];
     }
     int64_t total;
-    int64_t pre = block_excl_scan(s, &total);  // all reads of `in` by this CTA happen before
-    pre += block_base ? block_base[blockIdx.x] : 0;
+    int64_t pre = block_excl_scan(sum, &total);  // all reads of `in` by this CTA happen before
+    if (threadIdx.x < 32) {
+        const int lane = threadIdx.x;
+        int64_t excl = 0;
+        if (b == 0) {
+            if (lane == 0) st_status(status, ST_PRE | (uint64_t)total);
+        } else {
+            if (lane == 0) st_status(status + b, ST_AGG | (uint64_t)total);
+            for (int64_t j = b - 1;; j -= 32) {
+                const int64_t idx = j - lane;  // lane 0 = closest predecessor
+                uint64_t st = idx >= 0 ? ld_status(status + idx) : ST_PRE;
+                while (__any_sync(0xffffffffu, (st >> 62) == 0))
+                    if ((st >> 62) == 0) st = ld_status(status + idx);
+                const unsigned pm = __ballot_sync(0xffffffffu, (st >> 62) == 2);
+                const int first = pm ? __ffs(pm) - 1 : 32;
+                int64_t x = lane <= first ? (int64_t)(st & ST_VAL) : 0;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+                excl += x;
+                if (pm) break;
+            }
+            if (lane == 0) st_status(status + b, ST_PRE | (uint64_t)(excl + total));
+        }
+        if (lane == 0) s_base = excl;
+    }
+    __syncthreads();
+    pre += s_base;
 #pragma unroll
     for (int i = 0; i < SCAN_IPT; i++) {
         if (base + i < n) out[base + i] = pre;
@@ -89,15 +121,11 @@ void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buff
         TSG_LAUNCH(k_set_zero_i64, 1, 1, 0, s, out);
         return;
     }
-    int64_t nb = ceil_div(n, SCAN_TILE);
-    if (nb == 1) {
-        TSG_LAUNCH((k_scan_down<Tin>), 1, SCAN_T, 0, s, in, n, out, (const int64_t *)nullptr);
-        return;
-    }
-    int64_t *sums = tmp.get<int64_t>(nb + 1);
-    TSG_LAUNCH((k_scan_reduce<Tin>), (unsigned)nb, SCAN_T, 0, s, in, n, sums);
-    exclusive_scan<int64_t>(sums, sums, nb, s, tmp);
-    TSG_LAUNCH((k_scan_down<Tin>), (unsigned)nb, SCAN_T, 0, s, in, n, out, (const int64_t *)sums);
+    const int64_t nb = ceil_div(n, SCAN_TILE);
+    uint64_t *status = tmp.get<uint64_t>(nb + 1);  // [0, nb): tile status, [nb]: ticket
+    TSG_CUDA(cudaMemsetAsync(status, 0, sizeof(uint64_t) * (nb + 1), s));
+    TSG_LAUNCH((k_scan_1pass<Tin>), (unsigned)nb, SCAN_T, 0, s, in, n, out, status,
+               reinterpret_cast<unsigned long long *>(status + nb));
 }
 
 template void exclusive_scan<int64_t>(const int64_t *, int64_t *, int64_t, cudaStream_t, Buffers &);
