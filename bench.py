@@ -32,7 +32,7 @@ METRIC = "fp64 C=A^2 GFLOPS (2×products/time) at 1/2/4/8 B200; % HBM roofline"
 UNIT = "GFLOPS"
 L2_BYTES = 126 * 2 ** 20
 ROW_BLOCKS = {"C5": 4}
-E2E_BLOCKS = 4                 # tile-row blocks of the e2e leg when C fits the pinned host buffer
+E2E_BLOCKS = int(os.environ.get("TSG_E2E_BLOCKS", "4"))  # tile-row blocks of the e2e leg when C fits the pinned host buffer
 E2E_PINNED_MAX = 24 * 2 ** 30  # bytes of pinned host memory the e2e leg may use for C
 VDT = {"f64": np.float64, "f32": np.float32, "f16": np.float16}  # tile-row blocks per step on one GPU (C5's C is ~144 GB in tile form)
 
