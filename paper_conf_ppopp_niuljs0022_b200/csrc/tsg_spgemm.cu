@@ -42,6 +42,49 @@ struct Timer {
 };
 }  // namespace
 
+namespace {
+// A side stream forked from `s` (one cached non-blocking stream and two events per host thread
+// and device); join() makes `s` wait for the side work, and the destructor joins if nothing did
+class SideStream {
+   public:
+    explicit SideStream(cudaStream_t s) : s_(s) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        static thread_local Res res[16];
+        r_ = &res[dev & 15];
+        if (!r_->side) {
+            TSG_CUDA(cudaStreamCreateWithFlags(&r_->side, cudaStreamNonBlocking));
+            TSG_CUDA(cudaEventCreateWithFlags(&r_->fork, cudaEventDisableTiming));
+            TSG_CUDA(cudaEventCreateWithFlags(&r_->joinev, cudaEventDisableTiming));
+        }
+        TSG_CUDA(cudaEventRecord(r_->fork, s_));
+        TSG_CUDA(cudaStreamWaitEvent(r_->side, r_->fork, 0));
+    }
+    cudaStream_t stream() const { return r_->side; }
+    void done() { TSG_CUDA(cudaEventRecord(r_->joinev, r_->side)); recorded_ = true; }
+    void join() {
+        if (joined_) return;
+        if (!recorded_) done();
+        TSG_CUDA(cudaStreamWaitEvent(s_, r_->joinev, 0));
+        joined_ = true;
+    }
+    ~SideStream() {
+        if (joined_) return;
+        if (!recorded_) cudaEventRecord(r_->joinev, r_->side);
+        cudaStreamWaitEvent(s_, r_->joinev, 0);
+    }
+
+   private:
+    struct Res {
+        cudaStream_t side = nullptr;
+        cudaEvent_t fork = nullptr, joinev = nullptr;
+    };
+    cudaStream_t s_;
+    Res *r_;
+    bool recorded_ = false, joined_ = false;
+};
+}  // namespace
+
 void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Allocator &al, cudaStream_t s,
                 tsg_tiles *C, tsg_stats *st) {
     reset_call_launches();
@@ -70,14 +113,16 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     uint16_t *rowOccB = tmp.get<uint16_t>(B->nt);
     launch_occupancy(A->mask, ntA, nullptr, colOccA, s);
     launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
+    // transposed masks: first used by step 2, so they are computed on a side stream while step 1
+    // runs (joined before step 2, and on every exit path by the guard's destructor)
     uint16_t *mTA = tmp.get<uint16_t>(TILE * ntA);
-    launch_transpose(A->mask, ntA, mTA, s);
     uint16_t *mTB = mTA;  // A^2 (B's tiles are A's tiles): one transpose serves both.  A row slice
                           // of B shares B's mask pointer but not its tile count: transpose B then.
-    if (B->mask != A->mask || B->nt != A->nt) {
-        mTB = tmp.get<uint16_t>(TILE * B->nt);
-        launch_transpose(B->mask, B->nt, mTB, s);
-    }
+    if (B->mask != A->mask || B->nt != A->nt) mTB = tmp.get<uint16_t>(TILE * B->nt);
+    SideStream side(s);
+    launch_transpose(A->mask, ntA, mTA, side.stream());
+    if (mTB != mTA) launch_transpose(B->mask, B->nt, mTB, side.stream());
+    side.done();
     const bool lists = !(flags & TSG_STEP1_SCAN_ONLY) &&
                        ((flags & TSG_STEP1_LIST_ALWAYS) || (B->nt > 0 && B->nnz < 2 * B->nt));
     int64_t *lptr = nullptr;
@@ -178,6 +223,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     launch_compact(PC, s);
 
     // ---------------- a2: step 2
+    side.join();
     StepParams P{};
     P.ntC = ntC;
     P.pairBeg = pairBeg;

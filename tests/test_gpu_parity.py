@@ -520,3 +520,49 @@ def test_dense_tensor_core_nonfinite(tsg):
         assert_tiles_equal(got, ref, values=None)
         absref = oracle.csr_to_tiles(_abs_csr(a, b)).val
         assert_values_close(got["val"], ref.val, absref)
+
+
+def test_copy_to_host_async_pipeline(tsg):
+    """tsg_tiles_copy_to_host_async on a second stream, overlapping the next block's SpGEMM (the
+    bench's e2e leg): every block's host copy equals the oracle's tiles of that row block."""
+    import torch
+
+    A = gen.stencil27(12)
+    T = tiles_of(tsg, A)
+    cuts = [0, T.tile_m // 3, 2 * T.tile_m // 3, T.tile_m]
+    ref = oracle.expected_tiles(A, A, fma=True)
+    s_copy = torch.cuda.Stream()
+    outs, live = [], []
+    for b0, b1 in zip(cuts[:-1], cuts[1:]):
+        C = tsg.spgemm(tsg.slice_rows(T, b0, b1), T)
+        ev = torch.cuda.Event()
+        ev.record()
+        s_copy.wait_event(ev)
+        bufs = {k: torch.empty(v.numel(), dtype=torch.int16 if v.dtype == torch.uint16 else v.dtype, pin_memory=True)
+                for k, v in C.arrays().items()}
+        C.copy_to_host(bufs, stream=s_copy, blocking=False)
+        outs.append(bufs)
+        live.append(C)
+    s_copy.synchronize()
+    # stitch the blocks back together and compare with C = A^2
+    tp = [0]
+    cols, nnzs, rps, masks, idxs, vals = [], [], [], [], [], []
+    base_t = base_z = 0
+    for h in outs:
+        tp.extend((h["tile_ptr"][1:].numpy() + base_t).tolist())
+        nnzs.append(h["tile_nnz"][:-1].numpy() + base_z)
+        base_t += int(h["tile_ptr"][-1])
+        base_z += int(h["tile_nnz"][-1])
+        cols.append(h["tile_col"].numpy())
+        rps.append(h["row_ptr"].numpy())
+        masks.append(h["mask"].numpy().view(np.uint16))
+        idxs.append(h["idx"].numpy())
+        vals.append(h["val"].numpy())
+    nnzs.append(np.array([base_z]))
+    assert np.array_equal(np.array(tp), ref.tile_ptr)
+    assert np.array_equal(np.concatenate(cols), ref.tile_col)
+    assert np.array_equal(np.concatenate(nnzs), ref.tile_nnz)
+    assert np.array_equal(np.concatenate(rps), ref.row_ptr)
+    assert np.array_equal(np.concatenate(masks), ref.mask)
+    assert np.array_equal(np.concatenate(idxs), ref.idx)
+    assert bitwise_equal_values(np.concatenate(vals), ref.val)
