@@ -109,19 +109,28 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     TSG_CUDA(cudaMemsetAsync(cnt, 0, sizeof(DevCounters), s));
 
     // ---------------- a0: occupancy words, optional B row lists, optional product count
-    uint16_t *colOccA = tmp.get<uint16_t>(ntA);
+    // A inside B's tile arrays (A^2, or a row slice of B: SURVEY 8(e)'s rank shards and row blocks):
+    // A's tile t is B's tile t + off, so one pass over B gives A's helper words too
+    const int64_t off = (int64_t)(A->mask - B->mask) / TILE;
+    const bool inB = A->mask >= B->mask && (A->mask - B->mask) % TILE == 0 && off + ntA <= B->nt;
     uint16_t *rowOccB = tmp.get<uint16_t>(B->nt);
-    launch_occupancy(A->mask, ntA, nullptr, colOccA, s);
-    launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
+    uint16_t *colOccA;
+    if (inB) {
+        uint16_t *colOccB = tmp.get<uint16_t>(B->nt);
+        launch_occupancy(B->mask, B->nt, rowOccB, colOccB, s);
+        colOccA = colOccB + off;
+    } else {
+        colOccA = tmp.get<uint16_t>(ntA);
+        launch_occupancy(A->mask, ntA, nullptr, colOccA, s);
+        launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
+    }
     // transposed masks: first used by step 2, so they are computed on a side stream while step 1
     // runs (joined before step 2, and on every exit path by the guard's destructor)
-    uint16_t *mTA = tmp.get<uint16_t>(TILE * ntA);
-    uint16_t *mTB = mTA;  // A^2 (B's tiles are A's tiles): one transpose serves both.  A row slice
-                          // of B shares B's mask pointer but not its tile count: transpose B then.
-    if (B->mask != A->mask || B->nt != A->nt) mTB = tmp.get<uint16_t>(TILE * B->nt);
+    uint16_t *mTB = tmp.get<uint16_t>(TILE * B->nt);
+    uint16_t *mTA = inB ? mTB + TILE * off : tmp.get<uint16_t>(TILE * ntA);
     SideStream side(s);
-    launch_transpose(A->mask, ntA, mTA, side.stream());
-    if (mTB != mTA) launch_transpose(B->mask, B->nt, mTB, side.stream());
+    launch_transpose(B->mask, B->nt, mTB, side.stream());
+    if (!inB) launch_transpose(A->mask, ntA, mTA, side.stream());
     side.done();
     const bool lists = !(flags & TSG_STEP1_SCAN_ONLY) &&
                        ((flags & TSG_STEP1_LIST_ALWAYS) || (B->nt > 0 && B->nnz < 2 * B->nt));
