@@ -211,14 +211,20 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    # one process per GPU; ranks beyond the visible GPUs share them (functional checks of the
+    # multi-rank path on a 1-GPU box with TSG_DIST_BACKEND=gloo -- not a measurement)
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     dist = None
     if world > 1:
         import torch.distributed as dist
 
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("TSG_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     A = gen.config(args.config)
     if args.dtype != "f64":
@@ -322,8 +328,8 @@ def main():
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
-    if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(dom)
+    if os.path.exists(tp) and world == 1 and K == 1 and args.dtype == "f64" and not args.aat:
+        traffic = json.load(open(tp)).get(dom)  # captured for the whole single-GPU fp64 call only
     bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz, vb) + \
         K * tile_bytes(Bt.tile_m, Bt.num_tiles, Bt.nnz, vb) + tile_bytes(Ashard.tile_m, ntC, nnzC, cb)
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",
