@@ -312,6 +312,38 @@ def main():
         prods = int(p.item())
     value = 2.0 * prods / (ms / 1e3) / 1e9
 
+    # the collectives around the sharded step, measured next to it (not in the
+    # metric: B is resident and C stays sharded): broadcast of B's seven arrays from rank 0 and the
+    # uneven all-gather + rebasing of the C shards into the full C on every rank
+    multi = None
+    if dist:
+        def timed(fn, reps=3):
+            ts = []
+            for _ in range(reps):
+                dist.barrier()
+                torch.cuda.synchronize()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                fn()
+                e1.record(stream)
+                e1.synchronize()
+                t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ts.append(float(t.item()))
+            return float(np.median(ts))
+
+        meta = (T.m, T.n, T.num_tiles, T.nnz)
+        t_b = timed(lambda: tdist.broadcast_tiles(Bt.arrays() if rank == 0 else None, meta if rank == 0 else None,
+                                                  0, dev))
+        t_r = None
+        if K == 1:
+            Cl = tsg.spgemm(shards[0], Bt)
+            t_r = timed(lambda: tdist.allgatherv_tiles(Cl), reps=2)
+            del Cl
+        multi = {"t_bcast_ms": t_b, "bcast_bytes": int(sum(v.numel() * v.element_size() for v in Bt.arrays().values())),
+                 "t_reassemble_ms": t_r, "backend": os.environ.get("TSG_DIST_BACKEND", "nccl"),
+                 "note": "not in the metric: B resident, C left sharded (SURVEY 8(e))"}
+
     # roofline of the dominant kernel (step 3 numeric unless another step is longer)
     bw, bw_src = peaks()
     nnzC, ntC = stats_last["nnz_c"], stats_last["tiles_c"]
@@ -441,6 +473,7 @@ def main():
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": int(launches),
+        "multi_gpu": multi,
         "clocks": clocks,
     }
     print(json.dumps(line), flush=True)
