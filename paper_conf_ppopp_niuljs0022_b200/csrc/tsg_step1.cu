@@ -628,7 +628,9 @@ __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
             valid = (P.rowOccB[posB] & P.colOccA[t]) != 0;
         }
         const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : ~0u;
-        sJ[u] = jr;
+        // the candidate's (pair, c) items (step 2's work estimate) ride in the top 5 bits
+        const uint32_t wk = st < 0 ? 1u : (uint32_t)__popc((uint32_t)(P.rowOccB[posB] & P.colOccA[t]));
+        sJ[u] = valid ? jr | (wk << 27) : ~0u;
         sPos[u] = posB;
         sK[u] = (uint32_t)lo;
         if (valid) atomicOr(&bm[jr >> 5], 1u << (jr & 31));
@@ -645,17 +647,21 @@ __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
         pre[w] = (uint32_t)run;
         run += __popc(bm[w]);
     }
+    uint32_t *cursor = reinterpret_cast<uint32_t *>(P.bigKeysB + o);  // per C tile, pass 3
     for (int64_t r = threadIdx.x; r < nC; r += RANK_T) {
         P.tCnt[base + r] = 0;
         P.tWork[base + r] = 0;
+        cursor[r] = 0;
     }
     __syncthreads();
-    // pass 2: pairs per C tile (and its tile column)
+    // pass 2: pairs and work per C tile (and its tile column)
     for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
-        const uint32_t jr = sJ[u];
-        if (jr == ~0u) continue;
+        const uint32_t jw = sJ[u];
+        if (jw == ~0u) continue;
+        const uint32_t jr = jw & 0x7ffffffu;
         const uint32_t rank = pre[jr >> 5] + __popc(bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
         atomicAdd(&P.tCnt[base + rank], 1u);
+        atomicAdd(&P.tWork[base + rank], jw >> 27);
         P.tJ[base + rank] = jlo + (int32_t)jr;
     }
     __syncthreads();
@@ -671,16 +677,17 @@ __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
         runc += P.tCnt[base + r];
     }
     __syncthreads();
-    // pass 3: scatter the pairs with per-tile cursors (tWork is the cursor until pass 4)
+    // pass 3: scatter the pairs with per-tile cursors
     for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
-        const uint32_t jr = sJ[u];
-        if (jr == ~0u) continue;
+        const uint32_t jw = sJ[u];
+        if (jw == ~0u) continue;
+        const uint32_t jr = jw & 0x7ffffffu;
         const uint32_t rank = pre[jr >> 5] + __popc(bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
-        const uint32_t slot = P.tStart[base + rank] + atomicAdd(&P.tWork[base + rank], 1u);
+        const uint32_t slot = P.tStart[base + rank] + atomicAdd(&cursor[rank], 1u);
         P.pairs[base + slot] = ((uint64_t)(a0 + sK[u]) << 32) | sPos[u];
     }
     __syncthreads();
-    // pass 4: each C tile's pairs in ascending A tile position (= ascending K), work estimate
+    // pass 4: each C tile's pairs in ascending A tile position (= ascending K)
     for (int64_t r = threadIdx.x; r < nC; r += RANK_T) {
         uint64_t *pp = P.pairs + base + P.tStart[base + r];
         const uint32_t n = P.tCnt[base + r];
@@ -693,12 +700,6 @@ __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
             }
             pp[k] = x;
         }
-        uint32_t wk = 0;
-        for (uint32_t i = 0; i < n; i++) {
-            const uint64_t x = pp[i];
-            wk += __popc((uint32_t)P.colOccA[(int64_t)(x >> 32)] & (uint32_t)P.rowOccB[(uint32_t)x]);
-        }
-        P.tWork[base + r] = wk;
     }
     if (threadIdx.x == 0) {
         P.nC[I] = nC;
