@@ -114,12 +114,66 @@ void Allocator::free(void *p, size_t bytes, cudaStream_t s) const {
         cudaFreeAsync(p, s);
 }
 
-int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {
-    int64_t v = 0;
-    TSG_CUDA(cudaMemcpyAsync(&v, dptr, sizeof(v), cudaMemcpyDeviceToHost, s));
+// Small device -> host reads (the blocking scalar reads between the steps) go through a kernel
+// that writes them into mapped pinned host memory, not through a D2H copy: a D2H copy queues
+// behind whatever the copy engine is already doing (a caller streaming the previous result to
+// the host), a kernel's posted writes do not.
+namespace {
+struct ExportArgs {
+    const uint8_t *src[4];
+    uint32_t bytes[4], off[4];
+    int n;
+    uint8_t *dst;
+};
+__global__ void k_export(ExportArgs a) {
+    for (int k = 0; k < a.n; k++)
+        for (uint32_t i = threadIdx.x; i < a.bytes[k]; i += blockDim.x) a.dst[a.off[k] + i] = a.src[k][i];
+}
+struct Mapped {
+    uint8_t *h = nullptr;
+    uint8_t *d = nullptr;
+};
+constexpr size_t MAPPED_BYTES = 4096;
+}  // namespace
+
+void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
+    int dev = 0;
+    TSG_CUDA(cudaGetDevice(&dev));
+    static thread_local Mapped m[16];
+    Mapped &mp = m[dev & 15];
+    if (!mp.h) {
+        void *h = nullptr, *d = nullptr;
+        TSG_CUDA(cudaHostAlloc(&h, MAPPED_BYTES, cudaHostAllocMapped | cudaHostAllocPortable));
+        TSG_CUDA(cudaHostGetDevicePointer(&d, h, 0));
+        mp.h = static_cast<uint8_t *>(h);
+        mp.d = static_cast<uint8_t *>(d);
+    }
+    ExportArgs a{};
+    uint32_t off = 0;
+    TSG_REQUIRE(segs.size() <= 4, TSG_ERR_INTERNAL, "too many device reads");
+    for (const DevRead &r : segs) {
+        TSG_REQUIRE(off + r.bytes <= MAPPED_BYTES, TSG_ERR_INTERNAL, "device read too large");
+        a.src[a.n] = static_cast<const uint8_t *>(r.dev);
+        a.bytes[a.n] = (uint32_t)r.bytes;
+        a.off[a.n] = off;
+        a.n++;
+        off += (uint32_t)((r.bytes + 15) & ~(size_t)15);
+    }
+    a.dst = mp.d;
+    TSG_LAUNCH(k_export, 1, 256, 0, s, a);
     const double t0 = now_ms();
     TSG_CUDA(cudaStreamSynchronize(s));
     t_host_sync_ms += now_ms() - t0;
+    int k = 0;
+    for (const DevRead &r : segs) {
+        memcpy(r.host, mp.h + a.off[k], r.bytes);
+        k++;
+    }
+}
+
+int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {
+    int64_t v = 0;
+    read_device({{&v, dptr, sizeof(v)}}, s);
     return v;
 }
 
@@ -357,12 +411,8 @@ tsg_status tsg_tiles_slice_rows(const tsg_tiles *T, int64_t b, int64_t e, void *
         TSG_REQUIRE(0 <= b && b <= e && e <= T->tm, TSG_ERR_INVALID_ARG, "tile row range out of bounds");
         cudaStream_t s = (cudaStream_t)stream;
         int64_t t0 = 0, t1 = 0, z0 = 0, z1 = 0;
-        TSG_CUDA(cudaMemcpyAsync(&t0, T->tile_ptr + b, 8, cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaMemcpyAsync(&t1, T->tile_ptr + e, 8, cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaStreamSynchronize(s));
-        TSG_CUDA(cudaMemcpyAsync(&z0, T->tile_nnz + t0, 8, cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaMemcpyAsync(&z1, T->tile_nnz + t1, 8, cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaStreamSynchronize(s));
+        read_device({{&t0, T->tile_ptr + b, 8}, {&t1, T->tile_ptr + e, 8}}, s);
+        read_device({{&z0, T->tile_nnz + t0, 8}, {&z1, T->tile_nnz + t1, 8}}, s);
         Allocator A;  // default pool for the two rebased offset arrays
         Buffers buf(A, s);
         int64_t *tp = buf.get<int64_t>(e - b + 1);

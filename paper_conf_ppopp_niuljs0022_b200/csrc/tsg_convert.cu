@@ -191,8 +191,7 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
         TSG_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), s));
         TSG_LAUNCH(k_validate_csr, grid_for(m, 256), 256, 0, s, m, n, rp, ci, bad);
         int hbad = 0;
-        TSG_CUDA(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaStreamSynchronize(s));
+        read_device({{&hbad, bad, sizeof(int)}}, s);
         TSG_REQUIRE(!hbad, TSG_ERR_UNSORTED, "CSR input has unsorted, duplicate or out-of-range columns");
     }
     int64_t *tile_ptr = out.get<int64_t>(tm + 1);

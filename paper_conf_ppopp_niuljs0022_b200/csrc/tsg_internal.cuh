@@ -2,6 +2,8 @@
 // Nothing here is visible through the C ABI (include/tsg.h).
 #pragma once
 
+#include <initializer_list>
+
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -208,6 +210,14 @@ void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buff
 
 // read one int64 from device memory (blocking on stream s)
 int64_t read_scalar(const int64_t *dptr, cudaStream_t s);
+// blocking read of up to 4 small device ranges (<= 4 KB in total) into host memory, through a
+// kernel writing mapped pinned memory (no D2H copy-engine traffic); counts into t_host_sync_ms
+struct DevRead {
+    void *host;
+    const void *dev;
+    size_t bytes;
+};
+void read_device(std::initializer_list<DevRead> segs, cudaStream_t s);
 
 // per-call launch counter (thread-local)
 void reset_call_launches();

@@ -170,13 +170,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     // sync #0: candidate total and row classes
     DevCounters hc{};
     int64_t Utot = 0;
-    TSG_CUDA(cudaMemcpyAsync(&Utot, costOff + ntA, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    TSG_CUDA(cudaMemcpyAsync(&hc, cnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-    {
-        const double t0 = now_ms();
-        TSG_CUDA(cudaStreamSynchronize(s));
-        t_host_sync_ms += now_ms() - t0;
-    }
+    read_device({{&Utot, costOff + ntA, sizeof(int64_t)}, {&hc, cnt, sizeof(DevCounters)}}, s);
     syncs++;
     TSG_REQUIRE(Utot < ((int64_t)1 << 40), TSG_ERR_OVERFLOW, "too many step-1 candidates");
 
@@ -308,13 +302,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     }
     int64_t nnzC = 0;
     DevCounters hc2{};
-    TSG_CUDA(cudaMemcpyAsync(&nnzC, tile_nnz + ntC, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    TSG_CUDA(cudaMemcpyAsync(&hc2, cnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-    {
-        const double t0 = now_ms();
-        TSG_CUDA(cudaStreamSynchronize(s));
-        t_host_sync_ms += now_ms() - t0;
-    }
+    read_device({{&nnzC, tile_nnz + ntC, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
     syncs++;
     uint8_t *idx = out.get<uint8_t>(nnzC);
     void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
@@ -355,8 +343,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     C->al = al;
     if (st) {
         DevCounters fin{};
-        TSG_CUDA(cudaMemcpyAsync(&fin, cnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-        TSG_CUDA(cudaStreamSynchronize(s));
+        read_device({{&fin, cnt, sizeof(DevCounters)}}, s);
         memset(st, 0, sizeof(*st));
         st->products = (flags & TSG_STATS_PRODUCTS) ? (int64_t)fin.products : -1;
         st->tiles_structural = -1;
