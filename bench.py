@@ -130,7 +130,33 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str 
     el = time.perf_counter() - t0
     return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
-                      f"(oracle/tsg_oracle.c), {el:.2f} s", "seconds": el, "products": int(prods)}
+                      f"(oracle/tsg_oracle.c), {el:.2f} s", "seconds": el, "products": int(prods),
+            "host_cores": os.cpu_count(), "_C": C}
+
+
+def sample_parity(tsg, T, Bt, C_ref, tol: float = 1e-12):
+    """The GPU result on the oracle's row sample (rows [0, R) of C = A*B, the tile rows covering them
+    multiplied by the same kernels): CSR structure bit for bit, values within tol * sum|a*b|."""
+    R = C_ref.m
+    tr = (R + 15) // 16
+    Ab = tsg.slice_rows(T, 0, tr) if tr != T.tile_m else T
+    Cg = tsg.spgemm(Ab, Bt)
+    rp, ci, v = (x.cpu().numpy() for x in tsg.tiles_to_csr(Cg))
+    del Cg, Ab
+    rp = rp[:R + 1]
+    nz = int(rp[-1])
+    structure_ok = bool(np.array_equal(rp, C_ref.rowptr) and np.array_equal(ci[:nz], C_ref.col))
+    err = None
+    ok = False
+    if structure_ok:
+        d = np.abs(v[:nz].astype(np.float64) - C_ref.val.astype(np.float64))
+        bound = tol * C_ref.abs
+        ok = bool(np.all(d <= bound))
+        err = float(np.max(d / np.where(C_ref.abs > 0, C_ref.abs, 1.0))) if nz else 0.0
+    return {"rows": int(R), "nnz": nz, "structure_ok": structure_ok, "max_rel_err": err,
+            "within_tolerance": ok,
+            "tolerance": f"|c - c_ref| <= {tol:g} * sum|a*b| per entry" +
+                         (" (north_star)" if tol <= 1e-12 else " (fp32 accumulation, reading D1)")}
 
 
 def gen_row_block(A, R):
@@ -492,10 +518,14 @@ def main():
             dist.destroy_process_group()
         return 0
     cpu = None
+    parity = None
     if not args.no_cpu_baseline and not args.profile and world == 1:
         cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr, prec="f64" if args.dtype == "f64" else "f32")
         cpu.pop("seconds", None)
         cpu.pop("products", None)
+        C_ref = cpu.pop("_C")
+        parity = sample_parity(tsg, T, Bt, C_ref, tol=1e-12 if args.dtype == "f64" else 1e-5)
+        del C_ref
     clocks = clk.summary() if not args.profile else None
     line = {
         "metric": _metric(args), "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -516,6 +546,7 @@ def main():
                    "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw},
         "roofline": roof,
         "cpu_baseline": cpu,
+        "parity": parity,
         "e2e": e2e,
         "gpu_launches": int(launches),
         "multi_gpu": multi,
