@@ -17,7 +17,7 @@ $(PKG)/libtsg.so: $(OBJ)
 	$(NVCC) $(ARCH) -shared -o $@ $(OBJ) -lcudart
 
 oracle/liboracle.so: oracle/tsg_oracle.c
-	gcc -O2 -ffp-contract=off -fPIC -shared -std=c11 -o $@ $< -lm
+	gcc -O2 -ffp-contract=off -fPIC -shared -std=c11 -fopenmp -o $@ $< -lm
 
 ptxas: EXTRA = -Xptxas -v
 ptxas: clean all

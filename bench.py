@@ -106,7 +106,7 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str = "f64"):
+def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str = "f64", with_omp: bool = False):
     """The oracle as it stands (single thread) on a bounded row sample of A*B (B = A by default)."""
     import oracle
 
@@ -128,7 +128,14 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str 
     t0 = time.perf_counter()
     C = oracle.spgemm(A, B, rows=rows, prec=prec)
     el = time.perf_counter() - t0
-    return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+    omp = None
+    if with_omp and prec == "f64":  # SURVEY 8(d) oracle_omp: the same code over row chunks, all host cores
+        nt = os.cpu_count() or 1
+        t0 = time.perf_counter()
+        oracle.spgemm(A, B, rows=rows, prec=prec, threads=nt)
+        eo = time.perf_counter() - t0
+        omp = {"value": 2.0 * prods / eo / 1e9, "unit": UNIT, "threads": nt, "seconds": round(eo, 3)}
+    return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle", "oracle_omp": omp,
             "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
                       f"(oracle/tsg_oracle.c), {el:.2f} s", "seconds": el, "products": int(prods),
             "host_cores": os.cpu_count(), "_C": C}
@@ -520,7 +527,8 @@ def main():
     cpu = None
     parity = None
     if not args.no_cpu_baseline and not args.profile and world == 1:
-        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr, prec="f64" if args.dtype == "f64" else "f32")
+        cpu = oracle_baseline(A, budget_s=args.cpu_budget_s, B=Bcsr, prec="f64" if args.dtype == "f64" else "f32",
+                              with_omp=True)
         cpu.pop("seconds", None)
         cpu.pop("products", None)
         C_ref = cpu.pop("_C")

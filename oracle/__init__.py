@@ -31,7 +31,7 @@ def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (plain C, no fused multiply-add contraction)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-std=c11",
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-std=c11", "-fopenmp",
                                "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
@@ -56,6 +56,10 @@ def lib():
         L.orc_gustavson_rowcounts.argtypes = [i64, i64, _i64p, _i32p, _i64p, _i32p, C.c_void_p, i64, _i64p]
         L.orc_gustavson.argtypes = [i64, i64, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p, C.c_void_p, i64,
                                     _i64p, _i32p, _f64p, C.c_void_p, C.c_int]
+        L.orc_gustavson_rowcounts_omp.argtypes = [i64, i64, _i64p, _i32p, _i64p, _i32p, C.c_void_p, i64, _i64p,
+                                                  C.c_int]
+        L.orc_gustavson_omp.argtypes = [i64, i64, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p, C.c_void_p, i64,
+                                        _i64p, _i32p, _f64p, C.c_void_p, C.c_int, C.c_int]
         L.orc_gustavson_f32.argtypes = [i64, i64, _i64p, _i32p, _f32p, _i64p, _i32p, _f32p, C.c_void_p, i64,
                                          _i64p, _i32p, _f32p, C.c_void_p, C.c_int]
         L.orc_csr_to_tiles_count.argtypes = [i64, i64, _i64p, _i32p, _i64p]
@@ -161,11 +165,13 @@ def transpose(A) -> OracleCSR:
     return OracleCSR(A.n, A.m, rpT, colT, valT)
 
 
-def spgemm(A, B, fma: bool = False, rows=None, prec: str = "f64") -> OracleCSR:
+def spgemm(A, B, fma: bool = False, rows=None, prec: str = "f64", threads: int = 1) -> OracleCSR:
     """O1: C = A*B by Gustavson's row-row Algorithm 1.  ``rows`` selects a subset.
 
     prec="f32": the same loop in single precision (f3); values are taken as float32
-    (a float16 input is widened exactly), the result's val is float32, abs stays fp64."""
+    (a float16 input is widened exactly), the result's val is float32, abs stays fp64.
+    threads > 1 (fp64): the row list split over OpenMP threads, each chunk by the same C loop
+    (the oracle_omp baseline of SURVEY 8(d); bit-for-bit the single-threaded result)."""
     if A.n != B.m:
         raise ValueError("shape mismatch")
     if prec not in ("f64", "f32"):
@@ -179,17 +185,29 @@ def spgemm(A, B, fma: bool = False, rows=None, prec: str = "f64") -> OracleCSR:
     else:
         rows = _arr(rows, np.int64)
         R, rp_ptr, nrows = rows.size, rows.ctypes.data_as(C.c_void_p), rows.size
+    omp = threads > 1 and prec == "f64"
+    if omp and rows is None:  # the OpenMP driver splits an explicit row list
+        rows = np.arange(A.m, dtype=np.int64)
+        R, rp_ptr, nrows = rows.size, rows.ctypes.data_as(C.c_void_p), rows.size
     rowlen = np.zeros(max(R, 1), dtype=np.int64)
-    _chk(L.orc_gustavson_rowcounts(A.m, B.n, Arp, Aci, Brp, Bci, rp_ptr, nrows, rowlen), "rowcounts")
+    if omp:
+        _chk(L.orc_gustavson_rowcounts_omp(A.m, B.n, Arp, Aci, Brp, Bci, rp_ptr, nrows, rowlen, int(threads)),
+             "rowcounts")
+    else:
+        _chk(L.orc_gustavson_rowcounts(A.m, B.n, Arp, Aci, Brp, Bci, rp_ptr, nrows, rowlen), "rowcounts")
     rp = np.zeros(R + 1, dtype=np.int64)
     np.cumsum(rowlen[:R], out=rp[1:])
     nnz = int(rp[-1])
     col = np.zeros(max(nnz, 1), dtype=np.int32)
     val = np.zeros(max(nnz, 1), dtype=vdt)
     ab = np.zeros(max(nnz, 1), dtype=np.float64)
-    f = L.orc_gustavson if prec == "f64" else L.orc_gustavson_f32
-    _chk(f(A.m, B.n, Arp, Aci, Av, Brp, Bci, Bv, rp_ptr, nrows, rp, col, val, ab.ctypes.data_as(C.c_void_p),
-           int(fma)), "gustavson")
+    if omp:
+        _chk(L.orc_gustavson_omp(A.m, B.n, Arp, Aci, Av, Brp, Bci, Bv, rp_ptr, nrows, rp, col, val,
+                                 ab.ctypes.data_as(C.c_void_p), int(fma), int(threads)), "gustavson")
+    else:
+        f = L.orc_gustavson if prec == "f64" else L.orc_gustavson_f32
+        _chk(f(A.m, B.n, Arp, Aci, Av, Brp, Bci, Bv, rp_ptr, nrows, rp, col, val, ab.ctypes.data_as(C.c_void_p),
+               int(fma)), "gustavson")
     return OracleCSR(R, B.n, rp, col[:nnz], val[:nnz], ab[:nnz])
 
 

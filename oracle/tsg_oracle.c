@@ -16,6 +16,7 @@
  *                           Section 3.3 step 1 (C' = A'B') and Algorithm 2
  *                           (set intersection + bit-mask OR)
  *   O5 orc_products         number of intermediate products (Table 2 caption)
+ *   -- orc_gustavson*_omp   O1 over contiguous row chunks on OpenMP threads (a baseline, same results)
  *   -- orc_spmv             y = A x, for the row-sum invariant C·1 = A·(B·1)
  *
  * Status codes: 0 ok, -1 bad argument, -2 out of memory, -3 inconsistent input.
@@ -135,6 +136,41 @@ int orc_gustavson(int64_t m, int64_t n, const int64_t *Arp, const int32_t *Aci, 
     }
     free(stamp); free(acc); free(acc_abs); free(list);
     return 0;
+}
+
+/* O1 on all host cores (the oracle_omp baseline).  The row sample is split into
+ * nthreads contiguous chunks and each chunk is computed by the unchanged single-threaded
+ * orc_gustavson_rowcounts / orc_gustavson above on its own OpenMP thread (private accumulators).
+ * The per-row arithmetic is identical, so the result equals the single-threaded one bit for bit
+ * (tests/test_oracle_pins.py).  `rows` must be given (the row ids of the sample). */
+int orc_gustavson_rowcounts_omp(int64_t m, int64_t n, const int64_t *Arp, const int32_t *Aci,
+                                const int64_t *Brp, const int32_t *Bci, const int64_t *rows,
+                                int64_t nrows, int64_t *rowlen, int nthreads) {
+    if (!rows || nthreads < 1) return -1;
+    int rc = 0;
+#pragma omp parallel for num_threads(nthreads) schedule(static) reduction(min : rc)
+    for (int c = 0; c < nthreads; c++) {
+        const int64_t r0 = nrows * c / nthreads, r1 = nrows * (c + 1) / nthreads;
+        const int e = orc_gustavson_rowcounts(m, n, Arp, Aci, Brp, Bci, rows + r0, r1 - r0, rowlen + r0);
+        if (e < rc) rc = e;
+    }
+    return rc;
+}
+
+int orc_gustavson_omp(int64_t m, int64_t n, const int64_t *Arp, const int32_t *Aci, const double *Aval,
+                      const int64_t *Brp, const int32_t *Bci, const double *Bval, const int64_t *rows,
+                      int64_t nrows, const int64_t *Crp, int32_t *Cci, double *Cval, double *Cabs,
+                      int fma_mode, int nthreads) {
+    if (!rows || nthreads < 1) return -1;
+    int rc = 0;
+#pragma omp parallel for num_threads(nthreads) schedule(static) reduction(min : rc)
+    for (int c = 0; c < nthreads; c++) {
+        const int64_t r0 = nrows * c / nthreads, r1 = nrows * (c + 1) / nthreads;
+        const int e = orc_gustavson(m, n, Arp, Aci, Aval, Brp, Bci, Bval, rows + r0, r1 - r0, Crp + r0, Cci, Cval,
+                                    Cabs, fma_mode);
+        if (e < rc) rc = e;
+    }
+    return rc;
 }
 
 /* O1 in single precision (the paper's Section 4.7 setup computes with half

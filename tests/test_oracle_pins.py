@@ -447,3 +447,19 @@ def test_gustavson_f32_accumulates_in_single_precision():
     for fma in (False, True):
         assert oracle.spgemm(A, B, fma=fma, prec="f32").val.tolist() == [1.0]
         assert oracle.spgemm(A, B, fma=fma).val.tolist() == [1.0 + 2.0 ** -23]
+
+
+def test_oracle_omp_equals_single_thread():
+    """oracle_omp: the row list split over OpenMP threads, each chunk by the same C
+    loop, gives the single-threaded result bit for bit -- including more threads than rows."""
+    for A, rows in ((gen.config("C1"), np.arange(4096, dtype=np.int64)),
+                    (gen.rmat(9), np.arange(0, 512, 3, dtype=np.int64)),
+                    (gen.config("C1"), np.arange(5, dtype=np.int64))):
+        ref = oracle.spgemm(A, A, rows=rows)
+        for th in (2, 3, 8):
+            got = oracle.spgemm(A, A, rows=rows, threads=th)
+            assert np.array_equal(got.rowptr, ref.rowptr) and np.array_equal(got.col, ref.col)
+            assert np.array_equal(got.val.view(np.int64), ref.val.view(np.int64))
+            assert np.array_equal(got.abs, ref.abs)
+    full = oracle.spgemm(gen.config("C1"), gen.config("C1"), threads=4)
+    assert full.nnz == 51972  # the C1 closed form (SURVEY 8(c))
