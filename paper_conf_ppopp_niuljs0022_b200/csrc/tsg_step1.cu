@@ -439,23 +439,31 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
         // for the owner) and keeps, in order, those with a product (reading B3): tile column +
         // work in the top bits, and the candidate's index k (16 bits; the B tile position is
         // st + k, or list[st + k] in list mode).  Four candidates per lane in flight.
-        int64_t cntv = 0;
+        // (32-bit indices: the row's candidates fit the stage, B tile positions fit 31 bits)
+        const int ioff = (int)off, ilen = (int)len;
+        const uint32_t st32 = (uint32_t)st;
+        const uint32_t *lst = isl ? P.list + st : nullptr;
+        uint32_t *sJw = &sJ[w][ioff];
+        uint16_t *sKw = &sK[w][ioff];
+        int cntv = 0;
 #pragma unroll 4
-        for (int64_t k = 0; k < len; k++) {
-            const uint32_t pos = isl ? P.list[st + k] : (uint32_t)(st + k);
+        for (int k = 0; k < ilen; k++) {
+            const uint32_t pos = isl ? lst[k] : st32 + (uint32_t)k;
             const uint32_t wk = isl ? 1u : (uint32_t)__popc(co & (uint32_t)P.rowOccB[pos]);
             if (wk) {
-                sJ[w][off + cntv] = (uint32_t)P.tcB[pos] | (wk << 27);
-                sK[w][off + cntv] = (uint16_t)k;
+                sJw[cntv] = (uint32_t)P.tcB[pos] | (wk << 27);
+                sKw[cntv] = (uint16_t)k;
                 cntv++;
             }
         }
         __syncwarp();
-        const int64_t vlen = cntv;
-        const uint32_t *mj = &sJ[w][off];
-        int64_t s = 0;
+        const int vlen = cntv;
+        const uint32_t *mj = sJw;
+        int s = 0;
         uint32_t hv = vlen > 0 ? mj[0] : INF;
         auto adv = [&]() { hv = s < vlen ? mj[s] : INF; };
+        uint64_t *pout = P.pairs + base;
+        const uint64_t thi = (uint64_t)t << 32;
         for (;;) {
             const uint32_t J = __reduce_min_sync(FULL, hv & JM);
             if (J == JM) break;  // every lane exhausted (INF & JM == JM > any tile column)
@@ -463,9 +471,9 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
             const unsigned hm = __ballot_sync(FULL, hit);
             const uint32_t ws = __reduce_add_sync(FULL, hit ? hv >> 27 : 0u);
             if (hit) {
-                const int64_t k = sK[w][off + s];
-                const uint32_t pos = isl ? P.list[st + k] : (uint32_t)(st + k);
-                P.pairs[base + out.np + __popc(hm & lt)] = ((uint64_t)t << 32) | pos;
+                const uint32_t k = sKw[s];
+                const uint32_t pos = isl ? lst[k] : st32 + k;
+                pout[out.np + (uint32_t)__popc(hm & lt)] = thi | pos;
             }
             out.emit(P, base, lane, J, hm, ws);
             if (hit) {
