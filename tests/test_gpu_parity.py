@@ -566,3 +566,24 @@ def test_copy_to_host_async_pipeline(tsg):
     assert np.array_equal(np.concatenate(masks), ref.mask)
     assert np.array_equal(np.concatenate(idxs), ref.idx)
     assert bitwise_equal_values(np.concatenate(vals), ref.val)
+
+
+@pytest.mark.parametrize("chunk", ["0", "1", "3"])
+def test_work_distribution_gives_identical_results(tsg, chunk, monkeypatch):
+    """Step-2/3 work distribution: static grid-stride (0) or the work queue with 1 or 3 groups per
+    request (TSG_QUEUE_CHUNK, read at launch; small test inputs otherwise take the static path)."""
+    cases = (gen.stencil27(12), gen.strip_fem(6, 20, 6), gen.rmat(11),
+             gen.hub(8192, hub_rows=(0, 5000), hub_cols=(), density=0.002))
+    base = []
+    for A in cases:
+        T = tiles_of(tsg, A)
+        base.append(host(tsg.spgemm(T, T)))
+    monkeypatch.setenv("TSG_QUEUE_CHUNK", chunk)
+    for A, b in zip(cases, base):
+        T = tiles_of(tsg, A)
+        got = host(tsg.spgemm(T, T))
+        for k in ARRAYS[:-1]:
+            assert np.array_equal(got[k], b[k]), (chunk, k)
+        assert bitwise_equal_values(got["val"], b["val"])
+    A = cases[0]
+    assert_tiles_equal(host(tsg.spgemm(tiles_of(tsg, A), tiles_of(tsg, A))), oracle.expected_tiles(A, A, fma=True))
