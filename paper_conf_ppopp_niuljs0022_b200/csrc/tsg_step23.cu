@@ -1003,8 +1003,10 @@ static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s)
         TSG_LAUNCH((k_s3<TI, TO>), sp.grid, T3, 0, s, Q);
     }
     if (n_dense > 0) {
-        // dense tiles per group of 32: spread a group over up to 8 warps when dense tiles are common
-        const int split = (int)std::max<int64_t>(1, std::min<int64_t>(8, 32 * n_dense / (groups * 4)));
+        // dense tiles per group of 32: spread a group over up to 4 warps when dense tiles are common
+        // (measured on C3: 2 / 4 / 8 / 16 / 32 warps -> 0.743 / 0.716 / 0.734 / 0.780 / 0.839 ms)
+        int split = (int)std::max<int64_t>(1, std::min<int64_t>(4, 32 * n_dense / (groups * 4)));
+        if (const char *e = getenv("TSG_DENSE_SPLIT")) split = std::max(1, std::min(32, atoi(e)));  // tuning only
         // (dense tiles: static distribution, measured faster on C3)
         const Shape sp = step_shape(k_s3_dense<TI, TO>, T3, groups * split, INT64_MAX);
         Q.qchunk[4] = sp.chunk;
