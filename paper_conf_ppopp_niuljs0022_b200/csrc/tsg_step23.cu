@@ -42,8 +42,17 @@ __device__ __forceinline__ double vfma(double a, double b, double c) { return fm
 __device__ __forceinline__ float vfma(float a, float b, float c) { return fmaf(a, b, c); }
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int T2 = 256;    // step-2 CTA
-constexpr int T3 = 128;    // step-3 CTA (4 warps; 5.5 KB of shared memory per warp)
+#ifndef TSG_T2
+#define TSG_T2 256
+#endif
+#ifndef TSG_T3
+#define TSG_T3 128
+#endif
+#ifndef TSG_TS
+#define TSG_TS 256
+#endif
+constexpr int T2 = TSG_T2;  // step-2 CTA
+constexpr int T3 = TSG_T3;  // step-3 CTA (4 warps; 7.7 KB of shared memory per warp)
 constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
 constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
 
@@ -316,7 +325,7 @@ __device__ __forceinline__ void cp_wait_all() {
 // popcount addressing.  The kernel is latency bound (dependent chains pair -> tile metadata ->
 // values), so it runs alone at full occupancy (no staging, few registers) and pipelines the
 // per-pair metadata one pair ahead.
-constexpr int TS = 256;  // small-class CTA
+constexpr int TS = TSG_TS;  // small-class CTA
 constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <= 16)
 
 // STAGE (hypersparse inputs, where B's tile metadata misses in cache): a lane-private double buffer
