@@ -551,7 +551,12 @@ def main():
                    "step_ms_all": [round(x, 3) for x in step_ms],
                    "host_sync_alloc_ms": [round(float(np.mean([h[0] for h in host_ms])), 3),
                                           round(float(np.mean([h[1] for h in host_ms])), 3)],
-                   "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw},
+                   "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw,
+                   # per-call counts of the last timed call(s) (tsg_stats; summed over row blocks)
+                   "call_stats": {k: stats_last.get(k) for k in
+                                  ("candidates", "pairs", "tiles_c", "tiles_dense", "step1_merge_rows",
+                                   "step1_list_tiles", "host_syncs", "kernel_launches", "bytes_scratch",
+                                   "bytes_out", "tiles_structural")}},
         "roofline": roof,
         "cpu_baseline": cpu,
         "parity": parity,
