@@ -419,7 +419,7 @@ def main():
             bsizes.append({k: (v.numel(), _host_dtype(v)) for k, v in Cx.arrays().items()})
             bo += sum(v.numel() * v.element_size() for v in Cx.arrays().values())
             del Cx, Ab
-        pipeline = bo <= E2E_PINNED_MAX
+        pipeline = 2 * bo <= E2E_PINNED_MAX  # two sets of pinned host buffers (consecutive steps)
         if pipeline:  # one pinned host destination per block, two sets (consecutive steps alternate)
             bufs2 = [[{k: torch.empty(n, dtype=dt, pin_memory=True) for k, (n, dt) in sz.items()} for sz in bsizes]
                      for _ in range(2)]
