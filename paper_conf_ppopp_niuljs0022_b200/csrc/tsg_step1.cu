@@ -406,7 +406,10 @@ struct MergeOut {
     }
 };
 
-constexpr int MERGE_W = 4;       // warps (tile rows) per merge CTA
+#ifndef TSG_MERGE_W
+#define TSG_MERGE_W 4
+#endif
+constexpr int MERGE_W = TSG_MERGE_W;  // warps (tile rows) per merge CTA
 constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (6 B each)
 
 __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
