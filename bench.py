@@ -138,7 +138,7 @@ def oracle_baseline(A, budget_s: float = 12.0, max_rows=None, B=None, prec: str 
     return {"value": 2.0 * prods / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle", "oracle_omp": omp,
             "sample": f"rows [0,{R}) of {m} ({prods} products, nnz {C.nnz}), single-threaded C Gustavson "
                       f"(oracle/tsg_oracle.c), {el:.2f} s", "seconds": el, "products": int(prods),
-            "host_cores": os.cpu_count(), "_C": C}
+            "host_cores": os.cpu_count(), "cpu_model": _cpu_model(), "_C": C}
 
 
 def sample_parity(tsg, T, Bt, C_ref, tol: float = 1e-12):
@@ -218,10 +218,9 @@ def main():
     ap.add_argument("--cpu-budget-s", type=float, default=12.0)
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/baseline/e2e)")
-    ap.add_argument("--step3-rows", action="store_true", help="step 3 in the whole-tile-row kernel (experimental)")
-    ap.add_argument("--dense-tc", action="store_true",
-                    help="fp64 dense tiles on the tensor cores (DMMA 8x8x4; TSG_DENSE_TC): values within the "
-                         "north_star tolerance instead of bitwise equal to the ascending-k FMA order")
+    ap.add_argument("--path", default="auto", choices=["auto", "rows", "tiles"],
+                    help="pipeline: the library's dispatch (auto), the fused per-tile-row path wherever every "
+                         "tile row is narrow (rows), or the per-C-tile path (tiles); same C either way")
     ap.add_argument("--aat", action="store_true",
                     help="C = A * A^T (the paper's second workload, SURVEY f1); A^T is formed once with "
                          "tsg_tiles_transpose outside the timed region, like the CSR->tile conversion")
@@ -281,34 +280,34 @@ def main():
     shards = [tsg.slice_rows(T, b0, b1) if (b0, b1) != (0, T.tile_m) else T for b0, b1 in blocks]
     Ashard = tsg.slice_rows(T, I0, I1) if (I0, I1) != (0, T.tile_m) else T
 
-    def run_blocks(timing=True, products=False, keep=False):
-        """One step: C = A_shard * A block by block; returns summed stats (and C if one block)."""
-        tot, last = {}, None
-        for Ab in shards:
-            C = tsg.spgemm(Ab, Bt, stats=True, timing=timing, products=products, step3_rows=args.step3_rows,
-                           dense_tc=args.dense_tc)
-            for k, v in C.stats.items():
-                tot[k] = tot.get(k, 0) + v
-            last = C if (keep and len(shards) == 1) else None
-            del C
-        return tot, last
+    popts = {"auto": {}, "rows": dict(path_rows=True), "tiles": dict(path_general=True)}[args.path]
 
-    # one instrumented call for the exact counts (products are a property of the input)
-    st0, _ = run_blocks(timing=False, products=True)
+    def run_blocks(stats=False, timing=False, products=False):
+        """One step: C = A_shard * B block by block (the production call: no stats unless asked);
+        returns the summed stats of the blocks (None without stats)."""
+        tot = None
+        for Ab in shards:
+            C = tsg.spgemm(Ab, Bt, stats=stats or timing or products, timing=timing, products=products,
+                           structural=products, **popts)
+            if C.stats is not None:
+                tot = tot or {}
+                for k, v in C.stats.items():
+                    tot[k] = tot.get(k, 0) + v
+            del C
+        return tot
+
+    # one instrumented call for the exact counts (products and |C'| are properties of the input)
+    st0 = run_blocks(products=True)
     small_inputs = tile_bytes(T.tile_m, T.num_tiles, T.nnz) < 2 * L2_BYTES
     flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev) if small_inputs else None
 
-    def one_step(timing=True):
-        return run_blocks(timing=timing)[0]
-
     for _ in range(args.warmup):
-        one_step()
+        run_blocks()
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
     launches0 = tsg.kernel_launch_count()
-    step_ms, s3_ms, s2_ms, s1_ms, sa_ms, host_ms = [], [], [], [], [], []
-    stats_last = None
+    step_ms = []
     with ClockSampler(local) if not args.profile else _Null() as clk:
         torch.cuda.synchronize()
         if dist:
@@ -318,21 +317,29 @@ def main():
                 flush.fill_(1)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            st = one_step()
+            run_blocks()  # the production call: no stats, no per-step events
             e1.record(stream)
             e1.synchronize()
             step_ms.append(e0.elapsed_time(e1))
-            s1_ms.append(st["ms_step1"] + st["ms_index"])
-            s2_ms.append(st["ms_step2"])
-            s3_ms.append(st["ms_step3"])
-            sa_ms.append(st["ms_alloc"])
-            host_ms.append((st["ms_host_sync"], st["ms_host_alloc"]))
-            stats_last = st
         torch.cuda.synchronize()
         if dist:
             dist.barrier()
     launches = tsg.kernel_launch_count() - launches0
-    local_ms = float(np.mean(step_ms))
+    # per-step times (library-recorded CUDA events on the launching stream) from instrumented calls
+    # after the timed loop, medians
+    s1_ms, s2_ms, s3_ms, sa_ms, host_ms = [], [], [], [], []
+    stats_last = None
+    for _ in range(max(3, min(args.steps, 10))):
+        if flush is not None:
+            flush.fill_(1)
+        st = run_blocks(timing=True)
+        s1_ms.append(st["ms_step1"] + st["ms_index"])
+        s2_ms.append(st["ms_step2"])
+        s3_ms.append(st["ms_step3"])
+        sa_ms.append(st["ms_alloc"])
+        host_ms.append((st["ms_host_sync"], st["ms_host_alloc"]))
+        stats_last = st
+    local_ms = float(np.median(step_ms))
     ms = local_ms
     prods_local = st0["products"]
     prods = prods_local
@@ -380,8 +387,8 @@ def main():
     # roofline of the dominant kernel (step 3 numeric unless another step is longer)
     bw, bw_src = peaks()
     nnzC, ntC = stats_last["nnz_c"], stats_last["tiles_c"]
-    steps_ms = {"step1": float(np.mean(s1_ms)), "step2": float(np.mean(s2_ms)), "step3": float(np.mean(s3_ms))}
-    alloc_ms = float(np.mean(sa_ms))
+    steps_ms = {"step1": float(np.median(s1_ms)), "step2": float(np.median(s2_ms)), "step3": float(np.median(s3_ms))}
+    alloc_ms = float(np.median(sa_ms))
     alg = {  # algorithmic bytes per launch of each step's kernels
         # (B is read once per row block; value bytes vb for A and B, cb for C)
         "step1": 4 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1) + K * (6 * Bt.num_tiles + 8 * (Bt.tile_m + 1)) + 12 * ntC,
@@ -389,10 +396,13 @@ def main():
         "step3": (1 + vb) * (Ashard.nnz + K * Bt.nnz) + (1 + cb) * nnzC + 48 * (Ashard.num_tiles + K * Bt.num_tiles)
                  + 56 * ntC,
     }
+    if int(stats_last["path"]) == len(shards):  # the row path: "step2" is the fused step-1 merge + step-2 masks
+        alg["step2"] += alg["step1"]
+        alg["step1"] = 12 * Ashard.num_tiles + 8 * (Ashard.tile_m + 1)  # the plan: tile columns, costs, offsets
     dom = max(steps_ms, key=steps_ms.get)
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
     traffic = None
-    tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    tp = os.path.join(ROOT, "profiles", f"traffic_r02_{args.config}.json")
     if os.path.exists(tp) and world == 1 and K == 1 and args.dtype == "f64" and not args.aat:
         traffic = json.load(open(tp)).get(dom)  # captured for the whole single-GPU fp64 call only
     bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz, vb) + \
@@ -440,7 +450,7 @@ def main():
             live = []
             for i, (b0, b1) in enumerate(eblocks):
                 Ah = tsg.slice_rows(Th, b0, b1) if (b0, b1) != (0, Th.tile_m) else Th
-                Cx = tsg.spgemm(Ah, Bh, dense_tc=args.dense_tc)
+                Cx = tsg.spgemm(Ah, Bh, **popts)
                 if pipeline:
                     done = torch.cuda.Event()
                     done.record(stream)
@@ -475,7 +485,7 @@ def main():
                 keep = [Th, Bh]
                 for i, (b0, b1) in enumerate(eblocks):
                     Ah = tsg.slice_rows(Th, b0, b1) if (b0, b1) != (0, Th.tile_m) else Th
-                    Cx = tsg.spgemm(Ah, Bh, dense_tc=args.dense_tc)
+                    Cx = tsg.spgemm(Ah, Bh, **popts)
                     ev = torch.cuda.Event()
                     ev.record(stream)
                     s_copy.wait_event(ev)
@@ -547,16 +557,23 @@ def main():
                                   (f", {K} tile-row blocks per rank computed in turn" if K > 1 else ""),
                    "l2": ("512 MB flush between timed steps" if flush is not None else
                           f"inputs larger than L2 (A tiles {tile_bytes(T.tile_m, T.num_tiles, T.nnz) / 1e6:.0f} MB > 126 MB)"),
+                   "timing": "ms_per_step = median of the timed steps (CUDA events around the production "
+                             "tsg_spgemm call, no stats); step_ms = medians of separate instrumented calls",
+                   "t_ms_median": round(float(np.median(step_ms)), 4), "t_ms_mean": round(float(np.mean(step_ms)), 4),
                    "step_ms": {k: round(v, 4) for k, v in steps_ms.items()}, "alloc_sync_ms": round(alloc_ms, 4),
                    "step_ms_all": [round(x, 3) for x in step_ms],
+                   "path": {0: "per-C-tile pipeline", 1: "fused per-tile-row pipeline"}.get(
+                       int(stats_last["path"]) if K == 1 else -1, "mixed (row blocks)"),
+                   "step1_mode": _step1_mode(stats_last),
+                   "tiles_structural": int(st0["tiles_structural"]) if st0["tiles_structural"] >= 0 else None,
                    "host_sync_alloc_ms": [round(float(np.mean([h[0] for h in host_ms])), 3),
                                           round(float(np.mean([h[1] for h in host_ms])), 3)],
                    "bytes_alg": bytes_alg, "hbm_frac_path": bytes_alg / (ms / 1e3) / 1e9 / bw,
                    # per-call counts of the last timed call(s) (tsg_stats; summed over row blocks)
                    "call_stats": {k: stats_last.get(k) for k in
                                   ("candidates", "pairs", "tiles_c", "tiles_dense", "step1_merge_rows",
-                                   "step1_list_tiles", "host_syncs", "kernel_launches", "bytes_scratch",
-                                   "bytes_out", "tiles_structural")}},
+                                   "step1_big_rows", "step1_list_tiles", "host_syncs", "kernel_launches",
+                                   "bytes_scratch", "bytes_out")}},
         "roofline": roof,
         "cpu_baseline": cpu,
         "parity": parity,
@@ -569,6 +586,29 @@ def main():
     if dist:
         dist.destroy_process_group()
     return 0
+
+
+def _step1_mode(st):
+    """Step-1 formulation used (tsg_stats): warp merge of <= 32 sorted candidate lists per tile row,
+    and/or bitmap rank / sort for wide rows; A tiles expanded through B row lists (mode ii)."""
+    parts = []
+    if st.get("step1_merge_rows"):
+        parts.append(f"warp merge ({int(st['step1_merge_rows'])} tile rows)")
+    if st.get("step1_big_rows"):
+        parts.append(f"global-memory rank/sort ({int(st['step1_big_rows'])} tile rows)")
+    if st.get("step1_list_tiles"):
+        parts.append(f"B-row lists for {int(st['step1_list_tiles'])} A tiles")
+    return "; ".join(parts) or "shared-memory sort"
+
+
+def _cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def _metric(args):

@@ -45,7 +45,7 @@ extern "C" {
 #define TSG_TILE 16          /* tile size, fixed by the paper */
 #define TSG_DENSE_NNZ 96     /* t_nnz: dense accumulator iff tile nnz >= 96 (the paper's 192, re-tuned
                                 for these kernels on B200: reading A7) */
-#define TSG_ABI_VERSION 2
+#define TSG_ABI_VERSION 3
 
 typedef enum {
     TSG_OK = 0,
@@ -95,11 +95,14 @@ typedef struct {
     int32_t dtype;            /* tsg_dtype of val */
 } tsg_tiles_view;
 
-/* Per-call statistics of tsg_spgemm (all counts exact; times only with TSG_STATS_TIMING). */
+/* Per-call statistics of tsg_spgemm (all counts exact; times only with TSG_STATS_TIMING).
+ * Filling the counts costs one extra blocking read at the end of the call; pass NULL in timed
+ * production calls. */
 typedef struct {
     int64_t products;         /* sum_i sum_{k in A(i,:)} nnz(B(k,:)) (Table 2 caption P:2531-2538);
                                  -1 unless TSG_STATS_PRODUCTS */
-    int64_t tiles_structural; /* |C'| of the paper's step 1; -1 unless TSG_STATS_STRUCTURAL */
+    int64_t tiles_structural; /* |C'| = tiles of the structural tile product A'B' of the paper's step 1, empty
+                                 tiles included; -1 unless TSG_STATS_STRUCTURAL */
     int64_t tiles_c;          /* non-empty C tiles (= C.num_tiles) */
     int64_t nnz_c;
     int64_t candidates;       /* tile-pair candidates examined by step 1 */
@@ -108,33 +111,46 @@ typedef struct {
     int64_t tiles_sparse;
     int64_t kernel_launches;  /* kernels this call launched */
     int32_t step1_list_tiles; /* A tiles that used the B-row-list expansion (mode ii) */
-    int32_t host_syncs;       /* blocking device->host scalar reads performed */
-    float ms_index, ms_step1, ms_step2, ms_alloc, ms_step3, ms_total; /* CUDA-event times */
+    int32_t host_syncs;       /* blocking device->host scalar reads performed (the stats read excluded) */
+    float ms_index, ms_step1, ms_step2, ms_alloc, ms_step3, ms_total; /* CUDA-event times; on the row path
+                                 ms_step1 is the plan and ms_step2 the fused step-1 merge + step-2 masks */
     float ms_host_sync, ms_host_alloc; /* host wall time blocked in scalar reads / allocation calls */
-    int64_t step3_row_tiles;  /* C tiles whose step 3 ran in the whole-tile-row kernel */
-    int64_t step3_rows;       /* tile rows handled by that kernel */
+    int64_t path;             /* TSG_PATH_ROWS (1): fused per-tile-row kernels (every tile row narrow, and the
+                                 call small or A's tiles dense, or TSG_PATH_ROWS_FORCE); TSG_PATH_TILES (0):
+                                 the per-C-tile pipeline */
+    int64_t step1_big_rows;   /* tile rows whose step 1 ran in global memory (bitmap rank / radix sort) */
     int64_t step1_merge_rows; /* tile rows whose step 1 ran as a warp k-way merge (<= 32 A tiles) */
     int64_t bytes_scratch;    /* device scratch of the call (its peak; f4, cf. Fig 9 peak space P:2938-2968) */
     int64_t bytes_out;        /* device bytes of C's seven arrays (allocation sizes; Fig 11) */
 } tsg_stats;
 
+#define TSG_PATH_TILES 0
+#define TSG_PATH_ROWS 1
+
 /* flags for tsg_csr_to_tiles */
 #define TSG_INPUT_HOST 0x1u     /* row_ptr/col_idx/val are host memory; copied in on `stream` */
-#define TSG_VALIDATE 0x2u       /* check sorted/unique/in-range columns (TSG_ERR_UNSORTED) */
+#define TSG_VALIDATE 0x2u       /* check row_ptr against nnz (INVALID_ARG) and sorted/unique/in-range columns
+                                   (UNSORTED); without it the input is trusted */
 
-/* flags for tsg_spgemm */
-#define TSG_STATS_TIMING 0x1u     /* record per-step CUDA events (one extra sync at the end) */
-#define TSG_STATS_STRUCTURAL 0x2u /* also compute |C'| (diagnostic; extra pass) */
+/* flags for tsg_spgemm.  None of them changes the result: every combination returns the same C
+ * bit for bit (they select work splits, diagnostics and timing only). */
+#define TSG_STATS_TIMING 0x1u     /* record per-step CUDA events (read with the stats at the end) */
+#define TSG_STATS_STRUCTURAL 0x2u /* also count |C'| into stats->tiles_structural (diagnostic pass over the
+                                     structural tile product; tile columns of B <= 1.6e6) */
 #define TSG_STEP1_SCAN_ONLY 0x4u  /* force mode (i) tile-row scans in step 1 */
 #define TSG_STEP1_LIST_ALWAYS 0x8u/* build B-row lists and use them wherever they are cheaper */
 #define TSG_STATS_PRODUCTS 0x10u  /* also count intermediate products into stats->products */
-#define TSG_STEP3_ROWS 0x20u      /* step 3 in the whole-tile-row kernel where rows fit (experimental; same results) */
-#define TSG_STEP1_SORT_ONLY 0x40u /* step 1: no warp merge; every tile row expands + radix-sorts (same results) */
-#define TSG_DENSE_TC 0x80u        /* step 3: fp64 dense tiles on the tensor cores (DMMA 8x8x4); values within the
-                                     tolerance of the ascending-k FMA result instead of equal to it bit for bit */
+#define TSG_PATH_GENERAL 0x20u    /* use the per-C-tile pipeline even when every tile row is narrow */
+#define TSG_STEP1_SORT_ONLY 0x40u /* step 1: no warp merge; every tile row expands + radix-sorts (implies
+                                     the per-C-tile pipeline) */
+#define TSG_PATH_ROWS_FORCE 0x400u /* take the row path whenever every tile row is narrow (by default only
+                                      for small calls or dense-tile-heavy A; TSG_PATH_GENERAL wins) */
 #define TSG_SMALL_STAGE_ON 0x100u  /* step 3 small tiles: stage B row metadata by cp.async (default: iff nnz(B) < 4 tiles(B)) */
 #define TSG_SMALL_STAGE_OFF 0x200u /* step 3 small tiles: plain dependent loads (same results either way) */
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = TSG_DENSE_NNZ; 257 disables dense) */
+#define TSG_QUEUE_CHUNK_SHIFT 25     /* bits 25..28: per-C-tile pipeline work distribution, v = 0: automatic,
+                                        v = 1: static grid-stride, v >= 2: work queue with v-1 groups per request */
+#define TSG_SPGEMM_FLAGS 0x1fff077fu /* every defined bit (anything else is INVALID_ARG) */
 
 /*
  * tsg_csr_to_tiles -- CSR -> sparse-tile format (Section 3.2; conversion is timed
@@ -173,7 +189,10 @@ TSG_API tsg_status tsg_csr_to_tiles_typed(int64_t m, int64_t n, int64_t nnz, con
  * fused multiply-add, i.e. ascending global k (reading A8/A16): deterministic run to run.
  * Value types: C's dtype follows tsg_dtype's rules (F16 inputs are widened exactly to fp32 and
  * accumulated with fp32 FMA); mixed input dtypes are INVALID_ARG.
- * Syncs: 3 blocking scalar reads (candidate total, C tile count, nnz(C)).
+ * Syncs: blocking scalar reads through mapped host memory -- 2 on the row path (the step-1 candidate
+ * total after the plan; C's tile count and nnz(C) together after the fused steps 1-2, the paper's single
+ * allocation point P:982-988), 3 on the per-C-tile path (candidate total, C tile count, nnz(C)); one more
+ * at the end when `stats` is non-NULL.
  * Alignment: mask and row_ptr of A and B must be 16-byte aligned, val 8-byte aligned (tiles are
  * staged into shared memory in 16-byte chunks); handles made by this library always are.
  * Errors: INVALID_ARG (incl. alignment), SHAPE, OVERFLOW, OOM, CUDA, INTERNAL.

@@ -55,15 +55,21 @@ def _stream_ptr(stream=None) -> int:
 
 
 class _Handle:
-    """Owns one tsg_tiles*; destroys it when the last reference (incl. tensor views) goes."""
+    """Owns one tsg_tiles*; destroys it when the last reference (incl. tensor views) goes.
 
-    def __init__(self, ptr: int):
+    The arrays are freed stream-ordered on the stream the handle was made on (``stream``, a
+    cudaStream_t as int), so a free never overtakes the kernels that wrote them; work on other
+    streams that reads them must be ordered before the last reference is dropped (as with
+    torch's caching allocator and ``record_stream``)."""
+
+    def __init__(self, ptr: int, stream: int = 0):
         self.ptr = ptr
+        self.stream = stream
 
     def __del__(self):
         if self.ptr:
             try:
-                _lib.load().tsg_tiles_destroy(C.c_void_p(self.ptr), None)
+                _lib.load().tsg_tiles_destroy(C.c_void_p(self.ptr), C.c_void_p(self.stream or None))
             except Exception:
                 pass
             self.ptr = 0
@@ -131,9 +137,9 @@ class Tiles:
         return out
 
 
-def _from_handle(ptr: int, stats=None) -> Tiles:
+def _from_handle(ptr: int, stats=None, stream: int = 0) -> Tiles:
     L = _lib.load()
-    h = _Handle(ptr)
+    h = _Handle(ptr, stream)
     v = _lib.TilesView()
     _lib.check(L.tsg_tiles_get_view(C.c_void_p(ptr), C.byref(v)))
     torch = _torch()
@@ -177,15 +183,25 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
         arrs = []
         vdt = str(val.dtype).replace("torch.", "") if isinstance(val, torch.Tensor) else np.asarray(val).dtype.name
         if vdt not in _DTYPE_CODE:
-            vdt = "float64"
-        for a, dt in ((row_ptr, np.int64), (col_idx, np.int32), (val, getattr(np, vdt))):
+            raise TypeError(f"unsupported value type {val.dtype} (float64, float32 or float16)")
+        for a, dt, tdt in ((row_ptr, np.int64, torch.int64), (col_idx, np.int32, torch.int32),
+                           (val, getattr(np, vdt), getattr(torch, vdt))):
             if isinstance(a, torch.Tensor):
+                if a.dtype != tdt:
+                    if tdt.is_floating_point or not a.dtype.is_floating_point:
+                        a = a.to(tdt)
+                    else:
+                        raise TypeError(f"expected an integer tensor, got {a.dtype}")
                 a = a.contiguous()
                 arrs.append((a, C.c_void_p(a.data_ptr() if a.numel() else 0)))
             else:
                 a = np.ascontiguousarray(a, dtype=dt)
                 arrs.append((a, C.c_void_p(a.ctypes.data if a.size else 0)))
+        if len(arrs[0][0]) != m + 1:
+            raise ValueError(f"row_ptr has {len(arrs[0][0])} entries, expected m + 1 = {m + 1}")
         nnz = int(arrs[0][0][-1]) if m >= 0 and len(arrs[0][0]) else 0
+        if len(arrs[1][0]) < nnz or len(arrs[2][0]) < nnz:
+            raise ValueError(f"row_ptr[m] = {nnz} exceeds the length of col_idx / val")
         rc = L.tsg_csr_to_tiles_typed(m, n, nnz, arrs[0][1], arrs[1][1], arrs[2][1], _DTYPE_CODE[vdt], flags,
                                       None, C.c_void_p(_stream_ptr(stream)), C.byref(out))
     else:
@@ -197,49 +213,65 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
                                       _dptr(val, val.dtype), _DTYPE_CODE[vdt], flags, None,
                                       C.c_void_p(_stream_ptr(stream)), C.byref(out))
     _lib.check(rc)
-    return _from_handle(out.value)
+    return _from_handle(out.value, stream=_stream_ptr(stream))
 
 
 def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, products: bool = False,
-           scan_only: bool = False, list_always: bool = False, dense_threshold: int | None = None,
-           step3_rows: bool = False, sort_only: bool = False, dense_tc: bool = False, small_stage: bool | None = None,
-           stream=None) -> Tiles:
-    """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3)."""
+           structural: bool = False, scan_only: bool = False, list_always: bool = False,
+           dense_threshold: int | None = None, sort_only: bool = False, path_general: bool = False,
+           path_rows: bool = False,
+           small_stage: bool | None = None, queue_chunk: int | None = None, stream=None) -> Tiles:
+    """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3).
+
+    stats / timing / products / structural: fill ``C.stats`` (one extra blocking read), with CUDA-
+    event step times, the intermediate-product count, |C'| of the paper's step 1.  The other
+    options select work splits only (the result is the same bit for bit): step-1 modes, the dense
+    threshold t_nnz, ``path_general`` (the per-C-tile pipeline even for narrow tile rows), ``path_rows``
+    (the fused per-tile-row pipeline wherever every tile row is narrow),
+    ``queue_chunk`` (per-C-tile work distribution: 0 static, k > 0 k groups per request)."""
     L = _lib.load()
     flags = 0
     if timing:
         flags |= _lib.STATS_TIMING
     if products:
         flags |= _lib.STATS_PRODUCTS
+    if structural:
+        flags |= _lib.STATS_STRUCTURAL
     if scan_only:
         flags |= _lib.STEP1_SCAN_ONLY
     if list_always:
         flags |= _lib.STEP1_LIST_ALWAYS
-    if step3_rows:
-        flags |= _lib.STEP3_ROWS
     if sort_only:
         flags |= _lib.STEP1_SORT_ONLY
-    if dense_tc:
-        flags |= _lib.DENSE_TC
+    if path_general:
+        flags |= _lib.PATH_GENERAL
+    if path_rows:
+        flags |= _lib.PATH_ROWS_FORCE
     if small_stage is not None:
         flags |= _lib.SMALL_STAGE_ON if small_stage else _lib.SMALL_STAGE_OFF
     if dense_threshold is not None:
         if not 1 <= dense_threshold <= 257:
             raise ValueError("dense_threshold must be in [1, 257]")
         flags |= dense_threshold << _lib.DENSE_THRESHOLD_SHIFT
-    st = _lib.Stats() if (stats or timing or products) else None
+    if queue_chunk is not None:
+        if not 0 <= queue_chunk <= 14:
+            raise ValueError("queue_chunk must be in [0, 14]")
+        flags |= (queue_chunk + 1) << _lib.QUEUE_CHUNK_SHIFT
+    st = _lib.Stats() if (stats or timing or products or structural) else None
     out = C.c_void_p()
-    rc = L.tsg_spgemm(A.ptr, B.ptr, flags, None, C.c_void_p(_stream_ptr(stream)), C.byref(out),
+    sp = _stream_ptr(stream)
+    rc = L.tsg_spgemm(A.ptr, B.ptr, flags, None, C.c_void_p(sp), C.byref(out),
                       C.byref(st) if st is not None else None)
     _lib.check(rc)
-    return _from_handle(out.value, st.as_dict() if st is not None else None)
+    return _from_handle(out.value, st.as_dict() if st is not None else None, stream=sp)
 
 
 def transpose(T: Tiles, stream=None) -> Tiles:
     """A^T in the sparse-tile format (tsg_tiles_transpose), e.g. for C = A * A^T."""
     out = C.c_void_p()
-    _lib.check(_lib.load().tsg_tiles_transpose(T.ptr, None, C.c_void_p(_stream_ptr(stream)), C.byref(out)))
-    return _from_handle(out.value)
+    sp = _stream_ptr(stream)
+    _lib.check(_lib.load().tsg_tiles_transpose(T.ptr, None, C.c_void_p(sp), C.byref(out)))
+    return _from_handle(out.value, stream=sp)
 
 
 def tiles_to_csr(T: Tiles, stream=None):
@@ -248,9 +280,10 @@ def tiles_to_csr(T: Tiles, stream=None):
     torch = _torch()
     rp, ci, v = C.c_void_p(), C.c_void_p(), C.c_void_p()
     nnz = C.c_int64()
-    _lib.check(L.tsg_tiles_to_csr(T.ptr, None, C.c_void_p(_stream_ptr(stream)), C.byref(rp), C.byref(ci),
+    sp = _stream_ptr(stream)
+    _lib.check(L.tsg_tiles_to_csr(T.ptr, None, C.c_void_p(sp), C.byref(rp), C.byref(ci),
                                   C.byref(v), C.byref(nnz)))
-    owner = _CsrOwner([rp.value, ci.value, v.value])
+    owner = _CsrOwner([rp.value, ci.value, v.value], sp)
 
     def t(p, count, dt):
         if count == 0:
@@ -261,15 +294,18 @@ def tiles_to_csr(T: Tiles, stream=None):
 
 
 class _CsrOwner:
-    def __init__(self, ptrs):
+    """Frees the arrays of tsg_tiles_to_csr on the stream that produced them (stream-ordered)."""
+
+    def __init__(self, ptrs, stream: int = 0):
         self.ptrs = ptrs
+        self.stream = stream
 
     def __del__(self):
         try:
             L = _lib.load()
             for p in self.ptrs:
                 if p:
-                    L.tsg_free(C.c_void_p(p), 0, None, None)
+                    L.tsg_free(C.c_void_p(p), 0, None, C.c_void_p(self.stream or None))
         except Exception:
             pass
 
@@ -277,9 +313,10 @@ class _CsrOwner:
 def slice_rows(T: Tiles, tile_row_begin: int, tile_row_end: int, stream=None) -> Tiles:
     """Zero-copy view of tile rows [begin, end) (tsg_tiles_slice_rows).  Keeps T alive."""
     out = C.c_void_p()
+    sp = _stream_ptr(stream)
     _lib.check(_lib.load().tsg_tiles_slice_rows(T.ptr, int(tile_row_begin), int(tile_row_end),
-                                                C.c_void_p(_stream_ptr(stream)), C.byref(out)))
-    V = _from_handle(out.value)
+                                                C.c_void_p(sp), C.byref(out)))
+    V = _from_handle(out.value, stream=sp)
     V.handle.parent = T.handle  # the view borrows T's arrays
     return V
 

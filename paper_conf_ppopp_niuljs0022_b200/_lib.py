@@ -23,12 +23,14 @@ STATS_STRUCTURAL = 0x2
 STEP1_SCAN_ONLY = 0x4
 STEP1_LIST_ALWAYS = 0x8
 STATS_PRODUCTS = 0x10
-STEP3_ROWS = 0x20
+PATH_GENERAL = 0x20
+PATH_ROWS_FORCE = 0x400
 STEP1_SORT_ONLY = 0x40
-DENSE_TC = 0x80
 SMALL_STAGE_ON = 0x100
 SMALL_STAGE_OFF = 0x200
 DENSE_THRESHOLD_SHIFT = 16
+QUEUE_CHUNK_SHIFT = 25
+PATH_TILES, PATH_ROWS = 0, 1  # tsg_stats.path
 
 STATUS = {0: "TSG_OK", 1: "TSG_ERR_INVALID_ARG", 2: "TSG_ERR_SHAPE", 3: "TSG_ERR_UNSORTED",
           4: "TSG_ERR_OVERFLOW", 5: "TSG_ERR_OOM", 6: "TSG_ERR_CUDA", 7: "TSG_ERR_INTERNAL"}
@@ -57,7 +59,7 @@ class Stats(C.Structure):
                 ("ms_index", C.c_float), ("ms_step1", C.c_float), ("ms_step2", C.c_float),
                 ("ms_alloc", C.c_float), ("ms_step3", C.c_float), ("ms_total", C.c_float),
                 ("ms_host_sync", C.c_float), ("ms_host_alloc", C.c_float),
-                ("step3_row_tiles", C.c_int64), ("step3_rows", C.c_int64),
+                ("path", C.c_int64), ("step1_big_rows", C.c_int64),
                 ("step1_merge_rows", C.c_int64), ("bytes_scratch", C.c_int64), ("bytes_out", C.c_int64)]
 
     def as_dict(self) -> dict:

@@ -35,20 +35,23 @@ __device__ __forceinline__ int half_excl_scan(int v, int r, int *total) {
     return incl - v;
 }
 
-__global__ void k_validate_csr(int64_t m, int64_t n, const int64_t *__restrict__ rp,
+// TSG_VALIDATE: *bad = 2 if row_ptr is inconsistent with nnz (row_ptr[0] != 0, decreasing, or
+// row_ptr[m] != nnz: the arrays are sized by nnz), else 1 for unsorted / duplicate / out-of-range
+// columns (reading A12)
+__global__ void k_validate_csr(int64_t m, int64_t n, int64_t nnz, const int64_t *__restrict__ rp,
                                const int32_t *__restrict__ ci, int *__restrict__ bad) {
     int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     int64_t b = rp[i], e = rp[i + 1];
-    if (b > e || (i == 0 && b != 0)) {
-        *bad = 1;
+    if (b > e || b < 0 || e > nnz || (i == 0 && b != 0) || (i == m - 1 && e != nnz)) {
+        atomicMax(bad, 2);
         return;
     }
     int64_t prev = -1;
     for (int64_t p = b; p < e; p++) {
         int64_t c = ci[p];
         if (c <= prev || c >= n) {
-            *bad = 1;
+            atomicMax(bad, 1);
             return;
         }
         prev = c;
@@ -189,9 +192,10 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
     if (validate && m > 0) {
         int *bad = tmp.get<int>(1);
         TSG_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), s));
-        TSG_LAUNCH(k_validate_csr, grid_for(m, 256), 256, 0, s, m, n, rp, ci, bad);
+        TSG_LAUNCH(k_validate_csr, grid_for(m, 256), 256, 0, s, m, n, nnz, rp, ci, bad);
         int hbad = 0;
         read_device({{&hbad, bad, sizeof(int)}}, s);
+        TSG_REQUIRE(hbad != 2, TSG_ERR_INVALID_ARG, "CSR row_ptr inconsistent with nnz (row_ptr[0] != 0, decreasing, or row_ptr[m] != nnz)");
         TSG_REQUIRE(!hbad, TSG_ERR_UNSORTED, "CSR input has unsorted, duplicate or out-of-range columns");
     }
     int64_t *tile_ptr = out.get<int64_t>(tm + 1);

@@ -21,11 +21,9 @@ struct DevCounters {
     u64c n3small;      // step-3 class sizes
     u64c n3medium;
     u64c n3dense;
-    u64c n3rows;       // tile rows handled by the row kernel of step 3
-    u64c n3fallback;   // C tiles left to the per-tile kernel of step 3
-    u64c next3;        // work counter of the step-3 row kernel
     u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
     u64c n2dense;      // C tiles with nnz >= t_nnz (step 2 counts them; step 3 launches the dense kernel iff > 0)
+    u64c structural;   // |C'| (TSG_STATS_STRUCTURAL)
     u64c q[5][16];     // work-queue counters of the step-2/3 kernels, one 128-byte line each
 };
 
@@ -34,6 +32,7 @@ constexpr int ROW_NW = ROW_T / 32;
 constexpr int ROW_CAP = 4096;     // max candidates of a row sorted in shared memory
 constexpr int LIGHT_WORK = 16;    // step-2 thread-per-tile class: (pair, c) items of the tile
 constexpr int SMALL_NNZ = 8;      // step-3 lane-per-entry class (k_s3_small): C tile nnz (<= 16)
+constexpr int64_t ROWPATH_SMALL_U = 1 << 20;  // step-1 candidates below which narrow calls take the row path
 constexpr int MERGE_MAX_A = 32;   // step-1 warp-merge class: A tiles of the tile row (one lane each)
 
 // ---------------- a1 row sort
@@ -62,6 +61,13 @@ struct S1Params {
     uint64_t *bigKeysA, *bigKeysB;
     uint32_t *bigPosB, *bigKpos;
     DevCounters *cnt;
+    // the row path's fused step 2 (k_sym_rows): masks and row offsets of each C tile at its
+    // candidate-space slot, tile nnz in tWork, the row's nnz total
+    const uint16_t *mA, *mB;
+    uint16_t *sMaskC;   // [16 Utot]
+    uint8_t *sRowPtrC;  // [16 Utot]
+    int64_t *rowNnz;    // [tm]
+    int dense_threshold;  // counts the dense C tiles into cnt->n2dense
 };
 
 // ---------------- compaction of step-1 results into per-C-tile arrays + step-2 classes
@@ -110,52 +116,14 @@ struct StepParams {
     void *vC;              // values: double for F64 inputs, float for F32 and F16 inputs
     int dtype_in;          // tsg_dtype of A and B
     const uint32_t *work;  // step-2 class split
-    const uint8_t *skip;   // step 3: per C tile, 1 = computed by the row kernel (nullptr: none)
     // step-3 classes per group of 32 C tiles (bit i = tile 32g+i), written by step 2: medium / dense
     // tiles among the light tiles (k_s2_light) and among the heavy tiles (k_s2)
     uint32_t *medL, *medH, *denL, *denH;
     int qchunk[5];         // work-queue units per request (k_s2_light, k_s2, k_s3_small, k_s3, k_s3_dense)
+    int qoverride;         // work distribution override (-1 automatic, 0 static, k > 0 queue chunk k)
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
-    int dense_tc;          // step 3: fp64 dense tiles on the tensor cores (DMMA), TSG_DENSE_TC
     int small_stage;       // step 3: k_s3_small stages B row metadata with cp.async (hypersparse B)
-    DevCounters *cnt;
-};
-
-// ---------------- a4 step 3, row kernel: one CTA per C tile row, tiles staged by TMA bulk copies
-constexpr int R3_T = 256;          // threads
-constexpr int R3_NTC = 128;        // max C tiles of a row
-constexpr int R3_NAC = 32;         // max A tiles of a row (one warp plans them)
-constexpr int R3_NPC = 2048;       // max pairs of a row
-constexpr int R3_ACC = 8192;       // max accumulator doubles of a row (compact + dense blocks)
-constexpr int R3_SMEM = 100 * 1024;  // dynamic shared memory per CTA
-
-struct RowParams {
-    int64_t tm;
-    const int64_t *tpA;
-    const int32_t *tcA;
-    const int64_t *tnzA;
-    const uint8_t *rpA;
-    const uint16_t *mA;
-    const uint16_t *colOccA;
-    const double *vA;
-    const int64_t *tpB;
-    const int64_t *tnzB;
-    const uint8_t *rpB;
-    const uint16_t *mB;
-    const double *vB;
-    const uint64_t *pairs;
-    const int64_t *pairBeg;
-    const uint32_t *pairCnt;
-    const int64_t *tpC;
-    const int64_t *tnzC;  // offsets (ntC + 1)
-    const uint8_t *rpC;
-    const uint16_t *mC;
-    uint8_t *ixC;
-    double *vC;
-    int32_t *rowAcc;  // per tile row: accumulator doubles if the row kernel takes it, else -1
-    uint8_t *skip;    // per C tile
-    int dense_threshold;
     DevCounters *cnt;
 };
 
@@ -173,14 +141,35 @@ void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, co
                      int64_t *nC, int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s);
 void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
                      cudaStream_t s);
+void launch_sym_rows(const S1Params &P, int64_t tm, cudaStream_t s);
+bool launch_structural(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const int64_t *tpB, const int32_t *tcB,
+                       int64_t tnB, DevCounters *cnt, cudaStream_t s);
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s);
 void launch_compact(const CompactParams &P, cudaStream_t s);
+
+// ---------------- a4 on the row path (tsg_rows.cu)
+struct RowNumArgs {
+    int64_t tm;
+    const tsg_tiles *A, *B;
+    tsg_tiles *C;                 // tile_ptr filled; the other arrays allocated
+    const uint16_t *mTB, *rowOccB;
+    const int64_t *costOff;
+    const uint64_t *pairs;
+    const int32_t *tJ;
+    const uint32_t *tStart, *tCnt, *tNnz;
+    const uint16_t *sMaskC;
+    const uint8_t *sRowPtrC;
+    const int64_t *rowOff;        // [tm+1] exclusive scan of the rows' nnz
+    int dense_threshold, small_max;
+    int64_t n_dense;              // dense C tiles (counted by k_sym_rows)
+    void *dense;                  // scratch for their records (32 B each)
+    DevCounters *cnt;
+};
+constexpr int DENSE_REC_BYTES = 32;
+void launch_num_rows(const RowNumArgs &a, cudaStream_t s);
 
 // launchers (tsg_step23.cu)
 void launch_step2(const StepParams &P, cudaStream_t s);
 void launch_step3(const StepParams &P, int64_t n_dense, cudaStream_t s);
-// launchers (tsg_step3row.cu)
-void launch_step3_class(const RowParams &R, cudaStream_t s);
-void launch_step3_rows(const RowParams &R, cudaStream_t s);
 
 }  // namespace tsg

@@ -1,14 +1,19 @@
 // tsg_spgemm.cu -- host orchestration of one tsg_spgemm call: the three steps of TileSpGEMM
-// (Section 3.3) with the device prefix sums and allocations between them.
+// (Section 3.3) with the device prefix sums and the allocation between them.
 //
-//   a0  helper indices (tsg_step1.cu): occupancy words, optional B row lists
-//   a1  step 1 (tsg_step1.cu): exact C tile layout + contributing pairs in ascending K
-//   a2  step 2 (tsg_step23.cu): bit-mask symbolic phase, row offsets, tile nnz
-//   a3  device prefix sums + allocation of C (tsg_scan.cu, stream-ordered pool)
-//   a4  step 3 (tsg_step23.cu): numeric phase with the adaptive accumulator
-//
-// Blocking device->host reads: (0) candidate total and row classes, (1) number of C tiles,
-// (2) nnz(C).  Everything else is stream-ordered.
+//   a0  helper indices (tsg_step1.cu): occupancy words, transposed masks, optional B row lists
+//   a1  plan: candidate count per A tile, prefix sum, per-row class       -> blocking read #1
+//   Row path (every non-empty tile row has <= 32 A tiles: stencils, FEM, banded):
+//     a1+a2  k_sym_rows: per tile row, the exact C tile set + pairs (warp merge) and each C
+//            tile's masks / row offsets / nnz, at the row's candidate-space slots
+//     a3     prefix sums of the rows' tile counts and nnz                -> blocking read #2
+//            (C's tile count and nnz together), then C is allocated once
+//     a4     k_num_rows: per tile row, C's tile records copied into place + the numeric phase
+//   Per-C-tile path (wide tile rows: power-law graphs, hubs):
+//     a1     merge / shared-memory sort / bitmap rank per row class; scan -> read #2 (tile count)
+//     a2     k_s2_light / k_s2 per group of 32 C tiles; scan of tile nnz -> read #3 (nnz(C))
+//     a4     k_s3_small / k_s3 / k_s3_dense per group of 32 C tiles
+// Both paths give the same C bit for bit (tests/test_gpu_parity.py).
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
@@ -40,9 +45,7 @@ struct Timer {
             for (auto &e : ev) cudaEventDestroy(e);
     }
 };
-}  // namespace
 
-namespace {
 // A side stream forked from `s` (one cached non-blocking stream and two events per host thread
 // and device); join() makes `s` wait for the side work, and the destructor joins if nothing did
 class SideStream {
@@ -61,7 +64,10 @@ class SideStream {
         TSG_CUDA(cudaStreamWaitEvent(r_->side, r_->fork, 0));
     }
     cudaStream_t stream() const { return r_->side; }
-    void done() { TSG_CUDA(cudaEventRecord(r_->joinev, r_->side)); recorded_ = true; }
+    void done() {
+        TSG_CUDA(cudaEventRecord(r_->joinev, r_->side));
+        recorded_ = true;
+    }
     void join() {
         if (joined_) return;
         if (!recorded_) done();
@@ -88,6 +94,7 @@ class SideStream {
 void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Allocator &al, cudaStream_t s,
                 tsg_tiles *C, tsg_stats *st) {
     reset_call_launches();
+    TSG_REQUIRE((flags & ~(uint32_t)TSG_SPGEMM_FLAGS) == 0, TSG_ERR_INVALID_ARG, "unknown tsg_spgemm flag");
     TSG_REQUIRE(A->nt < ((int64_t)1 << 31) && B->nt < ((int64_t)1 << 31), TSG_ERR_OVERFLOW, "input has >= 2^31 tiles");
     TSG_REQUIRE(A->tn == B->tm, TSG_ERR_SHAPE, "tile shapes disagree");
     TSG_REQUIRE(A->dtype == B->dtype, TSG_ERR_INVALID_ARG, "A and B value types differ");
@@ -97,7 +104,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
                 TSG_ERR_INVALID_ARG, "mask and row_ptr arrays must be 16-byte aligned, val aligned to its type");
     int TH = (int)((flags >> TSG_DENSE_THRESHOLD_SHIFT) & 0x1ffu);
     if (TH == 0) TH = TSG_DENSE_NNZ;
-    if (const char *e = getenv("TSG_DENSE_THRESHOLD")) TH = std::max(1, std::min(257, atoi(e)));  // tuning only
+    TSG_REQUIRE(TH <= 257, TSG_ERR_INVALID_ARG, "dense threshold > 257");
+    const int qv = (int)((flags >> TSG_QUEUE_CHUNK_SHIFT) & 0xfu);
     Timer tm_;
     tm_.init((flags & TSG_STATS_TIMING) && st, s);
     tm_.mark(0);
@@ -124,8 +132,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         launch_occupancy(A->mask, ntA, nullptr, colOccA, s);
         launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
     }
-    // transposed masks: first used by step 2, so they are computed on a side stream while step 1
-    // runs (joined before step 2, and on every exit path by the guard's destructor)
+    // transposed masks: first used by step 2 / 3, so they are computed on a side stream while
+    // step 1 runs (joined before their first use, and on every exit path by the guard's destructor)
     uint16_t *mTB = tmp.get<uint16_t>(TILE * B->nt);
     uint16_t *mTA = inB ? mTB + TILE * off : tmp.get<uint16_t>(TILE * ntA);
     SideStream side(s);
@@ -148,9 +156,12 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         int32_t *rnnz = tmp.get<int32_t>(TILE * tmB);
         launch_products(tmB, B->tile_ptr, B->mask, ntA, A->tile_col, A->mask, rnnz, cnt, s);
     }
+    bool structural = false;
+    if (st && (flags & TSG_STATS_STRUCTURAL) && tmA > 0)
+        structural = launch_structural(tmA, A->tile_ptr, A->tile_col, B->tile_ptr, B->tile_col, B->tn, cnt, s);
     tm_.mark(1);
 
-    // ---------------- a1: step 1
+    // ---------------- a1: plan
     int64_t *cost = tmp.get<int64_t>(ntA);
     int64_t *startA = tmp.get<int64_t>(ntA);
     int32_t *jloA = tmp.get<int32_t>(ntA);
@@ -167,12 +178,13 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     int64_t *bigOff = tmp.get<int64_t>(tmA);
     launch_row_plan(tmA, A->tile_ptr, costOff, jloA, jhiA, !(flags & TSG_STEP1_SORT_ONLY), rowJlo, rowJhi, rowClass,
                     nC, bigList, bigOff, cnt, s);
-    // sync #0: candidate total and row classes
+    // blocking read #1: candidate total and row classes (sizes of the step-1 scratch)
     DevCounters hc{};
     int64_t Utot = 0;
     read_device({{&Utot, costOff + ntA, sizeof(int64_t)}, {&hc, cnt, sizeof(DevCounters)}}, s);
     syncs++;
     TSG_REQUIRE(Utot < ((int64_t)1 << 40), TSG_ERR_OVERFLOW, "too many step-1 candidates");
+    tm_.mark(2);
 
     S1Params P1{};
     P1.tpA = A->tile_ptr;
@@ -197,128 +209,155 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.bigList = bigList;
     P1.bigOff = bigOff;
     P1.cnt = cnt;
-    if (hc.nbig > 0) {
-        P1.bigKeysA = tmp.get<uint64_t>(hc.big_u);
-        P1.bigKeysB = tmp.get<uint64_t>(hc.big_u);
-        P1.bigPosB = tmp.get<uint32_t>(hc.big_u);
-        P1.bigKpos = tmp.get<uint32_t>(hc.big_u);
-    }
-    launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, (int64_t)hc.nmerge, s);
+    P1.mA = A->mask;
+    P1.mB = B->mask;
+
+    // the row path needs every non-empty tile row to be a merge row (<= 32 A tiles).  It wins where
+    // the call is small (fewer launches and blocking reads: C1) or A's tiles are dense enough to
+    // make dense C tiles common (C3: 0.89 vs 1.0 ms); on sparse-tile stencils (C2: 17 nnz per A
+    // tile) the per-C-tile kernels run at higher occupancy and are faster
+    const bool narrow = !(flags & (TSG_PATH_GENERAL | TSG_STEP1_SORT_ONLY)) && hc.nbig == 0 && hc.max_u_small == 0 &&
+                        tmA > 0;
+    const bool rowpath = narrow && ((flags & TSG_PATH_ROWS_FORCE) || A->nnz >= 32 * A->nt || Utot <= ROWPATH_SMALL_U);
+    int64_t ntC = 0, nnzC = 0;
     int64_t *tile_ptr = out.get<int64_t>(tmA + 1);
-    exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
-    tm_.mark(2);
-    // sync #1: number of C tiles
-    const int64_t ntC = read_scalar(tile_ptr + tmA, s);
-    syncs++;
-    TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
+    if (rowpath) {
+        P1.sMaskC = tmp.get<uint16_t>(TILE * Utot);
+        P1.sRowPtrC = tmp.get<uint8_t>(TILE * Utot);
+        P1.rowNnz = tmp.get<int64_t>(tmA);
+        P1.dense_threshold = TH;
+        launch_sym_rows(P1, tmA, s);
+        tm_.mark(3);
+        // ---------------- a3: tile and nonzero offsets of the rows; the one allocation of C
+        int64_t *rowOff = tmp.get<int64_t>(tmA + 1);
+        exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
+        exclusive_scan<int64_t>(P1.rowNnz, rowOff, tmA, s, tmp);
+        DevCounters hc2{};
+        read_device({{&ntC, tile_ptr + tmA, sizeof(int64_t)}, {&nnzC, rowOff + tmA, sizeof(int64_t)},
+                     {&hc2, cnt, sizeof(DevCounters)}}, s);
+        syncs++;
+        TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
+        C->tile_col = out.get<int32_t>(ntC);
+        C->tile_nnz = out.get<int64_t>(ntC + 1);
+        C->row_ptr = out.get<uint8_t>(TILE * ntC);
+        C->mask = out.get<uint16_t>(TILE * ntC);
+        C->idx = out.get<uint8_t>(nnzC);
+        C->val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
+        C->tile_ptr = tile_ptr;
+        tm_.mark(4);
+        side.join();
+        // ---------------- a4: step 3
+        RowNumArgs R{};
+        R.tm = tmA;
+        R.A = A;
+        R.B = B;
+        R.C = C;
+        R.mTB = mTB;
+        R.rowOccB = rowOccB;
+        R.costOff = costOff;
+        R.pairs = P1.pairs;
+        R.tJ = P1.tJ;
+        R.tStart = P1.tStart;
+        R.tCnt = P1.tCnt;
+        R.tNnz = P1.tWork;
+        R.sMaskC = P1.sMaskC;
+        R.sRowPtrC = P1.sRowPtrC;
+        R.rowOff = rowOff;
+        R.dense_threshold = TH;
+        R.small_max = SMALL_NNZ;
+        R.n_dense = (int64_t)hc2.n2dense;
+        R.dense = hc2.n2dense ? tmp.get<uint8_t>(DENSE_REC_BYTES * (int64_t)hc2.n2dense) : nullptr;
+        R.cnt = cnt;
+        launch_num_rows(R, s);
+        tm_.mark(5);
+    } else {
+        if (hc.nbig > 0) {
+            P1.bigKeysA = tmp.get<uint64_t>(hc.big_u);
+            P1.bigKeysB = tmp.get<uint64_t>(hc.big_u);
+            P1.bigPosB = tmp.get<uint32_t>(hc.big_u);
+            P1.bigKpos = tmp.get<uint32_t>(hc.big_u);
+        }
+        launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, (int64_t)hc.nmerge, s);
+        exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
+        // blocking read #2: number of C tiles
+        ntC = read_scalar(tile_ptr + tmA, s);
+        syncs++;
+        TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
+        tm_.mark(3);
+        // C's tile arrays, per-tile pair ranges
+        int32_t *tile_col = out.get<int32_t>(ntC);
+        int64_t *tile_nnz = out.get<int64_t>(ntC + 1);
+        uint8_t *row_ptr = out.get<uint8_t>(TILE * ntC);
+        uint16_t *mask = out.get<uint16_t>(TILE * ntC);
+        int64_t *pairBeg = tmp.get<int64_t>(ntC);
+        uint32_t *pairCnt = tmp.get<uint32_t>(ntC);
+        uint32_t *work = tmp.get<uint32_t>(ntC);
+        CompactParams PC{tmA, A->tile_ptr, costOff, tile_ptr, P1.tJ, P1.tStart, P1.tCnt, P1.tWork,
+                         tile_col, pairBeg, pairCnt, work};
+        launch_compact(PC, s);
 
-    // ---------------- allocation of C's tile arrays, per-tile pair ranges, class lists
-    int32_t *tile_col = out.get<int32_t>(ntC);
-    int64_t *tile_nnz = out.get<int64_t>(ntC + 1);
-    uint8_t *row_ptr = out.get<uint8_t>(TILE * ntC);
-    uint16_t *mask = out.get<uint16_t>(TILE * ntC);
-    int64_t *pairBeg = tmp.get<int64_t>(ntC);
-    uint32_t *pairCnt = tmp.get<uint32_t>(ntC);
-    uint32_t *work = tmp.get<uint32_t>(ntC);
-    tm_.mark(3);
-    CompactParams PC{tmA, A->tile_ptr, costOff, tile_ptr, P1.tJ, P1.tStart, P1.tCnt, P1.tWork,
-                     tile_col, pairBeg, pairCnt, work};
-    launch_compact(PC, s);
-
-    // ---------------- a2: step 2
-    side.join();
-    StepParams P{};
-    P.ntC = ntC;
-    P.pairBeg = pairBeg;
-    P.pairCnt = pairCnt;
-    P.pairs = P1.pairs;
-    P.tnzA = A->tile_nnz;
-    P.rpA = A->row_ptr;
-    P.mA = A->mask;
-    P.mTA = mTA;
-    P.colOccA = colOccA;
-    P.ixA = A->idx;
-    P.vA = A->val;
-    P.dtype_in = A->dtype;
-    P.tnzB = B->tile_nnz;
-    P.rpB = B->row_ptr;
-    P.mB = B->mask;
-    P.rowOccB = rowOccB;
-    P.mTB = mTB;
-    P.ixB = B->idx;
-    P.vB = B->val;
-    P.tnzC = tile_nnz;
-    P.rpC = row_ptr;
-    P.mC = mask;
-    P.work = work;
-    {
-        const int64_t ng = (ntC + 31) / 32;
-        P.medL = tmp.get<uint32_t>(ng);
-        P.medH = tmp.get<uint32_t>(ng);
-        P.denL = tmp.get<uint32_t>(ng);
-        P.denH = tmp.get<uint32_t>(ng);
-    }
-    P.dense_threshold = TH;
-    P.small_max = SMALL_NNZ;
-    P.dense_tc = ((flags & TSG_DENSE_TC) || getenv("TSG_DENSE_TC")) ? 1 : 0;  // env: tuning only
-    // small-tile B staging pays where B's tile metadata misses in cache: hypersparse tiles
-    // (fewer than 4 nonzeros per B tile on average, e.g. R-MAT); flags force either way
-    P.small_stage = (flags & TSG_SMALL_STAGE_ON) ? 1 : (flags & TSG_SMALL_STAGE_OFF) ? 0 : (B->nnz < 4 * B->nt);
-    if (const char *e = getenv("TSG_SMALL_NNZ")) P.small_max = std::max(0, std::min(16, atoi(e)));  // tuning only
-    P.cnt = cnt;
-    launch_step2(P, s);
-    // ---------------- a3: offsets of C's nonzeros, allocation
-    exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp);
-    tm_.mark(4);
-    // step-3 row classes: whole C tile rows for the row kernel, the rest per tile
-    RowParams R{};
-    R.tm = tmA;
-    R.tpA = A->tile_ptr;
-    R.tcA = A->tile_col;
-    R.tnzA = A->tile_nnz;
-    R.rpA = A->row_ptr;
-    R.mA = A->mask;
-    R.colOccA = colOccA;
-    R.vA = static_cast<const double *>(A->val);
-    R.tpB = B->tile_ptr;
-    R.tnzB = B->tile_nnz;
-    R.rpB = B->row_ptr;
-    R.mB = B->mask;
-    R.vB = static_cast<const double *>(B->val);
-    R.pairs = P1.pairs;
-    R.pairBeg = pairBeg;
-    R.pairCnt = pairCnt;
-    R.tpC = tile_ptr;
-    R.tnzC = tile_nnz;
-    R.rpC = row_ptr;
-    R.mC = mask;
-    R.dense_threshold = TH;
-    R.cnt = cnt;
-    const bool rowk = (flags & TSG_STEP3_ROWS) != 0 && A->dtype == TSG_F64;  // the row kernel is fp64 only
-    if (rowk) {
-        R.rowAcc = tmp.get<int32_t>(tmA);
-        R.skip = tmp.get<uint8_t>(ntC);
-        launch_step3_class(R, s);
-    }
-    int64_t nnzC = 0;
-    DevCounters hc2{};
-    read_device({{&nnzC, tile_nnz + ntC, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
-    syncs++;
-    uint8_t *idx = out.get<uint8_t>(nnzC);
-    void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
-    tm_.mark(5);
-
-    // ---------------- a4: step 3
-    P.ixC = idx;
-    P.vC = val;
-    R.ixC = idx;
-    R.vC = static_cast<double *>(val);
-    if (rowk && hc2.n3rows > 0) launch_step3_rows(R, s);
-    if (!rowk || hc2.n3fallback > 0) {
-        P.skip = rowk ? R.skip : nullptr;
+        // ---------------- a2: step 2
+        side.join();
+        StepParams P{};
+        P.ntC = ntC;
+        P.pairBeg = pairBeg;
+        P.pairCnt = pairCnt;
+        P.pairs = P1.pairs;
+        P.tnzA = A->tile_nnz;
+        P.rpA = A->row_ptr;
+        P.mA = A->mask;
+        P.mTA = mTA;
+        P.colOccA = colOccA;
+        P.ixA = A->idx;
+        P.vA = A->val;
+        P.dtype_in = A->dtype;
+        P.tnzB = B->tile_nnz;
+        P.rpB = B->row_ptr;
+        P.mB = B->mask;
+        P.rowOccB = rowOccB;
+        P.mTB = mTB;
+        P.ixB = B->idx;
+        P.vB = B->val;
+        P.tnzC = tile_nnz;
+        P.rpC = row_ptr;
+        P.mC = mask;
+        P.work = work;
+        {
+            const int64_t ng = (ntC + 31) / 32;
+            P.medL = tmp.get<uint32_t>(ng);
+            P.medH = tmp.get<uint32_t>(ng);
+            P.denL = tmp.get<uint32_t>(ng);
+            P.denH = tmp.get<uint32_t>(ng);
+        }
+        P.qoverride = qv == 0 ? -1 : qv - 1;
+        P.dense_threshold = TH;
+        P.small_max = SMALL_NNZ;
+        // small-tile B staging pays where B's tile metadata misses in cache: hypersparse tiles
+        // (fewer than 4 nonzeros per B tile on average, e.g. R-MAT); flags force either way
+        P.small_stage = (flags & TSG_SMALL_STAGE_ON) ? 1 : (flags & TSG_SMALL_STAGE_OFF) ? 0 : (B->nnz < 4 * B->nt);
+        P.cnt = cnt;
+        launch_step2(P, s);
+        // ---------------- a3: offsets of C's nonzeros, allocation
+        exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp);
+        DevCounters hc2{};
+        read_device({{&nnzC, tile_nnz + ntC, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
+        syncs++;
+        uint8_t *idx = out.get<uint8_t>(nnzC);
+        void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
+        tm_.mark(4);
+        // ---------------- a4: step 3
+        P.ixC = idx;
+        P.vC = val;
         launch_step3(P, (int64_t)hc2.n2dense, s);
+        tm_.mark(5);
+        C->tile_ptr = tile_ptr;
+        C->tile_col = tile_col;
+        C->tile_nnz = tile_nnz;
+        C->row_ptr = row_ptr;
+        C->mask = mask;
+        C->idx = idx;
+        C->val = val;
     }
-    tm_.mark(6);
 
     // ---------------- the result handle
     C->m = A->m;
@@ -327,17 +366,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     C->tn = B->tn;
     C->nt = ntC;
     C->nnz = nnzC;
-    C->tile_ptr = tile_ptr;
-    C->tile_col = tile_col;
-    C->tile_nnz = tile_nnz;
-    C->row_ptr = row_ptr;
-    C->mask = mask;
-    C->idx = idx;
-    C->val = val;
     C->dtype = dtC;
-    void *arr[7] = {tile_ptr, tile_col, tile_nnz, row_ptr, mask, idx, val};
     for (int k = 0; k < 7; k++) {
-        C->bytes[k] = out.take(arr[k]);
+        C->bytes[k] = out.take(C->array(k));
         C->owns[k] = true;
     }
     C->al = al;
@@ -346,15 +377,15 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         read_device({{&fin, cnt, sizeof(DevCounters)}}, s);
         memset(st, 0, sizeof(*st));
         st->products = (flags & TSG_STATS_PRODUCTS) ? (int64_t)fin.products : -1;
-        st->tiles_structural = -1;
+        st->tiles_structural = structural ? (int64_t)fin.structural : ((flags & TSG_STATS_STRUCTURAL) && tmA == 0 ? 0 : -1);
         st->tiles_c = ntC;
         st->nnz_c = nnzC;
         st->candidates = Utot;
         st->pairs = (int64_t)fin.pairs;
         st->tiles_dense = (int64_t)fin.n3dense;
         st->tiles_sparse = ntC - (int64_t)fin.n3dense;
-        st->step3_rows = (int64_t)fin.n3rows;
-        st->step3_row_tiles = rowk ? ntC - (int64_t)fin.n3fallback : 0;
+        st->path = rowpath ? TSG_PATH_ROWS : TSG_PATH_TILES;
+        st->step1_big_rows = (int64_t)fin.nbig;
         st->step1_list_tiles = (int32_t)fin.list_tiles;
         st->step1_merge_rows = (int64_t)fin.nmerge;
         st->bytes_scratch = (int64_t)tmp.handed();
@@ -366,11 +397,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         st->ms_host_alloc = (float)t_host_alloc_ms;
         if (tm_.on) {
             st->ms_index = tm_.ms(0, 1);
-            st->ms_step1 = tm_.ms(1, 2);
-            st->ms_alloc = tm_.ms(2, 3) + tm_.ms(4, 5);
-            st->ms_step2 = tm_.ms(3, 4);
-            st->ms_step3 = tm_.ms(5, 6);
-            st->ms_total = tm_.ms(0, 6);
+            st->ms_step1 = tm_.ms(1, 2) + (rowpath ? 0.f : tm_.ms(2, 3));
+            st->ms_step2 = rowpath ? tm_.ms(2, 3) : tm_.ms(3, 4);
+            st->ms_alloc = rowpath ? tm_.ms(3, 4) : 0.f;
+            st->ms_step3 = tm_.ms(4, 5);
+            st->ms_total = tm_.ms(0, 5);
         }
     }
 }

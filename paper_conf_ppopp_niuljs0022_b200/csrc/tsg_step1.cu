@@ -7,7 +7,9 @@
 // row's candidates by tile column J (stable, so pairs stay in ascending K), and the heads of
 // equal-J runs are the non-empty C tiles.  Pairs without products (colOcc(A)&rowOcc(B) == 0) are
 // dropped (reading B3), so C never stores an empty tile (reading A6).
-#include "tsg_kernels.cuh"
+#include <algorithm>
+
+#include "tsg_device.cuh"
 
 namespace tsg {
 namespace {
@@ -91,6 +93,33 @@ __global__ void k_products(int64_t ntA, const int32_t *__restrict__ tcA, const u
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(FULL, p, o);
     if ((threadIdx.x & 31) == 0 && p) atomicAdd(&cnt->products, p);
+}
+
+// ------------------------------------------------------------------------------------------
+// diagnostic (TSG_STATS_STRUCTURAL): |C'| of the paper's step 1, the structural tile product A'B'
+// with its empty tiles: per tile row, the distinct tile columns J over
+// every B tile of every B tile row K with A_IK stored, marked in a shared-memory bitmap.
+// ------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_structural(const int64_t *__restrict__ tpA, const int32_t *__restrict__ tcA,
+                                                   const int64_t *__restrict__ tpB, const int32_t *__restrict__ tcB,
+                                                   int words, DevCounters *cnt) {
+    extern __shared__ uint32_t bm[];
+    const int64_t I = blockIdx.x;
+    for (int w = threadIdx.x; w < words; w += blockDim.x) bm[w] = 0;
+    __syncthreads();
+    for (int64_t a = tpA[I]; a < tpA[I + 1]; a++) {
+        const int64_t K = tcA[a];
+        for (int64_t b = tpB[K] + threadIdx.x; b < tpB[K + 1]; b += blockDim.x) {
+            const uint32_t J = (uint32_t)tcB[b];
+            atomicOr(&bm[J >> 5], 1u << (J & 31));
+        }
+    }
+    __syncthreads();
+    u64c c = 0;
+    for (int w = threadIdx.x; w < words; w += blockDim.x) c += __popc(bm[w]);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULL, c, o);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(&cnt->structural, c);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -412,14 +441,12 @@ struct MergeOut {
 constexpr int MERGE_W = TSG_MERGE_W;  // warps (tile rows) per merge CTA
 constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (6 B each)
 
-__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
+// One tile row's merge by one warp (sJw / sKw: the warp's MERGE_CAP staging slots).  Writes the
+// row's pairs and C tile records at its candidate-space slots; returns the row's C tile count
+// (warp-uniform).
+__device__ uint32_t merge_row(const S1Params &P, int64_t I, int lane, uint32_t *sJrow, uint16_t *sKrow) {
     constexpr uint32_t INF = 0xffffffffu;
     constexpr uint32_t JM = (1u << 27) - 1u;  // tile column bits (n < 2^31); bits 27..31: work
-    __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
-    __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
-    if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
     const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
     const int64_t base = P.costOff[a0];
     const int64_t U = P.costOff[a1] - base;
@@ -446,8 +473,8 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
         const int ioff = (int)off, ilen = (int)len;
         const uint32_t st32 = (uint32_t)st;
         const uint32_t *lst = isl ? P.list + st : nullptr;
-        uint32_t *sJw = &sJ[w][ioff];
-        uint16_t *sKw = &sK[w][ioff];
+        uint32_t *sJw = sJrow + ioff;
+        uint16_t *sKw = sKrow + ioff;
         int cntv = 0;
 #pragma unroll 4
         for (int k = 0; k < ilen; k++) {
@@ -485,7 +512,7 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
             }
         }
         out.finish(P, base, lane, I);
-        return;
+        return out.ntl;
     }
     // rows with more candidates than the stage holds: each lane keeps four candidates in flight
     constexpr uint32_t JINF = 0x7fffffffu;
@@ -537,6 +564,262 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
         if (hit) advance();
     }
     out.finish(P, base, lane, I);
+    return out.ntl;
+}
+
+__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
+    __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
+    __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
+    if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
+    merge_row(P, I, lane, sJ[w], sK[w]);
+}
+
+// ------------------------------------------------------------------------------------------
+// a1 + a2 fused (the row path: every tile row has <= 32 A tiles).  One warp per tile row: the
+// k-way merge above gives the row's C tiles and their contributing pairs (step 1), then, with the
+// row's A masks staged once in shared memory, each C tile's bit masks are OR-ed from its pairs
+// (step 2, Alg 2 l.19-25: mask_C[r] |= mask_B[c] for every nonzero (r,c) of A_IK) by
+// a half warp with lane r owning row r (no atomics), followed by the 16-entry row offsets and the
+// tile nnz.  Results go to the row's candidate-space slots (C is allocated once, after this
+// kernel); the row's nnz total goes to rowNnz[I] for the row-offset scan.
+// ------------------------------------------------------------------------------------------
+// Step 1 of one narrow tile row by bitmap ranks instead of the merge's serial steps (a warp, no
+// barriers): (1) every lane walks its A tile's candidate list and marks the tile columns J that
+// have a product (reading B3) in a bitmap over the row's J window; (2) a popcount prefix over the
+// words gives every marked J its rank = its C tile's index in the row (tile columns ascend, as
+// P:801-804 require), and the C tile records' J; (3) each candidate ORs its lane bit into its C
+// tile's lane mask -- lane order is ascending K, so a pair's slot in its tile's list is the tile's
+// start + the contributors on lower lanes (reading A8); (4) a scan of the masks' popcounts gives
+// the starts, (5) every candidate writes its pair.  Returns the row's C tile count, or ~0u when
+// the row has more than RK_MAXC C tiles (the caller falls back to the merge).  Same outputs, in
+// the same candidate-space slots, as merge_row.
+constexpr int RK_MAXU = 1024;  // candidates of the row (packed: jr or rank << 10 | k)
+constexpr int RK_WORDS = 256;  // bitmap words: a J window of <= 8192 tile columns
+constexpr int RK_MAXC = 512;   // C tiles of the row
+struct RankSmem {
+    uint32_t cand[RK_MAXU];
+    uint32_t bm[RK_WORDS];
+    uint32_t lm[RK_MAXC];
+    uint16_t pre[RK_WORDS];
+    uint16_t ps[RK_MAXC];
+};
+static_assert(sizeof(RankSmem) >= MERGE_CAP * 6, "the merge's staging fits the rank's");
+
+__device__ uint32_t rank_row(const S1Params &P, int64_t I, int lane, RankSmem &R) {
+    constexpr uint32_t BAD = 0xffffffffu;
+    const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
+    const int64_t base = P.costOff[a0];
+    const int32_t jlo = P.rowJlo[I];
+    const int words = (P.rowJhi[I] - jlo + 32) >> 5;
+    const int64_t t = a0 + lane;
+    int len = 0, off = 0;
+    int64_t st = 0;
+    bool isl = false;
+    uint32_t co = 0;
+    if (t < a1) {
+        off = (int)(P.costOff[t] - base);
+        len = (int)(P.costOff[t + 1] - base - off);
+        st = P.startA[t];
+        isl = st < 0;
+        if (isl) st = -st - 1;
+        co = P.colOccA[t];
+    }
+    const uint32_t *lst = isl ? P.list + st : nullptr;
+    const uint32_t st32 = (uint32_t)st;
+    for (int w = lane; w < words; w += 32) R.bm[w] = 0;
+    __syncwarp();
+    // (1) mark
+    uint32_t *cand = R.cand + off;
+#pragma unroll 4
+    for (int k = 0; k < len; k++) {
+        const uint32_t pos = isl ? lst[k] : st32 + (uint32_t)k;
+        const bool valid = isl || (co & (uint32_t)P.rowOccB[pos]) != 0;
+        uint32_t x = BAD;
+        if (valid) {
+            const uint32_t jr = (uint32_t)(P.tcB[pos] - jlo);
+            x = jr << 10 | (uint32_t)k;
+            atomicOr(&R.bm[jr >> 5], 1u << (jr & 31));
+        }
+        cand[k] = x;
+    }
+    __syncwarp();
+    // (2) ranks of the marked columns: word popcount prefix; the C tile records' J
+    uint32_t run = 0;
+    for (int w0 = 0; w0 < words; w0 += 32) {
+        const int w = w0 + lane;
+        const uint32_t bw = w < words ? R.bm[w] : 0u;
+        const uint32_t c = __popc(bw);
+        uint32_t incl = c;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t o = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl += o;
+        }
+        const uint32_t pre = run + incl - c;
+        if (w < words) R.pre[w] = (uint16_t)min(pre, 0xffffu);
+        run += __shfl_sync(FULL, incl, 31);
+        if (run <= (uint32_t)RK_MAXC) {
+            uint32_t m = bw, q = pre;
+            while (m) {
+                const int b = __ffs(m) - 1;
+                m &= m - 1;
+                P.tJ[base + q++] = jlo + 32 * w + b;
+            }
+        }
+    }
+    const uint32_t nC = run;
+    if (nC > (uint32_t)RK_MAXC) return ~0u;  // warp-uniform
+    for (uint32_t q = lane; q < nC; q += 32) R.lm[q] = 0;
+    __syncwarp();
+    // (3) contributors of every C tile, as lane masks (lane order = ascending K)
+    for (int k = 0; k < len; k++) {
+        const uint32_t x = cand[k];
+        if (x == BAD) continue;
+        const uint32_t jr = x >> 10;
+        const uint32_t rk = R.pre[jr >> 5] + __popc(R.bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
+        cand[k] = rk << 10 | (x & 1023u);
+        atomicOr(&R.lm[rk], 1u << lane);
+    }
+    __syncwarp();
+    // (4) pair starts of the C tiles (row-relative), pair counts
+    uint32_t np = 0;
+    for (uint32_t q0 = 0; q0 < nC; q0 += 32) {
+        const uint32_t q = q0 + lane;
+        const uint32_t c = q < nC ? __popc(R.lm[q]) : 0u;
+        uint32_t incl = c;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t o = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl += o;
+        }
+        if (q < nC) {
+            const uint32_t pst = np + incl - c;
+            R.ps[q] = (uint16_t)pst;
+            P.tStart[base + q] = pst;
+            P.tCnt[base + q] = c;
+        }
+        np += __shfl_sync(FULL, incl, 31);
+    }
+    __syncwarp();
+    // (5) the pairs, (posA << 32) | posB, in ascending K within every C tile
+    const unsigned lt = (1u << lane) - 1u;
+    const uint64_t thi = (uint64_t)t << 32;
+    for (int k = 0; k < len; k++) {
+        const uint32_t x = cand[k];
+        if (x == BAD) continue;
+        const uint32_t rk = x >> 10, kk = x & 1023u;
+        const uint32_t pos = isl ? lst[kk] : st32 + kk;
+        P.pairs[base + R.ps[rk] + __popc(R.lm[rk] & lt)] = thi | pos;
+    }
+    if (lane == 0) {
+        P.nC[I] = nC;
+        atomicAdd(&P.cnt->pairs, (u64c)np);
+    }
+    return nC;
+}
+
+__global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t tm) {
+    __shared__ __align__(16) RankSmem sR[MERGE_W];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
+    if (I >= tm) return;  // warp-uniform
+    if (P.rowClass[I] != ROW_MERGE) {  // empty row (the row path runs only when no other class exists)
+        if (lane == 0) P.rowNnz[I] = 0;
+        return;
+    }
+    uint32_t nC = ~0u;
+    {
+        const int64_t a0 = P.tpA[I];
+        const int64_t U = P.costOff[P.tpA[I + 1]] - P.costOff[a0];
+        if (U <= RK_MAXU && P.rowJhi[I] - P.rowJlo[I] < 32 * RK_WORDS) nC = rank_row(P, I, lane, sR[w]);
+    }
+    __syncwarp();
+    if (nC == ~0u)
+        nC = merge_row(P, I, lane, reinterpret_cast<uint32_t *>(&sR[w]),
+                       reinterpret_cast<uint16_t *>(reinterpret_cast<uint32_t *>(&sR[w]) + MERGE_CAP));
+    __syncwarp();  // the row's pairs and C tile records (global) are visible to the whole warp
+    const int64_t a0 = P.tpA[I];
+    const int nA = (int)(P.tpA[I + 1] - a0);
+    const int64_t base = P.costOff[a0];
+    // staging area (reuses the merge's): A row masks [32][16], then per half warp the B masks,
+    // B row occupancy and A slots of a batch of 16 pairs
+    unsigned char *wsm = reinterpret_cast<unsigned char *>(&sR[w]);
+    uint16_t *sMA = reinterpret_cast<uint16_t *>(wsm);
+    if (lane < nA) {
+        const uint4 *g = reinterpret_cast<const uint4 *>(P.mA + (a0 + lane) * TILE);
+        uint4 *d = reinterpret_cast<uint4 *>(sMA + lane * TILE);
+        d[0] = g[0];
+        d[1] = g[1];
+    }
+    const int r = lane & 15, half = lane >> 4;
+    unsigned char *hs = wsm + 1024 + half * 576;
+    uint16_t *sMB = reinterpret_cast<uint16_t *>(hs);        // [16][16]
+    uint16_t *sOB = reinterpret_cast<uint16_t *>(hs + 512);  // [16]
+    uint8_t *sS = hs + 544;                                  // [16]
+    __syncwarp();
+    int64_t rownnz = 0;
+    uint32_t ndense = 0;
+    for (uint32_t q0 = 0; q0 < nC; q0 += 2) {
+        const uint32_t q = q0 + half;
+        const bool hv = q < nC;
+        uint32_t st = 0, cnt = 0;
+        if (hv) {
+            st = P.tStart[base + q];
+            cnt = P.tCnt[base + q];
+        }
+        uint32_t acc = 0;
+        const uint32_t nbat = (cnt + 15) / 16;
+        const uint32_t nbw = max(nbat, __shfl_xor_sync(FULL, nbat, 16));
+        for (uint32_t bt = 0; bt < nbw; bt++) {
+            const uint32_t i = bt * 16 + r;
+            if (i < cnt) {
+                const uint64_t pr = P.pairs[base + st + i];
+                const int64_t pB = (int64_t)(uint32_t)pr;
+                cp16(sMB + r * TILE, P.mB + pB * TILE);
+                cp16(sMB + r * TILE + 8, P.mB + pB * TILE + 8);
+                sOB[r] = P.rowOccB[pB];
+                sS[r] = (uint8_t)((int64_t)(pr >> 32) - a0);
+            }
+            cp_wait_all();
+            __syncwarp();
+            const uint32_t nb = cnt > bt * 16 ? min(16u, cnt - bt * 16) : 0u;
+            for (uint32_t k = 0; k < nb; k++) {
+                uint32_t ma = (uint32_t)sMA[sS[k] * TILE + r] & sOB[k];
+                const uint16_t *mb = sMB + k * TILE;
+                while (ma) {
+                    const int c = __ffs(ma) - 1;
+                    ma &= ma - 1;
+                    acc |= mb[c];
+                }
+            }
+            __syncwarp();
+        }
+        const int cn = __popc(acc);
+        int incl = cn;
+#pragma unroll
+        for (int d = 1; d < 16; d <<= 1) {
+            const int o = __shfl_up_sync(FULL, incl, d, 16);
+            if (r >= d) incl += o;
+        }
+        const int tot = __shfl_sync(FULL, incl, 15, 16);
+        if (hv) {
+            P.sMaskC[(base + q) * TILE + r] = (uint16_t)acc;
+            P.sRowPtrC[(base + q) * TILE + r] = (uint8_t)(incl - cn);
+            if (r == 0) {
+                P.tWork[base + q] = (uint32_t)tot;  // the tile's nnz (the row path has no step-2 class split)
+                rownnz += tot;
+                ndense += tot >= P.dense_threshold;
+            }
+        }
+    }
+    rownnz += __shfl_xor_sync(FULL, rownnz, 16);
+    ndense += __shfl_xor_sync(FULL, ndense, 16);
+    if (lane == 0) {
+        P.rowNnz[I] = rownnz;
+        if (ndense) atomicAdd(&P.cnt->n2dense, (u64c)ndense);
+    }
 }
 
 __global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int64_t tm, int cap) {
@@ -823,6 +1106,20 @@ void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStr
 
 void launch_compact(const CompactParams &P, cudaStream_t s) {
     TSG_LAUNCH(k_compact, grid_for(P.tm, 8), 256, 0, s, P);
+}
+
+bool launch_structural(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const int64_t *tpB, const int32_t *tcB,
+                       int64_t tnB, DevCounters *cnt, cudaStream_t s) {
+    const int64_t words = (tnB + 31) / 32;
+    if (words * 4 > 200 * 1024) return false;  // B too wide for the shared-memory bitmap
+    const size_t smem = (size_t)std::max<int64_t>(words, 1) * 4;
+    TSG_CUDA(cudaFuncSetAttribute(k_structural, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    TSG_LAUNCH(k_structural, (unsigned)tmA, 256, smem, s, tpA, tcA, tpB, tcB, (int)words, cnt);
+    return true;
+}
+
+void launch_sym_rows(const S1Params &P, int64_t tm, cudaStream_t s) {
+    TSG_LAUNCH(k_sym_rows, grid_for(tm, MERGE_W), MERGE_W * 32, 0, s, P, tm);
 }
 
 void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,

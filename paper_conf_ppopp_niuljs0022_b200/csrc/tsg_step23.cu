@@ -26,20 +26,10 @@
 #include <map>
 #include <mutex>
 
-#include <cuda_fp16.h>
-
-#include "tsg_kernels.cuh"
+#include "tsg_device.cuh"
 
 namespace tsg {
 namespace {
-
-// ---- value types: TI = stored input type, TO = accumulator/output type
-// (double x double -> double, float x float -> float, half x half -> float)
-template <typename TO> __device__ __forceinline__ TO vcvt(double x) { return (TO)x; }
-template <typename TO> __device__ __forceinline__ TO vcvt(float x) { return (TO)x; }
-template <typename TO> __device__ __forceinline__ TO vcvt(__half x) { return (TO)__half2float(x); }
-__device__ __forceinline__ double vfma(double a, double b, double c) { return fma(a, b, c); }
-__device__ __forceinline__ float vfma(float a, float b, float c) { return fmaf(a, b, c); }
 
 constexpr unsigned FULL = 0xffffffffu;
 #ifndef TSG_T2
@@ -55,68 +45,6 @@ constexpr int T2 = TSG_T2;  // step-2 CTA
 constexpr int T3 = TSG_T3;  // step-3 CTA (4 warps; 7.7 KB of shared memory per warp)
 constexpr int BATCH = 16;  // step 2: pairs staged per half warp at a time
 constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also the small path's 16 slots)
-
-// 16x16 bit-matrix transpose across the 16 lanes of a half warp: lane i holds row i (bit c =
-// M[i][c]); afterwards lane c holds column c (bit i = M[i][c]).  Four butterfly stages.
-__device__ __forceinline__ uint32_t bit_transpose16(uint32_t v, int r) {
-#pragma unroll
-    for (int s = 8; s > 0; s >>= 1) {
-        const uint32_t m = s == 8 ? 0x00ffu : s == 4 ? 0x0f0fu : s == 2 ? 0x3333u : 0x5555u;
-        const uint32_t x = __shfl_xor_sync(FULL, v, s);
-        v = (r & s) ? ((v & ~m & 0xffffu) | ((x >> s) & m)) : ((v & m) | ((x << s) & ~m & 0xffffu));
-    }
-    return v;
-}
-
-// rows r of a 16x16 tile (mask words w[0..7], two rows per word) with mask[r] & occ != 0, as bits
-__device__ __forceinline__ uint32_t rows_meeting(const uint4 &a0, const uint4 &a1, uint32_t occ) {
-    const uint32_t o2 = occ * 0x10001u;
-    const uint32_t w[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-    uint32_t rows = 0;
-#pragma unroll
-    for (int k = 0; k < 8; k++) {
-        const uint32_t h = __vcmpne2(w[k] & o2, 0u);
-        rows |= ((h & 1u) << (2 * k)) | (((h >> 16) & 1u) << (2 * k + 1));
-    }
-    return rows;
-}
-
-// Dynamic work distribution for the step-2/3 kernels: warps take the next `chunk` units (groups
-// of 32 C tiles) from a per-kernel counter, so the warps running at any moment work on
-// neighbouring C tiles (their pairs' A and B tiles stay in L2) and a warp that drew light groups
-// takes more.  The next chunk is requested one chunk ahead, so the atomic's latency overlaps the
-// current work; `chunk` (host-chosen, about 16 requests per warp) keeps the counter cold.
-struct WorkQueue {
-    unsigned long long *ctr;
-    int64_t n;
-    int chunk;          // 0: static grid-stride distribution (unit = first, first + stride, ...)
-    long long nxt = 0;  // lane 0: first unit of the next chunk
-    int64_t cur = 0, end = 0, stride = 0;
-    __device__ WorkQueue(unsigned long long *c, int64_t units, int ch, int lane, int warps_per_cta)
-        : ctr(c), n(units), chunk(ch) {
-        if (ch == 0) {
-            cur = (int64_t)blockIdx.x * warps_per_cta + (threadIdx.x >> 5);
-            stride = (int64_t)gridDim.x * warps_per_cta;
-        } else if (lane == 0) {
-            nxt = (long long)atomicAdd(ctr, (unsigned long long)ch);
-        }
-    }
-    __device__ __forceinline__ bool next(int64_t &u, int lane) {
-        if (chunk == 0) {
-            u = cur;
-            cur += stride;
-            return u < n;
-        }
-        if (cur >= end) {
-            cur = (int64_t)__shfl_sync(FULL, nxt, 0);
-            if (cur >= n) return false;
-            end = min(cur + (int64_t)chunk, n);
-            if (lane == 0) nxt = (long long)atomicAdd(ctr, (unsigned long long)chunk);
-        }
-        u = cur++;
-        return true;
-    }
-};
 
 // ==========================================================================================
 // step 2
@@ -202,11 +130,6 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
     if ((threadIdx.x & 31) == 0 && nd) atomicAdd(&P.cnt->n2dense, nd);
 }
 
-__device__ __forceinline__ void cp16s(void *dst_smem, const void *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
-}
-
 __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
@@ -242,10 +165,10 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
                 if (q < np) {
                     const uint64_t pr = pp[q];
                     const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-                    cp16s(&sMA[hw][r][0], P.mA + pA * TILE);
-                    cp16s(&sMA[hw][r][8], P.mA + pA * TILE + 8);
-                    cp16s(&sMB[hw][r][0], P.mB + pB * TILE);
-                    cp16s(&sMB[hw][r][8], P.mB + pB * TILE + 8);
+                    cp16(&sMA[hw][r][0], P.mA + pA * TILE);
+                    cp16(&sMA[hw][r][8], P.mA + pA * TILE + 8);
+                    cp16(&sMB[hw][r][0], P.mB + pB * TILE);
+                    cp16(&sMB[hw][r][8], P.mB + pB * TILE + 8);
                     sOB[hw][r] = P.rowOccB[pB];
                 }
                 asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
@@ -309,14 +232,6 @@ static_assert(BATCH3 == 16 && BATCH == 16, "staging lane r of a half warp stages
 static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
 static_assert(WREG >= 5120, "the tensor-core dense path stages 5 KB");
 
-__device__ __forceinline__ void cp16(void *dst_smem, const void *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_wait_all() {
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
-}
-
 // small tiles (nnz <= small_max): one lane per C nonzero (output-stationary; the paper's sparse
 // accumulator, with each slot owned by one lane).  Entry q of tile t is (r, j): r =
 // the last row whose offset row_ptr_C[r] <= q, j = the (q - row_ptr_C[r])-th set bit of
@@ -348,7 +263,7 @@ __global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
     WorkQueue wq(&P.cnt->q[2][0], ngroups, P.qchunk[2], lane, TS / 32);
     for (int64_t g; wq.next(g, lane);) {
         const int64_t tl = g * 32 + lane;
-        const bool v = tl < P.ntC && !(P.skip && P.skip[tl]);
+        const bool v = tl < P.ntC;
         const int nz = v ? (int)(P.tnzC[tl + 1] - P.tnzC[tl]) : 0;
         const bool small = v && nz < P.dense_threshold && nz <= P.small_max;
         const int mine = small ? nz : 0;
@@ -668,26 +583,6 @@ __device__ __forceinline__ void s3_medium(const StepParams &P, const MedMeta &M,
 // mask_C at the end.  Structurally absent A entries are skipped; absent B entries
 // are staged as 0 so a finite a adds an exact +-0 (value unchanged); a non-finite a falls back to
 // mask-predicated FMAs so Inf*0 never appears.
-// eight consecutive accumulator-type values from shared memory (16-byte vector loads)
-__device__ __forceinline__ void lds8(const double *p, double (&b)[8]) {
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-        const double2 v = reinterpret_cast<const double2 *>(p)[k];
-        b[2 * k] = v.x;
-        b[2 * k + 1] = v.y;
-    }
-}
-__device__ __forceinline__ void lds8(const float *p, float (&b)[8]) {
-#pragma unroll
-    for (int k = 0; k < 2; k++) {
-        const float4 v = reinterpret_cast<const float4 *>(p)[k];
-        b[4 * k] = v.x;
-        b[4 * k + 1] = v.y;
-        b[4 * k + 2] = v.z;
-        b[4 * k + 3] = v.w;
-    }
-}
-
 template <typename TI, typename TO>
 __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigned char *wr, int lane) {
     constexpr int AP = 17;  // padded row pitch of the staged A tile (conflict-free column reads)
@@ -762,105 +657,6 @@ __device__ __forceinline__ void s3_dense(const StepParams &P, int64_t t, unsigne
     __syncwarp();
 }
 
-// dense tile (nnz >= t_nnz), fp64 on the tensor cores (opt-in TSG_DENSE_TC): the warp holds the
-// 16x16 C tile as 2x2 DMMA m8n8k4 accumulator fragments; per pair both tiles are staged densely
-// (zero-filled, A row-major and B transposed, pitch 20 doubles: conflict-free fragment loads) and
-// 4 k-steps x 4 blocks of DMMA.8x8x4 multiply them (16 instructions for the 4096 dense FMAs).
-// The k-chunks of four are summed inside the tensor core, so values agree with the ascending-k
-// FMA order to rounding (the north_star tolerance), not bit for bit; run-to-run deterministic.
-// A pair holding a non-finite value is multiplied entry by entry instead (Inf*0 never appears).
-__device__ __forceinline__ void dmma884(double &d0, double &d1, double a, double b) {
-    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
-                 : "+d"(d0), "+d"(d1)
-                 : "d"(a), "d"(b));
-}
-
-template <typename TI>
-__device__ __forceinline__ void s3_dense_tc(const StepParams &P, int64_t t, unsigned char *wr, int lane) {
-    constexpr int PT = 20;
-    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
-    double *As = reinterpret_cast<double *>(wr);  // [16][PT]: A(r, c) at r*PT + c
-    double *Bt = As + TILE * PT;                  // [16][PT]: B(c, j) at j*PT + c
-    const int g = lane >> 2, tq = lane & 3;
-    double acc[2][2][2];
-#pragma unroll
-    for (int i = 0; i < 8; i++) (&acc[0][0][0])[i] = 0.0;
-    const uint64_t *pp = P.pairs + P.pairBeg[t];
-    const uint32_t np = P.pairCnt[t];
-    for (uint32_t p = 0; p < np; p++) {
-        const uint64_t pr = pp[p];
-        const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-#pragma unroll
-        for (int e = lane; e < 2 * TILE * PT * 8 / 16; e += 32) reinterpret_cast<uint4 *>(As)[e] = make_uint4(0u, 0u, 0u, 0u);
-        __syncwarp();
-        bool nf = false;
-        for (int64_t e = P.tnzA[pA] + lane; e < P.tnzA[pA + 1]; e += 32) {
-            const uint32_t ix = P.ixA[e];
-            const double v = vcvt<double>(vA[e]);
-            nf |= !isfinite(v);
-            As[(ix >> 4) * PT + (ix & 15)] = v;
-        }
-        for (int64_t e = P.tnzB[pB] + lane; e < P.tnzB[pB + 1]; e += 32) {
-            const uint32_t ix = P.ixB[e];
-            const double v = vcvt<double>(vB[e]);
-            nf |= !isfinite(v);
-            Bt[(ix & 15) * PT + (ix >> 4)] = v;
-        }
-        const bool anynf = __any_sync(FULL, nf);
-        __syncwarp();
-        if (!anynf) {
-#pragma unroll
-            for (int ks = 0; ks < 4; ks++) {
-                const double a0 = As[g * PT + 4 * ks + tq], a1 = As[(8 + g) * PT + 4 * ks + tq];
-                const double b0 = Bt[g * PT + 4 * ks + tq], b1 = Bt[(8 + g) * PT + 4 * ks + tq];
-                dmma884(acc[0][0][0], acc[0][0][1], a0, b0);
-                dmma884(acc[0][1][0], acc[0][1][1], a0, b1);
-                dmma884(acc[1][0][0], acc[1][0][1], a1, b0);
-                dmma884(acc[1][1][0], acc[1][1][1], a1, b1);
-            }
-        } else {
-            // entry by entry over the structural intersection (the lane's eight C entries)
-#pragma unroll
-            for (int mi = 0; mi < 2; mi++) {
-                const int r = 8 * mi + g;
-                const uint32_t mAr = P.mA[pA * TILE + r];
-#pragma unroll
-                for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-                    for (int h = 0; h < 2; h++) {
-                        const int j = 8 * ni + 2 * tq + h;
-                        uint32_t x = mAr & P.mTB[pB * TILE + j];
-                        while (x) {
-                            const int c = __ffs(x) - 1;
-                            x &= x - 1;
-                            acc[mi][ni][h] = fma(As[r * PT + c], Bt[j * PT + c], acc[mi][ni][h]);
-                        }
-                    }
-            }
-        }
-        __syncwarp();
-    }
-    double *vC = static_cast<double *>(P.vC);
-#pragma unroll
-    for (int mi = 0; mi < 2; mi++) {
-        const int r = 8 * mi + g;
-        const uint32_t mC = P.mC[t * TILE + r];
-        const int64_t ob = P.tnzC[t] + P.rpC[t * TILE + r];
-#pragma unroll
-        for (int ni = 0; ni < 2; ni++)
-#pragma unroll
-            for (int h = 0; h < 2; h++) {
-                const int j = 8 * ni + 2 * tq + h;
-                if ((mC >> j) & 1u) {
-                    const int q = __popc(mC & ((1u << j) - 1u));
-                    P.ixC[ob + q] = (uint8_t)((r << 4) | j);
-                    vC[ob + q] = acc[mi][ni][h];
-                }
-            }
-    }
-    __syncwarp();
-}
-
 // medium tiles: warps take groups of 32 consecutive C tiles; the group's medium tiles go two at a
 // time, a half warp each.  Register- and shared-memory-lean (no dense code): 7 CTAs per SM.
 template <typename TI, typename TO>
@@ -879,7 +675,6 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
     for (int64_t g; wq.next(g, lane);) {
         unsigned mm = P.medL[g] | P.medH[g];  // the group's medium tiles (step 2 classified them)
         if (!mm) continue;                    // warp-uniform
-        if (P.skip) mm &= ~__ballot_sync(FULL, g * 32 + lane < P.ntC && P.skip[g * 32 + lane]);
         if (lane == 0 && mm) atomicAdd(&P.cnt->n3medium, (u64c)__popc(mm));
         auto pop2 = [&]() {  // next two medium tiles of the group (one per half warp)
             const int f0 = __ffs(mm) - 1;
@@ -922,19 +717,12 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
         const int part = (int)(u - g * split);
         unsigned dm = P.denL[g] | P.denH[g];  // the group's dense tiles (step 2 classified them)
         if (!dm) continue;                    // warp-uniform
-        if (P.skip) dm &= ~__ballot_sync(FULL, g * 32 + lane < P.ntC && P.skip[g * 32 + lane]);
         if (lane == 0 && part == 0 && dm) atomicAdd(&P.cnt->n3dense, (u64c)__popc(dm));
         unsigned dd = dm;
         for (int k = 0; dd; k = k + 1 == split ? 0 : k + 1) {
             const int f = __ffs(dd) - 1;
             dd &= dd - 1;
             if (k != part) continue;
-            if constexpr (sizeof(TO) == 8) {
-                if (P.dense_tc) {
-                    s3_dense_tc<TI>(P, g * 32 + f, wr, lane);
-                    continue;
-                }
-            }
             s3_dense<TI, TO>(P, g * 32 + f, wr, lane);
         }
     }
@@ -952,7 +740,7 @@ struct Shape {
     int chunk;
 };
 template <typename K>
-Shape step_shape(K kernel, int threads, int64_t units, int64_t min_per_warp = 4) {
+Shape step_shape(K kernel, int threads, int64_t units, int qoverride, int64_t min_per_warp = 4) {
     static std::mutex mu;
     static std::map<std::pair<const void *, int>, int> cache;  // (kernel, device) -> resident CTAs per GPU
     const int wpc = threads / 32;
@@ -973,7 +761,7 @@ Shape step_shape(K kernel, int threads, int64_t units, int64_t min_per_warp = 4)
     units = std::max<int64_t>(units, 1);
     const int64_t per_warp = units / ((int64_t)resident * wpc);
     int64_t chunk = per_warp >= min_per_warp ? std::max<int64_t>(1, std::min<int64_t>(8, per_warp / 256)) : 0;
-    if (const char *e = getenv("TSG_QUEUE_CHUNK")) chunk = atoi(e);  // tuning only (0 = static)
+    if (qoverride >= 0) chunk = qoverride;  // TSG_QUEUE_CHUNK_SHIFT (tests of the distribution)
     if (chunk <= 0) return {(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, wpc), 148LL * 32)), 0};
     return {(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, wpc), resident)), (int)chunk};
 }
@@ -984,7 +772,7 @@ void launch_step2(const StepParams &P, cudaStream_t s) {
     if (P.ntC <= 0) return;
     const int64_t groups = (P.ntC + 31) / 32;
     StepParams Q = P;
-    const Shape sl = step_shape(k_s2_light, T2L, groups), sh = step_shape(k_s2, T2, groups);
+    const Shape sl = step_shape(k_s2_light, T2L, groups, P.qoverride), sh = step_shape(k_s2, T2, groups, P.qoverride);
     Q.qchunk[0] = sl.chunk;
     Q.qchunk[1] = sh.chunk;
     TSG_LAUNCH(k_s2_light, sl.grid, T2L, 0, s, Q);
@@ -997,17 +785,17 @@ static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s)
     StepParams Q = P;
     if (P.small_max > 0) {
         if (P.small_stage) {
-            const Shape sp = step_shape(k_s3_small<TI, TO, true>, TS, groups);
+            const Shape sp = step_shape(k_s3_small<TI, TO, true>, TS, groups, P.qoverride);
             Q.qchunk[2] = sp.chunk;
             TSG_LAUNCH((k_s3_small<TI, TO, true>), sp.grid, TS, 0, s, Q);
         } else {
-            const Shape sp = step_shape(k_s3_small<TI, TO, false>, TS, groups);
+            const Shape sp = step_shape(k_s3_small<TI, TO, false>, TS, groups, P.qoverride);
             Q.qchunk[2] = sp.chunk;
             TSG_LAUNCH((k_s3_small<TI, TO, false>), sp.grid, TS, 0, s, Q);
         }
     }
     {
-        const Shape sp = step_shape(k_s3<TI, TO>, T3, groups);
+        const Shape sp = step_shape(k_s3<TI, TO>, T3, groups, P.qoverride);
         Q.qchunk[3] = sp.chunk;
         TSG_LAUNCH((k_s3<TI, TO>), sp.grid, T3, 0, s, Q);
     }
@@ -1015,9 +803,8 @@ static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s)
         // dense tiles per group of 32: spread a group over up to 4 warps when dense tiles are common
         // (measured on C3: 2 / 4 / 8 / 16 / 32 warps -> 0.743 / 0.716 / 0.734 / 0.780 / 0.839 ms)
         int split = (int)std::max<int64_t>(1, std::min<int64_t>(4, 32 * n_dense / (groups * 4)));
-        if (const char *e = getenv("TSG_DENSE_SPLIT")) split = std::max(1, std::min(32, atoi(e)));  // tuning only
         // (dense tiles: static distribution, measured faster on C3)
-        const Shape sp = step_shape(k_s3_dense<TI, TO>, T3, groups * split, INT64_MAX);
+        const Shape sp = step_shape(k_s3_dense<TI, TO>, T3, groups * split, P.qoverride, INT64_MAX);
         Q.qchunk[4] = sp.chunk;
         TSG_LAUNCH((k_s3_dense<TI, TO>), sp.grid, T3, 0, s, Q, split);
     }

@@ -52,7 +52,7 @@ def test_non_compute_entry_points(lib):
     lib.tsg_status_string.restype = C.c_char_p
     assert lib.tsg_status_string(0) == b"TSG_OK"
     assert lib.tsg_status_string(5) == b"TSG_ERR_OOM"
-    assert lib.tsg_abi_version() == 2
+    assert lib.tsg_abi_version() == 3
     lib.tsg_last_error.restype = C.c_char_p
     assert isinstance(lib.tsg_last_error(), bytes)
 

@@ -132,10 +132,15 @@ def pair_cases():
 PAIRS = pair_cases()
 
 
+@pytest.mark.parametrize("mode", ["default", "per-tile", "rows"])
 @pytest.mark.parametrize("name,A,B", PAIRS, ids=[p[0] for p in PAIRS])
-def test_spgemm_matches_oracle(tsg, name, A, B):
+def test_spgemm_matches_oracle(tsg, name, A, B, mode):
+    """Both pipelines against the oracle: the default dispatch, the per-C-tile pipeline forced with
+    path_general, and the row path forced wherever every tile row of A is narrow (path_rows)."""
     TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
-    C = tsg.spgemm(TA, TB, stats=True, products=True)
+    general = mode == "per-tile"
+    C = tsg.spgemm(TA, TB, stats=True, products=True, structural=True, path_general=general,
+                   path_rows=mode == "rows")
     ref = oracle.expected_tiles(A, B)
     ref_fma = oracle.expected_tiles(A, B, fma=True)
     got = host(C)
@@ -150,6 +155,9 @@ def test_spgemm_matches_oracle(tsg, name, A, B):
     assert st["pairs"] == d["pairs"]
     assert st["products"] == d["products"]
     assert st["tiles_dense"] == int((np.diff(ref.tile_nnz) >= tsg.DENSE_NNZ).sum())
+    # |C'| of the paper's step 1, empty tiles included, against the oracle's O4
+    assert st["tiles_structural"] == d["tiles_structural"] >= st["tiles_c"]
+    assert st["path"] == (0 if general else st["path"])
     # CSR assembly of the result
     rp, ci, v = tsg.tiles_to_csr(C)
     O = oracle.spgemm(A, B, fma=True)
@@ -163,10 +171,13 @@ def _abs_csr(A, B):
 
 
 @pytest.mark.parametrize("opts", [dict(scan_only=True), dict(list_always=True), dict(dense_threshold=1),
-                                  dict(dense_threshold=257), dict(dense_threshold=100), dict(step3_rows=True),
-                                  dict(step3_rows=True, dense_threshold=1), dict(sort_only=True),
-                                  dict(sort_only=True, list_always=True), dict(sort_only=True, scan_only=True),
-                                  dict(small_stage=True), dict(small_stage=False)])
+                                  dict(dense_threshold=257), dict(dense_threshold=100), dict(path_general=True),
+                                  dict(path_general=True, dense_threshold=1), dict(list_always=True, dense_threshold=1),
+                                  dict(path_rows=True), dict(path_rows=True, dense_threshold=1),
+                                  dict(path_rows=True, list_always=True),
+                                  dict(sort_only=True), dict(sort_only=True, list_always=True),
+                                  dict(sort_only=True, scan_only=True), dict(small_stage=True, path_general=True),
+                                  dict(small_stage=False, path_general=True)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
     for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12),
@@ -195,20 +206,27 @@ def test_step1_merge_coverage(tsg):
         assert_tiles_equal(host(C), oracle.expected_tiles(A, A, fma=True))
 
 
-def test_step3_row_kernel_coverage(tsg):
-    """Stencil/FEM tile rows go through the whole-row kernel; hub rows fall back per tile."""
-    for A, allrows in ((gen.stencil27(12), True), (gen.strip_fem(6, 20, 6), True),
-                       (gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004), False)):
+def test_row_path_coverage(tsg):
+    """Narrow inputs (every tile row <= 32 A tiles: stencil, FEM, C1) that are small or dense-tiled
+    take the fused per-tile-row pipeline with 2 blocking reads; inputs with a wide tile row take the
+    per-C-tile pipeline (3); path_general forces the latter, path_rows the former where possible.
+    Same C bit for bit either way."""
+    hub = gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)
+    for A, narrow in ((gen.stencil27(12), True), (gen.strip_fem(6, 20, 6), True), (gen.config("C1"), True),
+                      (hub, False)):
         T = tiles_of(tsg, A)
-        C = tsg.spgemm(T, T, stats=True, step3_rows=True)
+        C = tsg.spgemm(T, T, stats=True)
         st = C.stats
-        if allrows:
-            assert st["step3_row_tiles"] == C.num_tiles and st["step3_rows"] > 0
-        else:
-            assert st["step3_row_tiles"] < C.num_tiles
+        assert st["path"] == (1 if narrow else 0)
+        assert st["host_syncs"] == (2 if narrow else 3)
+        G = tsg.spgemm(T, T, stats=True, path_general=True)
+        assert G.stats["path"] == 0 and G.stats["host_syncs"] == 3
+        R = tsg.spgemm(T, T, stats=True, path_rows=True)
+        assert R.stats["path"] == (1 if narrow else 0)
         ref = oracle.expected_tiles(A, A, fma=True)
         assert_tiles_equal(host(C), ref)
-        assert tsg.spgemm(T, T, stats=True).stats["step3_row_tiles"] == 0
+        assert_tiles_equal(host(G), ref)
+        assert_tiles_equal(host(R), ref)
 
 
 @pytest.mark.parametrize("th", [None, 192])
@@ -294,7 +312,7 @@ def test_launch_counter_advances(tsg):
     n0 = tsg.kernel_launch_count()
     C = tsg.spgemm(T, T, stats=True)
     assert tsg.kernel_launch_count() - n0 == C.stats["kernel_launches"] > 5
-    assert C.stats["host_syncs"] == 3
+    assert C.stats["host_syncs"] == 2  # the row path: after the plan, and C's sizes after steps 1-2
 
 
 # ------------------------------------------------------------------------------------------
@@ -307,13 +325,15 @@ CLOSED = {  # SURVEY §8(c) closed forms (structure and counts are value indepen
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
-def test_full_size_sampled_rows(tsg, cfg):
+@pytest.mark.parametrize("cfg,opts", [("C2", {}), ("C2", dict(path_rows=True)), ("C3", {}),
+                                      ("C3", dict(path_general=True)), ("C4", {})],
+                         ids=["C2", "C2-rows", "C3", "C3-per-tile", "C4"])
+def test_full_size_sampled_rows(tsg, cfg, opts):
     import torch
 
     A = gen.config(cfg)
     T = tiles_of(tsg, A)
-    C = tsg.spgemm(T, T, stats=True, products=True)
+    C = tsg.spgemm(T, T, stats=True, products=True, **opts)
     st = C.stats
     if cfg in CLOSED:
         assert st["nnz_c"] == CLOSED[cfg]["nnz_c"] and st["products"] == CLOSED[cfg]["products"]
@@ -489,39 +509,6 @@ def test_mixed_precision_inputs_rejected(tsg):
     assert e.value.name == "TSG_ERR_INVALID_ARG"
 
 
-@pytest.mark.parametrize("name,A,B", [(n, a, b) for n, a, b in PAIRS if n in
-                                      ("C1", "strip-fem-8x30", "dense-64", "rmat-12", "rect", "hub")],
-                         ids=["C1", "strip-fem-8x30", "dense-64", "rmat-12", "rect", "hub"])
-def test_dense_tensor_core_variant(tsg, name, A, B):
-    """TSG_DENSE_TC: fp64 dense tiles on DMMA 8x8x4.  Structure bit-exact, values within the
-    north_star tolerance of the oracle (the tensor core sums k in chunks of four), deterministic."""
-    TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
-    ref = oracle.expected_tiles(A, B)
-    absref = oracle.csr_to_tiles(_abs_csr(A, B)).val
-    for th in (None, 1):
-        C = tsg.spgemm(TA, TB, dense_tc=True, dense_threshold=th)
-        got = host(C)
-        assert_tiles_equal(got, ref, values=None)
-        assert_values_close(got["val"], ref.val, absref)
-        again = host(tsg.spgemm(TA, TB, dense_tc=True, dense_threshold=th))
-        assert np.array_equal(got["val"].view(np.int64), again["val"].view(np.int64))
-
-
-def test_dense_tensor_core_nonfinite(tsg):
-    """A pair holding Inf/NaN is multiplied entry by entry: Inf*0 never appears."""
-    A = gen.dense_block(16, 16)
-    A.val[5] = np.inf
-    A.val[40] = np.nan
-    B = gen.random_sparse(16, 16, 0.5, 3)
-    for a, b in ((A, B), (B, A), (A, A)):
-        C = tsg.spgemm(tiles_of(tsg, a), tiles_of(tsg, b), dense_threshold=1, dense_tc=True)
-        ref = oracle.expected_tiles(a, b, fma=True)
-        got = host(C)
-        assert_tiles_equal(got, ref, values=None)
-        absref = oracle.csr_to_tiles(_abs_csr(a, b)).val
-        assert_values_close(got["val"], ref.val, absref)
-
-
 def test_copy_to_host_async_pipeline(tsg):
     """tsg_tiles_copy_to_host_async on a second stream, overlapping the next block's SpGEMM (the
     bench's e2e leg): every block's host copy equals the oracle's tiles of that row block."""
@@ -568,22 +555,76 @@ def test_copy_to_host_async_pipeline(tsg):
     assert bitwise_equal_values(np.concatenate(vals), ref.val)
 
 
-@pytest.mark.parametrize("chunk", ["0", "1", "3"])
-def test_work_distribution_gives_identical_results(tsg, chunk, monkeypatch):
-    """Step-2/3 work distribution: static grid-stride (0) or the work queue with 1 or 3 groups per
-    request (TSG_QUEUE_CHUNK, read at launch; small test inputs otherwise take the static path)."""
+@pytest.mark.parametrize("chunk", [0, 1, 3])
+def test_work_distribution_gives_identical_results(tsg, chunk):
+    """Per-C-tile pipeline work distribution: static grid-stride (0) or the work queue with 1 or 3
+    groups per request (small test inputs otherwise take the static path)."""
     cases = (gen.stencil27(12), gen.strip_fem(6, 20, 6), gen.rmat(11),
              gen.hub(8192, hub_rows=(0, 5000), hub_cols=(), density=0.002))
-    base = []
     for A in cases:
         T = tiles_of(tsg, A)
-        base.append(host(tsg.spgemm(T, T)))
-    monkeypatch.setenv("TSG_QUEUE_CHUNK", chunk)
-    for A, b in zip(cases, base):
-        T = tiles_of(tsg, A)
-        got = host(tsg.spgemm(T, T))
+        b = host(tsg.spgemm(T, T))
+        got = host(tsg.spgemm(T, T, path_general=True, queue_chunk=chunk))
         for k in ARRAYS[:-1]:
             assert np.array_equal(got[k], b[k]), (chunk, k)
         assert bitwise_equal_values(got["val"], b["val"])
     A = cases[0]
-    assert_tiles_equal(host(tsg.spgemm(tiles_of(tsg, A), tiles_of(tsg, A))), oracle.expected_tiles(A, A, fma=True))
+    assert_tiles_equal(host(tsg.spgemm(tiles_of(tsg, A), tiles_of(tsg, A), path_general=True, queue_chunk=chunk)),
+                       oracle.expected_tiles(A, A, fma=True))
+
+
+def test_unknown_flags_rejected(tsg):
+    import ctypes as C
+
+    from paper_conf_ppopp_niuljs0022_b200 import _lib
+
+    A = gen.config("C1")
+    T = tiles_of(tsg, A)
+    out = C.c_void_p()
+    for bad in (0x80, 0x800, 1 << 29):  # 0x80: the removed tensor-core flag
+        rc = _lib.load().tsg_spgemm(T.ptr, T.ptr, bad, None, None, C.byref(out), None)
+        assert rc == 1 and out.value is None
+
+
+def test_host_input_dtypes_and_row_ptr_validation(tsg):
+    """Host CSR given as torch CPU tensors of the wrong integer width is converted; an
+    unsupported value type raises; TSG_VALIDATE rejects row_ptr[m] != nnz with INVALID_ARG."""
+    import torch
+
+    A = gen.random_sparse(100, 90, 0.05, 7)
+    ref = oracle.csr_to_tiles(A)
+    T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).to(torch.int32), torch.from_numpy(A.col).to(torch.int64),
+                         torch.from_numpy(A.val), (A.m, A.n))
+    assert_tiles_equal(host(T), ref)
+    with pytest.raises(TypeError):
+        tsg.csr_to_tiles(A.rowptr, A.col, A.val.astype(np.complex128), (A.m, A.n))
+    with pytest.raises(ValueError):
+        tsg.csr_to_tiles(A.rowptr[:-1], A.col, A.val, (A.m, A.n))
+    # device input: row_ptr[m] larger than the column array
+    rp = torch.from_numpy(A.rowptr).cuda()
+    rp[-1] += 5
+    with pytest.raises(tsg.TsgError) as e:
+        tsg.csr_to_tiles(rp, torch.from_numpy(A.col).cuda(), torch.from_numpy(A.val).cuda(), (A.m, A.n),
+                         validate=True)
+    assert e.value.name == "TSG_ERR_INVALID_ARG"
+
+
+def test_free_is_ordered_on_the_producing_stream(tsg):
+    """A handle made under a side stream frees its arrays on that stream: dropping C
+    right after the call must not let the next allocation overwrite it while step 3 still runs."""
+    import torch
+
+    A = gen.stencil27(16)
+    T = tiles_of(tsg, A)
+    ref = host(tsg.spgemm(T, T))
+    s = torch.cuda.Stream()
+    for _ in range(3):
+        with torch.cuda.stream(s):
+            C = tsg.spgemm(T, T)
+            assert C.handle.stream == s.cuda_stream
+            del C
+            D = tsg.spgemm(T, T)
+        s.synchronize()
+        got = host(D)
+        for k in ARRAYS:
+            assert np.array_equal(got[k], ref[k]), k
