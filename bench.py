@@ -271,10 +271,14 @@ def main():
     Bcsr = _csr_transpose(A) if args.aat else A
     # shard C tile rows across ranks (strong scaling of one matrix), and within a
     # rank optionally into row blocks computed one after the other (C does not fit otherwise)
-    K = args.row_blocks or max(1, ROW_BLOCKS.get(args.config, 1) // world)
+    # row blocks per rank: a config whose C does not fit one GPU in one call (C5) is computed in
+    # blocks; ranks sharing a GPU (functional multi-rank runs on one box) share its memory too
+    ranks_per_gpu = -(-world // max(1, torch.cuda.device_count()))
+    K = args.row_blocks or max(1, -(-ROW_BLOCKS.get(args.config, 1) * ranks_per_gpu // world))
     from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
 
-    cuts = tdist.partition_tile_rows(A, Bcsr, world * K) if world * K > 1 else np.array([0, T.tile_m])
+    # product-balanced cuts computed by the library on the device (tsg_partition_tile_rows)
+    cuts = tdist.partition_device(T, Bt, world * K)
     blocks = [(int(cuts[rank * K + b]), int(cuts[rank * K + b + 1])) for b in range(K)]
     I0, I1 = blocks[0][0], blocks[-1][1]
     shards = [tsg.slice_rows(T, b0, b1) if (b0, b1) != (0, T.tile_m) else T for b0, b1 in blocks]
@@ -372,16 +376,30 @@ def main():
                 ts.append(float(t.item()))
             return float(np.median(ts))
 
-        meta = (T.m, T.n, T.num_tiles, T.nnz)
+        meta = (Bt.m, Bt.n, Bt.num_tiles, Bt.nnz, Bt.val.dtype)
         t_b = timed(lambda: tdist.broadcast_tiles(Bt.arrays() if rank == 0 else None, meta if rank == 0 else None,
                                                   0, dev))
-        t_r = None
+        # reassembly: count-exact gatherv of the C shards to rank 0 when the full C fits there
+        # (next to the step, not in the metric); otherwise C stays distributed (C5: ~144 GB)
+        t_r, where = None, "left distributed (each rank owns its tile rows)"
         if K == 1:
             Cl = tsg.spgemm(shards[0], Bt)
-            t_r = timed(lambda: tdist.allgatherv_tiles(Cl), reps=2)
+            cb = torch.tensor([sum(v.numel() * v.element_size() for v in Cl.arrays().values())], dtype=torch.int64,
+                              device=dev)
+            dist.all_reduce(cb)
+            free = torch.tensor([torch.cuda.mem_get_info(dev)[0] // ranks_per_gpu], dtype=torch.int64, device=dev)
+            dist.all_reduce(free, op=dist.ReduceOp.MIN)
+            if int(cb.item()) < 0.6 * int(free.item()):
+                t_r = timed(lambda: tdist.gatherv_tiles(Cl, 0), reps=2)
+                where = f"gatherv to rank 0 ({int(cb.item()) / 1e9:.2f} GB, count-exact point-to-point)"
+            else:
+                where = (f"left distributed: C is {int(cb.item()) / 1e9:.1f} GB, more than 60% of a rank's free "
+                         "device memory")
             del Cl
         multi = {"t_bcast_ms": t_b, "bcast_bytes": int(sum(v.numel() * v.element_size() for v in Bt.arrays().values())),
-                 "t_reassemble_ms": t_r, "backend": os.environ.get("TSG_DIST_BACKEND", "nccl"),
+                 "t_reassemble_ms": t_r, "reassembly": where, "partition": "device (tsg_partition_tile_rows)",
+                 "row_blocks_per_rank": K, "ranks_per_gpu": ranks_per_gpu,
+                 "backend": os.environ.get("TSG_DIST_BACKEND", "nccl"),
                  "note": "not in the metric: B resident, C left sharded (SURVEY 8(e))"}
 
     # roofline of the dominant kernel (step 3 numeric unless another step is longer)
@@ -420,7 +438,7 @@ def main():
         h_ci = torch.from_numpy(A.col).pin_memory()
         h_v = torch.from_numpy(A.val).pin_memory()
         Ke = K if K > 1 else E2E_BLOCKS
-        ecuts = tdist.partition_tile_rows(A, Bcsr, world * Ke) if world * Ke > 1 else np.array([0, T.tile_m])
+        ecuts = tdist.partition_device(T, Bt, world * Ke)
         eblocks = [(int(ecuts[rank * Ke + b]), int(ecuts[rank * Ke + b + 1])) for b in range(Ke)]
         bsizes, bo = [], 0
         for b0, b1 in eblocks:

@@ -220,6 +220,23 @@ TSG_API tsg_status tsg_tiles_to_csr(const tsg_tiles *T, const tsg_allocator *al,
  */
 TSG_API tsg_status tsg_tiles_transpose(const tsg_tiles *T, const tsg_allocator *al, void *stream, tsg_tiles **out);
 
+/*
+ * tsg_partition_tile_rows -- product-balanced split of C's tile rows for the multi-GPU path
+ * (the paper itself runs on one GPU).  Computes on the device the
+ * intermediate products of every tile row of A*B (Table 2's "products") and cuts
+ * [0, tile_m) into `parts` contiguous ranges at equal shares of their prefix sum: cuts[g] is the
+ * first tile row whose prefix reaches g * total / parts (monotone; cuts[0] = 0, cuts[parts] =
+ * A.tile_m).  Rank g then computes C's tile rows [cuts[g], cuts[g+1]) from
+ * tsg_tiles_slice_rows(A, cuts[g], cuts[g+1]) and all of B.
+ *   A, B      the operands (device handles; A.n == B.m)
+ *   parts     1..500
+ *   cuts      HOST array of parts + 1 int64 (written)
+ *   products  optional HOST int64: the total intermediate products of A*B
+ * Syncs: one blocking read (the cuts).  Errors: INVALID_ARG, SHAPE, OOM, CUDA.
+ */
+TSG_API tsg_status tsg_partition_tile_rows(const tsg_tiles *A, const tsg_tiles *B, int64_t parts, void *stream,
+                                           int64_t *cuts, int64_t *products);
+
 /* Fill *out with the handle's arrays and sizes (pointers stay owned by the handle). */
 TSG_API tsg_status tsg_tiles_get_view(const tsg_tiles *T, tsg_tiles_view *out);
 

@@ -23,7 +23,7 @@ from . import _lib
 from ._lib import TILE, DENSE_NNZ, TsgError  # noqa: F401
 
 __all__ = ["Tiles", "csr_to_tiles", "spgemm", "tiles_to_csr", "slice_rows", "wrap", "TsgError",
-           "kernel_launch_count", "workspace_release", "transpose"]
+           "kernel_launch_count", "workspace_release", "transpose", "partition_tile_rows"]
 
 _DT = {"int64": ("<i8", 8), "int32": ("<i4", 4), "uint8": ("|u1", 1), "uint16": ("<u2", 2), "float64": ("<f8", 8),
        "float32": ("<f4", 4), "float16": ("<f2", 2)}
@@ -341,6 +341,16 @@ def wrap(m: int, n: int, arrays: dict, keepalive=None) -> Tiles:
     T = _from_handle(out.value)
     T.handle.keep = (arrays, keepalive)
     return T
+
+
+def partition_tile_rows(A: Tiles, B: Tiles, parts: int, stream=None):
+    """Product-balanced cuts of C's tile rows for ``parts`` ranks, computed on the device
+    (tsg_partition_tile_rows).  Returns (cuts: numpy int64 [parts + 1], products)."""
+    cuts = np.zeros(int(parts) + 1, dtype=np.int64)
+    tot = C.c_int64()
+    _lib.check(_lib.load().tsg_partition_tile_rows(A.ptr, B.ptr, int(parts), C.c_void_p(_stream_ptr(stream)),
+                                                   C.c_void_p(cuts.ctypes.data), C.byref(tot)))
+    return cuts, int(tot.value)
 
 
 def kernel_launch_count() -> int:

@@ -74,7 +74,7 @@ class Allocator(C.Structure):
 SYMBOLS = ["tsg_csr_to_tiles", "tsg_csr_to_tiles_typed", "tsg_spgemm", "tsg_tiles_to_csr", "tsg_tiles_get_view", "tsg_tiles_wrap",
            "tsg_tiles_slice_rows", "tsg_tiles_copy_to_host", "tsg_tiles_copy_to_host_async", "tsg_tiles_destroy", "tsg_free",
            "tsg_status_string", "tsg_last_error", "tsg_abi_version", "tsg_kernel_launch_count",
-           "tsg_workspace_release", "tsg_tiles_transpose"]
+           "tsg_workspace_release", "tsg_tiles_transpose", "tsg_partition_tile_rows"]
 
 _lib = None
 
@@ -120,6 +120,8 @@ def load():
     L.tsg_kernel_launch_count.restype = i64
     L.tsg_tiles_transpose.restype = C.c_int
     L.tsg_tiles_transpose.argtypes = [vp, vp, vp, pp]
+    L.tsg_partition_tile_rows.restype = C.c_int
+    L.tsg_partition_tile_rows.argtypes = [vp, vp, i64, vp, vp, C.POINTER(i64)]
     L.tsg_workspace_release.restype = C.c_size_t
     L.tsg_workspace_release.argtypes = [vp]
     _lib = L

@@ -4,7 +4,7 @@
 #include <chrono>
 #include <cstring>
 
-#include "tsg_internal.cuh"
+#include "tsg_kernels.cuh"
 
 namespace tsg {
 
@@ -298,6 +298,27 @@ tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, co
             throw;
         }
         *C = T;
+    });
+}
+
+tsg_status tsg_partition_tile_rows(const tsg_tiles *A, const tsg_tiles *B, int64_t parts, void *stream,
+                                   int64_t *cuts, int64_t *products) {
+    return guarded([&] {
+        TSG_REQUIRE(A && B && cuts, TSG_ERR_INVALID_ARG, "NULL argument");
+        TSG_REQUIRE(parts >= 1 && parts <= 500, TSG_ERR_INVALID_ARG, "parts must be in [1, 500]");
+        TSG_REQUIRE(A->tn == B->tm, TSG_ERR_SHAPE, "tile shapes disagree");
+        cudaStream_t s = (cudaStream_t)stream;
+        Buffers tmp(Allocator{}, s, true);
+        int32_t *rnnz = tmp.get<int32_t>(TILE * B->tm);
+        int64_t *w = tmp.get<int64_t>(A->tm);
+        int64_t *pre = tmp.get<int64_t>(A->tm + 1);
+        int64_t *dcuts = tmp.get<int64_t>(parts + 1);
+        launch_row_products(A->tm, A->tile_ptr, A->tile_col, A->mask, B->tm, B->tile_ptr, B->mask, rnnz, w, s);
+        exclusive_scan<int64_t>(w, pre, A->tm, s, tmp);
+        launch_cuts(pre, A->tm, parts, dcuts, s);
+        int64_t tot = 0;
+        read_device({{cuts, dcuts, sizeof(int64_t) * (size_t)(parts + 1)}, {&tot, pre + A->tm, sizeof(int64_t)}}, s);
+        if (products) *products = tot;
     });
 }
 

@@ -142,6 +142,9 @@ void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, co
 void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
                      cudaStream_t s);
 void launch_sym_rows(const S1Params &P, int64_t tm, cudaStream_t s);
+void launch_row_products(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const uint16_t *maskA, int64_t tmB,
+                         const int64_t *tpB, const uint16_t *maskB, int32_t *rnnz, int64_t *w, cudaStream_t s);
+void launch_cuts(const int64_t *pre, int64_t tm, int64_t parts, int64_t *cuts, cudaStream_t s);
 bool launch_structural(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const int64_t *tpB, const int32_t *tcB,
                        int64_t tnB, DevCounters *cnt, cudaStream_t s);
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s);

@@ -123,6 +123,53 @@ __global__ void __launch_bounds__(256) k_structural(const int64_t *__restrict__ 
 }
 
 // ------------------------------------------------------------------------------------------
+// multi-GPU partition: intermediate products per tile row of A*B -- a warp per
+// tile row, lane = one A tile, sum over its nonzeros (r,c) of nnz(B row 16K + c) -- and the cuts
+// at equal shares of their prefix sum (searchsorted-left of g*total/parts, monotone)
+// ------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_row_products(int64_t tmA, const int64_t *__restrict__ tpA,
+                                                     const int32_t *__restrict__ tcA, const uint16_t *__restrict__ maskA,
+                                                     const int32_t *__restrict__ rnnz, int64_t *__restrict__ w) {
+    const int lane = threadIdx.x & 31;
+    const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (I >= tmA) return;
+    int64_t p = 0;
+    for (int64_t t = tpA[I] + lane; t < tpA[I + 1]; t += 32) {
+        const int64_t K = tcA[t];
+        for (int r = 0; r < TILE; r++) {
+            uint32_t m = maskA[t * TILE + r];
+            while (m) {
+                const int c = __ffs(m) - 1;
+                m &= m - 1;
+                p += rnnz[K * TILE + c];
+            }
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(FULL, p, o);
+    if (lane == 0) w[I] = p;
+}
+
+__global__ void k_cuts(const int64_t *__restrict__ pre, int64_t tm, int64_t parts, int64_t *__restrict__ cuts) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const int64_t total = pre[tm];
+    int64_t prev = 0;
+    cuts[0] = 0;
+    for (int64_t g = 1; g < parts; g++) {
+        // first i with pre[i] >= g * total / parts, i.e. pre[i] * parts >= g * total (exact)
+        int64_t lo = 0, hi = tm;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if ((__int128)pre[mid] * parts >= (__int128)g * total) hi = mid;
+            else lo = mid + 1;
+        }
+        prev = max(prev, lo);
+        cuts[g] = prev;
+    }
+    cuts[parts] = tm;
+}
+
+// ------------------------------------------------------------------------------------------
 // a1 (plan): per A tile, how its candidate B tiles are enumerated.
 //   scan mode: every tile of B tile row K (filtered later by occupancy);
 //   list mode: when A_IK touches a single column c, exactly the B row list of k = 16K + c
@@ -1078,6 +1125,16 @@ void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint1
 void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
                     uint32_t *list, cudaStream_t s) {
     TSG_LAUNCH(k_rowlist, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, lptr, lcnt, list);
+}
+
+void launch_row_products(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const uint16_t *maskA, int64_t tmB,
+                         const int64_t *tpB, const uint16_t *maskB, int32_t *rnnz, int64_t *w, cudaStream_t s) {
+    TSG_LAUNCH(k_brow_nnz, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, rnnz);
+    TSG_LAUNCH(k_row_products, grid_for(tmA, 8), 256, 0, s, tmA, tpA, tcA, maskA, (const int32_t *)rnnz, w);
+}
+
+void launch_cuts(const int64_t *pre, int64_t tm, int64_t parts, int64_t *cuts, cudaStream_t s) {
+    TSG_LAUNCH(k_cuts, 1, 32, 0, s, pre, tm, parts, cuts);
 }
 
 void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int64_t ntA, const int32_t *tcA,

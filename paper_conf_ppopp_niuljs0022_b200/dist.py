@@ -3,18 +3,22 @@ which runs on one GPU -- P:3760-3766 calls distributed blocking SpGEMM related w
 
 C tile rows are independent: tile row I of C needs tile row I of A and all of B.  So
 
-1. ``partition_tile_rows``: contiguous tile-row ranges [I_g, I_{g+1}) cut at equal shares of the
-   prefix sum of per-tile-row intermediate products (load balance by work, not rows);
+1. ``partition_device`` (tsg_partition_tile_rows in the library): contiguous tile-row ranges
+   [I_g, I_{g+1}) cut on the device at equal shares of the prefix sum of per-tile-row
+   intermediate products (load balance by work, not rows); ``partition_tile_rows`` is the same
+   rule from host CSR (used to check the device cuts);
 2. ``broadcast_tiles``: rank ``src`` holds B; its seven Section-3.2 arrays go to every rank with
    ``torch.distributed.broadcast`` (NCCL over NVLink on the B200 box);
 3. each rank runs the local ``tsg.spgemm(slice_rows(A, I_g, I_{g+1}), B)``;
-4. ``allgatherv_tiles``: the per-rank C shards are gathered (uneven all_gather, padded) and the
-   ``tile_ptr`` / ``tile_nnz`` offsets rebased by the exclusive scan of the per-rank counts
-   (``assemble``), giving every rank the full C.
+4. reassembly, count-exact (no padding): ``gatherv_tiles`` sends every shard to one rank with
+   point-to-point transfers of exactly its bytes; ``allgatherv_tiles`` gives every rank the full C
+   with one exact-size broadcast per source.  ``assemble`` rebases ``tile_ptr`` / ``tile_nnz`` by
+   the exclusive scan of the per-rank tile and nonzero counts.  When the full C does not fit one
+   GPU (C5: ~144 GB in tile form) it is left distributed -- every rank owns its tile rows.
 
 Only collectives and host bookkeeping live here; every arithmetic step of the method runs in
-libtsg's kernels.  ``assemble`` and the collectives are device-agnostic (torch tensors), so the
-world_size-2 gloo tests in tests/test_dist_gloo.py cover them on CPU.
+libtsg's kernels.  The collectives are device-agnostic (torch tensors), so the world_size-2 gloo
+tests in tests/test_dist_gloo.py cover them on CPU.
 """
 from __future__ import annotations
 
@@ -22,6 +26,7 @@ import numpy as np
 
 TILE = 16
 ARRAYS = ("tile_ptr", "tile_col", "tile_nnz", "row_ptr", "mask", "idx", "val")
+_CODES = ("float64", "float32", "float16")
 
 
 def tile_row_products(A, B) -> np.ndarray:
@@ -36,18 +41,34 @@ def tile_row_products(A, B) -> np.ndarray:
     return pad.reshape(tm, TILE).sum(axis=1)
 
 
-def partition_tile_rows(A, B, world: int) -> np.ndarray:
-    """cuts[g] .. cuts[g+1] = tile rows of rank g; equal shares of the product prefix sum."""
-    w = tile_row_products(A, B)
+def cuts_from_weights(w: np.ndarray, world: int) -> np.ndarray:
+    """cuts[g] = first tile row whose product prefix reaches g * total / world (monotone)."""
     tm = w.size
     if world <= 1 or tm == 0:
         return np.array([0, tm] if world <= 1 else [0] * world + [tm], dtype=np.int64)
-    pre = np.concatenate(([0], np.cumsum(w)))
-    total = pre[-1]
-    targets = (np.arange(1, world) * total) / world
-    inner = np.searchsorted(pre, targets, side="left")
-    cuts = np.concatenate(([0], np.clip(inner, 0, tm), [tm])).astype(np.int64)
-    return np.maximum.accumulate(cuts)
+    pre = np.concatenate(([0], np.cumsum(w))).astype(np.int64)
+    total = int(pre[-1])
+    # exact integer form of searchsorted-left of g*total/world: first i with pre[i]*world >= g*total
+    cuts = [0]
+    for g in range(1, world):
+        cuts.append(int(np.searchsorted(pre * world, g * total, side="left")))
+    cuts.append(tm)
+    return np.maximum.accumulate(np.clip(np.array(cuts, dtype=np.int64), 0, tm))
+
+
+def partition_tile_rows(A, B, world: int) -> np.ndarray:
+    """Host-CSR form of the partition (cuts[g] .. cuts[g+1] = tile rows of rank g)."""
+    return cuts_from_weights(tile_row_products(A, B), world)
+
+
+def partition_device(A_tiles, B_tiles, world: int, stream=None) -> np.ndarray:
+    """The partition computed by the library on the device from the tile handles (no host CSR
+    needed, e.g. for a chained C = (A^2) A whose left operand only exists in tile form)."""
+    from . import partition_tile_rows as _dev
+
+    if world <= 1:
+        return np.array([0, A_tiles.tile_m], dtype=np.int64)
+    return _dev(A_tiles, B_tiles, world, stream)[0]
 
 
 def _wire(t):
@@ -57,17 +78,31 @@ def _wire(t):
     return t.view(torch.uint8) if t.dtype in (torch.uint16, torch.int16) else t
 
 
+def _unwire(t, k):
+    import torch
+
+    return t.view(torch.uint16) if k == "mask" else t
+
+
+def _shapes(m, nt, nnz, vdt):
+    import torch
+
+    tm = (m + TILE - 1) // TILE
+    return {"tile_ptr": (tm + 1, torch.int64), "tile_col": (nt, torch.int32), "tile_nnz": (nt + 1, torch.int64),
+            "row_ptr": (16 * nt, torch.uint8), "mask": (32 * nt, torch.uint8), "idx": (nnz, torch.uint8),
+            "val": (nnz, vdt)}
+
+
 def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, group=None):
     """Broadcast the seven arrays of a tile matrix from ``src``; returns (meta, arrays) everywhere.
 
-    meta = (m, n, num_tiles, nnz) for fp64 values, or (m, n, num_tiles, nnz, dtype) with dtype a
-    torch value type (f3).  On non-src ranks pass arrays=None, meta=None; they receive the 4-tuple
-    for fp64 and the 5-tuple otherwise.
+    meta = (m, n, num_tiles, nnz, dtype) with dtype a torch value type (a 4-tuple means fp64).  On
+    non-src ranks pass arrays=None, meta=None; every rank gets the 5-tuple back.
     """
     import torch
     import torch.distributed as dist
 
-    codes = [torch.float64, torch.float32, torch.float16]
+    codes = [getattr(torch, c) for c in _CODES]
     if meta is not None:
         vals = list(meta[:4]) + [codes.index(meta[4]) if len(meta) > 4 else 0]
     else:
@@ -75,10 +110,7 @@ def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, g
     mt = torch.tensor(vals, dtype=torch.int64, device=device)
     dist.broadcast(mt, src, group=group)
     m, n, nt, nnz, dc = (int(x) for x in mt.tolist())
-    tm = (m + TILE - 1) // TILE
-    shapes = {"tile_ptr": (tm + 1, torch.int64), "tile_col": (nt, torch.int32), "tile_nnz": (nt + 1, torch.int64),
-              "row_ptr": (16 * nt, torch.uint8), "mask": (32 * nt, torch.uint8), "idx": (nnz, torch.uint8),
-              "val": (nnz, codes[dc])}
+    shapes = _shapes(m, nt, nnz, codes[dc])
     out = {}
     for k in ARRAYS:
         if arrays is not None:
@@ -87,32 +119,50 @@ def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, g
             t = torch.empty(shapes[k][0], dtype=shapes[k][1], device=device)
         if t.numel():
             dist.broadcast(t, src, group=group)
-        out[k] = t.view(torch.uint16) if k == "mask" else t
-    return ((m, n, nt, nnz) if dc == 0 else (m, n, nt, nnz, codes[dc])), out
+        out[k] = _unwire(t, k)
+    return (m, n, nt, nnz, codes[dc]), out
 
 
-def allgatherv(t, group=None):
-    """Uneven all_gather of a 1-D tensor: returns the list of every rank's tensor."""
+def _local(C):
+    arrays = C.arrays() if hasattr(C, "arrays") else {k: C[k] for k in ARRAYS}
+    m_local = C.m if hasattr(C, "m") else C["m"]
+    n = C.n if hasattr(C, "n") else C["n"]
+    return arrays, int(m_local), int(n)
+
+
+def _counts(arrays, m_local, group):
+    """(m, num_tiles, nnz, value dtype code) of every rank: one all_gather of 4 int64."""
     import torch
     import torch.distributed as dist
 
+    dev = arrays["tile_ptr"].device
+    vdt = str(arrays["val"].dtype).replace("torch.", "")
+    mine = torch.tensor([m_local, arrays["tile_col"].numel(), arrays["val"].numel(), _CODES.index(vdt)],
+                        dtype=torch.int64, device=dev)
     world = dist.get_world_size(group)
-    n = torch.tensor([_wire(t).numel()], dtype=torch.int64, device=t.device)
+    allc = [torch.zeros_like(mine) for _ in range(world)]
+    dist.all_gather(allc, mine, group=group)
+    return [tuple(int(x) for x in c.tolist()) for c in allc]
+
+
+def allgatherv(t, group=None):
+    """Count-exact all-gather of a 1-D tensor: one broadcast per source of exactly its elements."""
+    import torch
+    import torch.distributed as dist
+
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    src = _wire(t.contiguous())
+    n = torch.tensor([src.numel()], dtype=torch.int64, device=t.device)
     sizes = [torch.zeros_like(n) for _ in range(world)]
     dist.all_gather(sizes, n, group=group)
-    sizes = [int(s.item()) for s in sizes]
-    mx = max(sizes) if sizes else 0
-    if mx == 0:
-        return [t[:0] for _ in range(world)]
-    src = _wire(t)
-    pad = torch.zeros(mx, dtype=src.dtype, device=t.device)
-    pad[:src.numel()] = src
-    bufs = [torch.empty_like(pad) for _ in range(world)]
-    dist.all_gather(bufs, pad, group=group)
-    res = [b[:s] for b, s in zip(bufs, sizes)]
-    if t.dtype != src.dtype:
-        res = [r.view(t.dtype) for r in res]
-    return res
+    out = []
+    for g in range(world):
+        sz = int(sizes[g].item())
+        buf = src if g == rank else torch.empty(sz, dtype=src.dtype, device=t.device)
+        if sz:
+            dist.broadcast(buf, dist.get_global_rank(group, g) if group is not None else g, group=group)
+        out.append(buf.view(t.dtype) if t.dtype != src.dtype else buf)
+    return out
 
 
 def assemble(pieces: list, n: int):
@@ -143,32 +193,81 @@ def assemble(pieces: list, n: int):
 
 
 def allgatherv_tiles(C, group=None):
-    """Gather every rank's C shard (a Tiles object or an arrays dict with key 'm') on all ranks."""
-    arrays = C.arrays() if hasattr(C, "arrays") else {k: C[k] for k in ARRAYS}
-    m_local = C.m if hasattr(C, "m") else C["m"]
-    n = C.n if hasattr(C, "n") else C["n"]
-    import torch
-
-    dev = arrays["tile_ptr"].device
+    """Every rank's C shard (a Tiles object or an arrays dict with keys m, n) on every rank,
+    count-exact; returns (m, n, arrays)."""
+    arrays, m_local, n = _local(C)
     gathered = {k: allgatherv(arrays[k], group) for k in ARRAYS}
-    ms = allgatherv(torch.tensor([m_local], dtype=torch.int64, device=dev), group)
-    world = len(ms)
-    pieces = [dict(m=int(ms[g][0].item()), **{k: gathered[k][g] for k in ARRAYS}) for g in range(world)]
+    counts = _counts(arrays, m_local, group)
+    pieces = [dict(m=counts[g][0], **{k: gathered[k][g] for k in ARRAYS}) for g in range(len(counts))]
     return assemble(pieces, n)
 
 
-def spgemm_sharded(A_tiles, B_tiles, A_csr, B_csr, group=None):
-    """C = A*B with C tile rows sharded over the process group; returns (local C shard, full C arrays).
+def gatherv_tiles(C, dst: int = 0, group=None, out_device=None):
+    """Every rank's C shard sent to rank ``dst`` only, count-exact (point-to-point transfers of
+    exactly each shard's bytes).  ``out_device`` ("cpu" with pinned buffers, or the default: the
+    shard's device) receives them.  Returns (m, n, arrays) on ``dst`` and None elsewhere."""
+    import torch
+    import torch.distributed as dist
 
-    A_tiles/B_tiles must be present on every rank (see broadcast_tiles); A_csr/B_csr (host CSR)
-    give the partition weights.
-    """
+    arrays, m_local, n = _local(C)
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    counts = _counts(arrays, m_local, group)
+    glob = (lambda g: dist.get_global_rank(group, g)) if group is not None else (lambda g: g)
+    if rank != dst:
+        ops = [dist.P2POp(dist.isend, _wire(arrays[k].contiguous()), glob(dst), group=group)
+               for k in ARRAYS if arrays[k].numel()]
+        for r in dist.batch_isend_irecv(ops) if ops else []:
+            r.wait()
+        return None
+    dev = torch.device(out_device) if out_device is not None else arrays["tile_ptr"].device
+    pin = dev.type == "cpu" and torch.cuda.is_available()
+    pieces, ops = [], []
+    for g in range(world):
+        m_g, nt_g, nnz_g, dc = counts[g]
+        if g == rank:
+            pieces.append(dict(m=m_g, **{k: (arrays[k].to(dev) if dev != arrays[k].device else arrays[k])
+                                         for k in ARRAYS}))
+            continue
+        shapes = _shapes(m_g, nt_g, nnz_g, getattr(torch, _CODES[dc]))
+        bufs = {}
+        for k in ARRAYS:
+            nel, dt = shapes[k]
+            # receive into the shard's device (NCCL), staged to `dev` afterwards if that differs
+            recv_dev = arrays["tile_ptr"].device
+            bufs[k] = torch.empty(nel, dtype=dt, device=recv_dev)
+            if nel:
+                ops.append(dist.P2POp(dist.irecv, bufs[k], glob(g), group=group))
+        pieces.append(dict(m=m_g, **bufs))
+    for r in dist.batch_isend_irecv(ops) if ops else []:
+        r.wait()
+    if dev != arrays["tile_ptr"].device:
+        for p in pieces:
+            for k in ARRAYS:
+                if p[k].device != dev:
+                    h = torch.empty(p[k].shape, dtype=p[k].dtype, pin_memory=pin)
+                    h.copy_(p[k])
+                    p[k] = h
+    for p in pieces:
+        p["mask"] = _unwire(_wire(p["mask"]), "mask")
+    return assemble(pieces, n)
+
+
+def spgemm_sharded(A_tiles, B_tiles, group=None, reassemble: str = "gather"):
+    """C = A*B with C tile rows sharded over the process group (cuts computed on the device).
+
+    reassemble: "gather" -> full C on rank 0 (None elsewhere), "all" -> full C on every rank,
+    "none" -> C stays distributed.  Returns (local C shard, cuts, reassembled or None)."""
     import torch.distributed as dist
 
     from . import slice_rows, spgemm
 
     world, rank = dist.get_world_size(group), dist.get_rank(group)
-    cuts = partition_tile_rows(A_csr, B_csr, world)
+    cuts = partition_device(A_tiles, B_tiles, world)
     shard = slice_rows(A_tiles, int(cuts[rank]), int(cuts[rank + 1]))
     Cl = spgemm(shard, B_tiles)
-    return Cl, allgatherv_tiles(Cl, group)
+    full = None
+    if reassemble == "gather":
+        full = gatherv_tiles(Cl, 0, group)
+    elif reassemble == "all":
+        full = allgatherv_tiles(Cl, group)
+    return Cl, cuts, full

@@ -75,7 +75,7 @@ def _worker(rank, world, port, result_path):
         arrs = _to_torch(TB) if rank == 0 else None
         meta_r, got = tdist.broadcast_tiles(arrs, meta, 0, torch.device("cpu"))
         ref = _to_torch(TB)
-        ok_b = meta_r == (A.m, A.n, TB.num_tiles, TB.nnz) and all(
+        ok_b = meta_r == (A.m, A.n, TB.num_tiles, TB.nnz, torch.float64) and all(
             torch.equal(got[k].view(torch.int16) if k == "mask" else got[k],
                         ref[k].view(torch.int16) if k == "mask" else ref[k]) for k in tdist.ARRAYS)
         # 2) local shard of C tile rows (oracle stands in for the GPU kernels)
@@ -85,27 +85,53 @@ def _worker(rank, world, port, result_path):
         sub = oracle.spgemm(A, A, fma=True, rows=rows)
         Cl = oracle.csr_to_tiles(gen.CSR(len(rows), A.n, sub.rowptr, sub.col, sub.val))
         piece = dict(m=len(rows), n=A.n, **_to_torch(Cl))
-        # 3) uneven all-gather + rebasing
-        m, n, full = tdist.allgatherv_tiles(piece)
+        # 3) count-exact all-gather + rebasing (every rank), and gatherv to rank 0 only
         exp = oracle.expected_tiles(A, A, fma=True)
-        ok_c = (m, n) == (A.m, A.n)
-        for k in tdist.ARRAYS:
-            a = full[k].view(torch.int16).numpy().view(np.uint16) if k == "mask" else full[k].numpy()
-            ok_c &= bool(np.array_equal(a, getattr(exp, k)))
+
+        def same(res):
+            if res is None:
+                return False
+            m, n, full = res
+            ok = (m, n) == (A.m, A.n)
+            for k in tdist.ARRAYS:
+                a = full[k].view(torch.int16).numpy().view(np.uint16) if k == "mask" else full[k].numpy()
+                ok &= bool(np.array_equal(a, getattr(exp, k)))
+            return ok
+
+        ok_c = same(tdist.allgatherv_tiles(piece))
+        g = tdist.gatherv_tiles(piece, dst=0)
+        ok_g = same(g) if rank == 0 else g is None
         with open(f"{result_path}.{rank}", "w") as f:
-            f.write(f"{int(ok_b)} {int(ok_c)} {I0} {I1}")
+            f.write(f"{int(ok_b)} {int(ok_c)} {int(ok_g)} {I0} {I1}")
     finally:
         dist.destroy_process_group()
 
 
-def test_gloo_broadcast_and_allgatherv_world2(tmp_path):
-    world = 2
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_broadcast_allgatherv_gatherv(tmp_path, world):
+    """World 2 and 3 (gloo, CPU): B broadcast, product-balanced shards, count-exact all-gather on
+    every rank and gatherv to rank 0 both reassemble exactly the oracle's C = A^2."""
     port = _free_port()
     mp.spawn(_worker, args=(world, port, str(tmp_path / "res")), nprocs=world, join=True)
     spans = []
     for r in range(world):
-        ok_b, ok_c, i0, i1 = open(tmp_path / f"res.{r}").read().split()
+        ok_b, ok_c, ok_g, i0, i1 = open(tmp_path / f"res.{r}").read().split()
         assert ok_b == "1", f"broadcast mismatch on rank {r}"
-        assert ok_c == "1", f"assembled C mismatch on rank {r}"
+        assert ok_c == "1", f"all-gathered C mismatch on rank {r}"
+        assert ok_g == "1", f"gatherv result wrong on rank {r}"
         spans.append((int(i0), int(i1)))
-    assert spans[0][0] == 0 and spans[0][1] == spans[1][0]
+    assert spans[0][0] == 0 and all(spans[g][1] == spans[g + 1][0] for g in range(world - 1))
+
+
+def test_exact_integer_cuts_match_float_searchsorted():
+    """The integer cut rule (first i with pre[i] * world >= g * total) is searchsorted-left of the
+    real-valued targets g * total / world."""
+    rng = np.random.default_rng(3)
+    for _ in range(50):
+        w = rng.integers(0, 1000, rng.integers(1, 300))
+        for world in (2, 3, 5, 8):
+            cuts = tdist.cuts_from_weights(w, world)
+            pre = np.concatenate(([0], np.cumsum(w)))
+            ref = np.maximum.accumulate(np.concatenate(
+                ([0], np.searchsorted(pre, np.arange(1, world) * pre[-1] / world, side="left"), [w.size])))
+            assert np.array_equal(cuts, ref)

@@ -628,3 +628,18 @@ def test_free_is_ordered_on_the_producing_stream(tsg):
         got = host(D)
         for k in ARRAYS:
             assert np.array_equal(got[k], ref[k]), k
+
+
+def test_device_partition_matches_host_rule(tsg):
+    """tsg_partition_tile_rows: per-tile-row products counted on the device and
+    cut at equal shares equal the host-CSR rule, and the total equals the oracle's products."""
+    from paper_conf_ppopp_niuljs0022_b200 import dist as tdist
+
+    for A in (gen.config("C1"), gen.rmat(11), gen.strip_fem(4, 40, 6), gen.stencil27(12),
+              gen.random_sparse(100, 115, 0.03, 3)):
+        B = gen.random_sparse(A.n, 77, 0.05, 5) if A.m != A.n else A
+        TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
+        for parts in (1, 2, 3, 8, 31):
+            cuts, prods = tsg.partition_tile_rows(TA, TB, parts)
+            assert np.array_equal(cuts, tdist.partition_tile_rows(A, B, parts)), (A.name, parts)
+            assert prods == oracle.products(A, B)
