@@ -219,7 +219,7 @@ def csr_to_tiles(row_ptr, col_idx, val, shape, validate: bool = False, stream=No
 def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, products: bool = False,
            structural: bool = False, scan_only: bool = False, list_always: bool = False,
            dense_threshold: int | None = None, sort_only: bool = False, path_general: bool = False,
-           path_rows: bool = False,
+           path_rows: bool = False, debug_high_offsets: bool = False,
            small_stage: bool | None = None, queue_chunk: int | None = None, stream=None) -> Tiles:
     """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3).
 
@@ -227,7 +227,8 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
     event step times, the intermediate-product count, |C'| of the paper's step 1.  The other
     options select work splits only (the result is the same bit for bit): step-1 modes, the dense
     threshold t_nnz, ``path_general`` (the per-C-tile pipeline even for narrow tile rows), ``path_rows``
-    (the fused per-tile-row pipeline wherever every tile row is narrow),
+    (the fused per-tile-row pipeline wherever every tile row is narrow), ``debug_high_offsets`` (C's
+    nonzero offsets carry +2^32 inside the call: a test of the 64-bit offset paths),
     ``queue_chunk`` (per-C-tile work distribution: 0 static, k > 0 k groups per request)."""
     L = _lib.load()
     flags = 0
@@ -247,6 +248,8 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
         flags |= _lib.PATH_GENERAL
     if path_rows:
         flags |= _lib.PATH_ROWS_FORCE
+    if debug_high_offsets:
+        flags |= _lib.DEBUG_HIGH_OFFSETS
     if small_stage is not None:
         flags |= _lib.SMALL_STAGE_ON if small_stage else _lib.SMALL_STAGE_OFF
     if dense_threshold is not None:

@@ -25,6 +25,7 @@ STEP1_LIST_ALWAYS = 0x8
 STATS_PRODUCTS = 0x10
 PATH_GENERAL = 0x20
 PATH_ROWS_FORCE = 0x400
+DEBUG_HIGH_OFFSETS = 0x800
 STEP1_SORT_ONLY = 0x40
 SMALL_STAGE_ON = 0x100
 SMALL_STAGE_OFF = 0x200

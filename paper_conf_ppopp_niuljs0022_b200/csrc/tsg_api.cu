@@ -184,6 +184,14 @@ __global__ void k_rebase(const int64_t *__restrict__ src, int64_t *__restrict__ 
 }
 }  // namespace
 
+__global__ void k_add_i64(int64_t *__restrict__ a, int64_t count, int64_t v) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < count) a[i] += v;
+}
+void launch_add_i64(int64_t *a, int64_t count, int64_t v, cudaStream_t s) {
+    TSG_LAUNCH(k_add_i64, grid_for(count, 256), 256, 0, s, a, count, v);
+}
+
 void launch_rebase(const int64_t *src, int64_t *dst, int64_t count, cudaStream_t s) {
     TSG_LAUNCH(k_rebase, grid_for(count, 256), 256, 0, s, src, dst, count);
 }

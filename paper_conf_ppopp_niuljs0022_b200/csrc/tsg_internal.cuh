@@ -229,6 +229,7 @@ void launch_csr_to_tiles(int64_t m, int64_t n, int64_t nnz, const int64_t *rp, c
                          tsg_tiles *out);
 void launch_tiles_to_csr(const tsg_tiles *T, int64_t *rp, int32_t *ci, void *v, cudaStream_t s);
 void launch_rebase(const int64_t *src, int64_t *dst, int64_t count, cudaStream_t s);
+void launch_add_i64(int64_t *a, int64_t count, int64_t v, cudaStream_t s);  // a[0..count) += v
 void launch_transpose_tiles(const tsg_tiles *T, const Allocator &al, cudaStream_t s, tsg_tiles *O);
 void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Allocator &al,
                 cudaStream_t s, tsg_tiles *C, tsg_stats *stats);

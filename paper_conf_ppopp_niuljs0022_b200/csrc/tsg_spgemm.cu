@@ -106,6 +106,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     if (TH == 0) TH = TSG_DENSE_NNZ;
     TSG_REQUIRE(TH <= 257, TSG_ERR_INVALID_ARG, "dense threshold > 257");
     const int qv = (int)((flags >> TSG_QUEUE_CHUNK_SHIFT) & 0xfu);
+    // TSG_DEBUG_HIGH_OFFSETS: C's nonzero offsets carry +2^32 during step 3 (against shifted bases)
+    const int64_t bias = (flags & TSG_DEBUG_HIGH_OFFSETS) ? ((int64_t)1 << 32) : 0;
     Timer tm_;
     tm_.init((flags & TSG_STATS_TIMING) && st, s);
     tm_.mark(0);
@@ -268,7 +270,17 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         R.n_dense = (int64_t)hc2.n2dense;
         R.dense = hc2.n2dense ? tmp.get<uint8_t>(DENSE_REC_BYTES * (int64_t)hc2.n2dense) : nullptr;
         R.cnt = cnt;
+        if (bias) {
+            launch_add_i64(rowOff, tmA + 1, bias, s);
+            C->idx -= bias;
+            C->val = static_cast<uint8_t *>(C->val) - bias * (int64_t)dtype_size(dtC);
+        }
         launch_num_rows(R, s);
+        if (bias) {
+            launch_add_i64(C->tile_nnz, ntC + 1, -bias, s);
+            C->idx += bias;
+            C->val = static_cast<uint8_t *>(C->val) + bias * (int64_t)dtype_size(dtC);
+        }
         tm_.mark(5);
     } else {
         if (hc.nbig > 0) {
@@ -346,9 +358,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
         tm_.mark(4);
         // ---------------- a4: step 3
-        P.ixC = idx;
-        P.vC = val;
+        P.ixC = idx - bias;
+        P.vC = static_cast<uint8_t *>(val) - bias * (int64_t)dtype_size(dtC);
+        if (bias) launch_add_i64(tile_nnz, ntC + 1, bias, s);
         launch_step3(P, (int64_t)hc2.n2dense, s);
+        if (bias) launch_add_i64(tile_nnz, ntC + 1, -bias, s);
         tm_.mark(5);
         C->tile_ptr = tile_ptr;
         C->tile_col = tile_col;

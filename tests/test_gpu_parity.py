@@ -581,7 +581,7 @@ def test_unknown_flags_rejected(tsg):
     A = gen.config("C1")
     T = tiles_of(tsg, A)
     out = C.c_void_p()
-    for bad in (0x80, 0x800, 1 << 29):  # 0x80: the removed tensor-core flag
+    for bad in (0x80, 0x1000, 1 << 29):  # 0x80: the removed tensor-core flag
         rc = _lib.load().tsg_spgemm(T.ptr, T.ptr, bad, None, None, C.byref(out), None)
         assert rc == 1 and out.value is None
 
@@ -643,3 +643,50 @@ def test_device_partition_matches_host_rule(tsg):
             cuts, prods = tsg.partition_tile_rows(TA, TB, parts)
             assert np.array_equal(cuts, tdist.partition_tile_rows(A, B, parts)), (A.name, parts)
             assert prods == oracle.products(A, B)
+
+
+def _high_word_view(tsg, T, bias=1 << 32):
+    """A handle over T's arrays whose nonzero offsets carry +bias (tile_nnz + bias) against idx /
+    val base pointers moved back by bias elements: every A/B value address the kernels form is
+    unchanged, but only if they keep the offsets' high words."""
+    import ctypes as C
+
+    import torch
+
+    from paper_conf_ppopp_niuljs0022_b200 import _lib
+
+    tz = (T.tile_nnz + bias).contiguous()
+    v = _lib.TilesView()
+    v.m, v.n, v.tile_m, v.tile_n, v.num_tiles, v.nnz = T.m, T.n, T.tile_m, T.tile_n, T.num_tiles, T.nnz
+    v.tile_ptr, v.tile_col, v.tile_nnz = T.tile_ptr.data_ptr(), T.tile_col.data_ptr(), tz.data_ptr()
+    v.row_ptr, v.mask = T.row_ptr.data_ptr(), T.mask.data_ptr()
+    v.idx = T.idx.data_ptr() - bias
+    v.val = T.val.data_ptr() - bias * T.val.element_size()
+    v.dtype = {torch.float64: 0, torch.float32: 1, torch.float16: 2}[T.val.dtype]
+    out = C.c_void_p()
+    _lib.check(_lib.load().tsg_tiles_wrap(C.byref(v), None, C.byref(out)))
+
+    class View:  # only the handle: its idx/val base pointers are not allocations torch could wrap
+        pass
+
+    V = View()
+    V.handle = tsg._Handle(out.value)
+    V.ptr = C.c_void_p(out.value)
+    V.keep = (T, tz)
+    return V
+
+
+@pytest.mark.parametrize("opts", [{}, dict(path_general=True), dict(path_rows=True), dict(dense_threshold=1)],
+                         ids=["default", "per-tile", "rows", "dense"])
+def test_int64_offsets_with_high_words(tsg, opts):
+    """64-bit offset paths (T4): inputs whose nonzero offsets exceed 2^32 and C's offsets biased by
+    2^32 inside the call (TSG_DEBUG_HIGH_OFFSETS) give the same C bit for bit."""
+    for A in (gen.config("C1"), gen.rmat(11), gen.strip_fem(6, 20, 6), gen.stencil27(10),
+              gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)):
+        T = tiles_of(tsg, A)
+        ref = host(tsg.spgemm(T, T, **opts))
+        V = _high_word_view(tsg, T)
+        got = host(tsg.spgemm(V, V, debug_high_offsets=True, **opts))
+        for k in ARRAYS[:-1]:
+            assert np.array_equal(got[k], ref[k]), (A.name, k)
+        assert bitwise_equal_values(got["val"], ref["val"])
