@@ -166,6 +166,7 @@ struct RowNumArgs {
     int dense_threshold, small_max;
     int64_t n_dense;              // dense C tiles (counted by k_sym_rows)
     void *dense;                  // scratch for their records (32 B each)
+    void *small;                  // scratch for the small C tiles' records (32 B each, <= ntC)
     DevCounters *cnt;
 };
 constexpr int DENSE_REC_BYTES = 32;

@@ -17,6 +17,8 @@
 //          holding C(r, 8h..8h+7) in registers.
 // Every C entry has one owner and receives its products in ascending k = 16K + c, so the values
 // are bitwise equal to the per-C-tile path and to the oracle's fma mode (readings A8, A16).
+#include <algorithm>
+
 #include "tsg_device.cuh"
 
 namespace tsg {
@@ -51,10 +53,11 @@ constexpr int WARP_SMEM = (OFF_WORK + WORK_BYTES + 15) & ~15;
 static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
 static_assert(OFF_WORK % 16 == 0, "work area 16-byte aligned");
 
-struct DenseRec {
+struct TileRec {  // a C tile left by k_num_rows to k_num_small / k_num_dense
     int64_t slot, off, pairs;
-    uint32_t cnt, pad;
+    uint32_t cnt, nz;
 };
+typedef TileRec DenseRec;
 
 struct RowNumParams {
     int64_t tm;
@@ -85,6 +88,7 @@ struct RowNumParams {
     void *vC;
     int dense_threshold, small_max;
     DenseRec *dense;  // dense C tiles, for k_num_dense
+    TileRec *small;   // small C tiles, for k_num_small
     DevCounters *cnt;
 };
 
@@ -319,7 +323,7 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
 #pragma unroll
     for (int j = 0; j < TILE; j++) acc[j * 16] = (TO)0;
     __syncwarp();
-    u64c nsm = 0, nmd = 0;
+    u64c nmd = 0;
     const unsigned lt = (1u << r) - 1u;
     const int64_t nCmax = max(nC, __shfl_xor_sync(FULL, nC, 16));
     for (int64_t q0 = 0; q0 < nCmax; q0 += 16) {
@@ -356,7 +360,6 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
         const unsigned BM = __ballot_sync(FULL, isM), BS = __ballot_sync(FULL, isS), BD = __ballot_sync(FULL, isD);
         unsigned bM = (BM >> (16 * half)) & 0xffffu;
         const unsigned bS = (BS >> (16 * half)) & 0xffffu, bD = (BD >> (16 * half)) & 0xffffu;
-        nsm += __popc(bS);
         nmd += __popc(bM);
 
         // ---- medium tiles: each half its next one, in step
@@ -371,60 +374,19 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
             both = __ballot_sync(FULL, bM != 0);
         }
 
-        // ---- small tiles: one lane per C nonzero
+        // ---- small tiles: recorded for k_num_small (a lane per C nonzero, its own kernel at full
+        // occupancy: the per-entry work is a chain of dependent loads)
         if (BS) {
-            const uint32_t mine = isS ? nz : 0u;
-            uint32_t in2 = mine;
-#pragma unroll
-            for (int d = 1; d < 16; d <<= 1) {
-                const uint32_t o = __shfl_up_sync(FULL, in2, d, 16);
-                if (r >= d) in2 += o;
-            }
-            const uint32_t ex2 = in2 - mine, tot = __shfl_sync(FULL, in2, 15, 16);
-            const uint32_t totm = max(tot, __shfl_xor_sync(FULL, tot, 16));
-            uint8_t *map = reinterpret_cast<uint8_t *>(&S);  // entry -> tile (<= 16 x small_max entries)
-            for (uint32_t k = 0; k < mine; k++) map[ex2 + k] = (uint8_t)r;
-            __syncwarp();
-            for (uint32_t e0 = 0; e0 < totm; e0 += 16) {
-                const uint32_t e = e0 + r;
-                const bool act = e < tot;
-                const int f = act ? map[e] : 0;
-                const uint32_t k = e - __shfl_sync(FULL, ex2, f + 16 * half);
-                const uint32_t fst = __shfl_sync(FULL, st, f + 16 * half), fcn = __shfl_sync(FULL, cn, f + 16 * half);
-                const int64_t foff = __shfl_sync(FULL, off, f + 16 * half);
-                if (act) {
-                    const int64_t fs = base + q0 + f;
-                    const uint4 rp = *reinterpret_cast<const uint4 *>(P.sRowPtrC + fs * TILE);
-                    // r = #{r' in 1..15 : row_ptr[r'] <= k}  (bytewise compare; row_ptr[0] = 0)
-                    const uint32_t kk = k * 0x01010101u;
-                    const int rr = (__popc(__vcmpleu4(rp.x, kk)) + __popc(__vcmpleu4(rp.y, kk)) +
-                                    __popc(__vcmpleu4(rp.z, kk)) + __popc(__vcmpleu4(rp.w, kk))) / 8 - 1;
-                    const uint32_t rpw = rr < 4 ? rp.x : rr < 8 ? rp.y : rr < 12 ? rp.z : rp.w;
-                    const int kr = (int)k - (int)((rpw >> (8 * (rr & 3))) & 0xffu);
-                    const int j = (int)__fns((uint32_t)P.sMaskC[fs * TILE + rr], 0, kr + 1);
-                    const uint32_t lowj = (1u << j) - 1u;
-                    TO a_acc = (TO)0;
-                    for (uint32_t p = 0; p < fcn; p++) {
-                        const uint64_t pr = P.pairs[base + fst + p];
-                        const int sa = (int)((int64_t)(pr >> 32) - a0);
-                        const int64_t pB = (int64_t)(uint32_t)pr;
-                        const uint32_t mAr = sMA[sa * TILE + rr];
-                        uint32_t x = mAr & P.mTB[pB * TILE + j];
-                        if (!x) continue;
-                        const TI *pa = vA + sZA[sa] + sRA[sa * TILE + rr];
-                        const TI *pb = vB + P.tnzB[pB];
-                        while (x) {
-                            const int c = __ffs(x) - 1;
-                            x &= x - 1;
-                            const TO av = vcvt<TO>(pa[__popc(mAr & ((1u << c) - 1u))]);
-                            const TO bv = vcvt<TO>(pb[P.rpB[pB * TILE + c] + __popc((uint32_t)P.mB[pB * TILE + c] & lowj)]);
-                            a_acc = vfma(av, bv, a_acc);
-                        }
-                    }
-                    P.ixC[foff + k] = (uint8_t)((rr << 4) | j);
-                    vC[foff + k] = a_acc;
-                }
-                __syncwarp();
+            uint32_t si = 0;
+            if (r == 0 && bS) si = (uint32_t)atomicAdd(&P.cnt->n3small, (u64c)__popc(bS));
+            si = __shfl_sync(FULL, si, 16 * half);
+            if (isS) {
+                TileRec &d = P.small[si + __popc(bS & lt)];
+                d.slot = slot;
+                d.off = off;
+                d.pairs = base + st;
+                d.cnt = cn;
+                d.nz = nz;
             }
         }
 
@@ -443,9 +405,89 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
             }
         }
     }
-    if (r == 0) {
-        if (nsm) atomicAdd(&P.cnt->n3small, nsm);
-        if (nmd) atomicAdd(&P.cnt->n3medium, nmd);
+    if (r == 0 && nmd) atomicAdd(&P.cnt->n3medium, nmd);
+}
+
+// small C tiles (nnz <= small_max) recorded by k_num_rows: one lane per C nonzero (the
+// output-stationary form of the paper's sparse accumulator): entry q of a tile is
+// (r, j), r = the last row with row_ptr_C[r] <= q, j = the (q - row_ptr_C[r])-th bit of
+// mask_C[r]; the lane walks the tile's pairs in ascending K and, per pair, the columns c of
+// mask_A[r] & colmask_B[j] in ascending order.  Warps take 32 records at a time.
+constexpr int NS_T = 256;
+template <typename TI, typename TO>
+__global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) {
+    __shared__ uint8_t mapsm[NS_T / 32][32 * 16];
+    const int lane = threadIdx.x & 31;
+    uint8_t *map = mapsm[threadIdx.x >> 5];
+    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
+    TO *vC = static_cast<TO *>(P.vC);
+    const int64_t n = (int64_t)P.cnt->n3small;
+    const int64_t gw = (int64_t)blockIdx.x * (NS_T / 32) + (threadIdx.x >> 5), nw = (int64_t)gridDim.x * (NS_T / 32);
+    for (int64_t g0 = gw * 32; g0 < n; g0 += nw * 32) {
+        const int64_t k = g0 + lane;
+        TileRec d{};
+        if (k < n) d = P.small[k];
+        const uint32_t mine = k < n ? d.nz : 0u;
+        uint32_t incl = mine;
+#pragma unroll
+        for (int s = 1; s < 32; s <<= 1) {
+            const uint32_t o = __shfl_up_sync(FULL, incl, s);
+            if (lane >= s) incl += o;
+        }
+        const uint32_t excl = incl - mine, tot = __shfl_sync(FULL, incl, 31);
+        for (uint32_t q = 0; q < mine; q++) map[excl + q] = (uint8_t)lane;
+        __syncwarp();
+        for (uint32_t e0 = 0; e0 < tot; e0 += 32) {
+            const uint32_t e = e0 + lane;
+            const bool act = e < tot;
+            const int f = act ? map[e] : 0;
+            const uint32_t q = e - __shfl_sync(FULL, excl, f);
+            const int64_t fs = __shfl_sync(FULL, d.slot, f), foff = __shfl_sync(FULL, d.off, f);
+            const int64_t fp = __shfl_sync(FULL, d.pairs, f);
+            const uint32_t fcn = __shfl_sync(FULL, d.cnt, f);
+            if (act) {
+                const uint4 rp = *reinterpret_cast<const uint4 *>(P.sRowPtrC + fs * TILE);
+                // r = #{r' in 1..15 : row_ptr[r'] <= q}  (bytewise compare; row_ptr[0] = 0)
+                const uint32_t qq = q * 0x01010101u;
+                const int rr = (__popc(__vcmpleu4(rp.x, qq)) + __popc(__vcmpleu4(rp.y, qq)) +
+                                __popc(__vcmpleu4(rp.z, qq)) + __popc(__vcmpleu4(rp.w, qq))) / 8 - 1;
+                const uint32_t rpw = rr < 4 ? rp.x : rr < 8 ? rp.y : rr < 12 ? rp.z : rp.w;
+                const int kr = (int)q - (int)((rpw >> (8 * (rr & 3))) & 0xffu);
+                const int j = (int)__fns((uint32_t)P.sMaskC[fs * TILE + rr], 0, kr + 1);
+                const uint32_t lowj = (1u << j) - 1u;
+                TO acc = (TO)0;
+                // the next pair's masks and offsets are loaded while the current one multiplies
+                uint64_t pr = P.pairs[fp];
+                int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+                uint32_t mAr = P.mA[pA * TILE + rr], mTj = P.mTB[pB * TILE + j];
+                int64_t zA = P.tnzA[pA] + P.rpA[pA * TILE + rr], zB = P.tnzB[pB];
+                if (fcn > 1) pr = P.pairs[fp + 1];
+                for (uint32_t p = 0; p < fcn; p++) {
+                    const int64_t cB = pB, czA = zA, czB = zB;
+                    uint32_t x = mAr & mTj;
+                    const uint32_t cmA = mAr;
+                    if (p + 1 < fcn) {
+                        pA = (int64_t)(pr >> 32);
+                        pB = (int64_t)(uint32_t)pr;
+                        mAr = P.mA[pA * TILE + rr];
+                        mTj = P.mTB[pB * TILE + j];
+                        zA = P.tnzA[pA] + P.rpA[pA * TILE + rr];
+                        zB = P.tnzB[pB];
+                        if (p + 2 < fcn) pr = P.pairs[fp + p + 2];
+                    }
+                    while (x) {
+                        const int c = __ffs(x) - 1;
+                        x &= x - 1;
+                        const TO a = vcvt<TO>(vA[czA + __popc(cmA & ((1u << c) - 1u))]);
+                        const TO b = vcvt<TO>(vB[czB + P.rpB[cB * TILE + c] + __popc((uint32_t)P.mB[cB * TILE + c] & lowj)]);
+                        acc = vfma(a, b, acc);
+                    }
+                }
+                P.ixC[foff + q] = (uint8_t)((rr << 4) | j);
+                vC[foff + q] = acc;
+            }
+        }
+        __syncwarp();
     }
 }
 
@@ -463,6 +505,18 @@ __global__ void __launch_bounds__(RN_T) k_num_dense(RowNumParams P, int64_t n) {
 template <typename TI, typename TO>
 void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s) {
     TSG_LAUNCH((k_num_rows<TI, TO>), grid_for(ceil_div(P.tm, 2), RN_W), RN_T, 0, s, P);
+    if (P.small) {  // persistent grid: the record count is read on the device
+        static int occ = 0;
+        int nsm = 148;
+        if (!occ) {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_small<TI, TO>, NS_T, 0);
+            occ = std::max(occ, 1) * nsm;
+        }
+        TSG_LAUNCH((k_num_small<TI, TO>), (unsigned)occ, NS_T, 0, s, P);
+    }
     if (n_dense > 0) TSG_LAUNCH((k_num_dense<TI, TO>), grid_for(n_dense, RN_W), RN_T, 0, s, P, n_dense);
 }
 
@@ -503,6 +557,7 @@ void launch_num_rows(const RowNumArgs &a, cudaStream_t s) {
     P.dense_threshold = a.dense_threshold;
     P.small_max = a.small_max;
     P.dense = static_cast<DenseRec *>(a.dense);
+    P.small = static_cast<TileRec *>(a.small);
     P.cnt = a.cnt;
     switch (a.A->dtype) {
         case TSG_F64: launch_t<double, double>(P, a.n_dense, s); break;
