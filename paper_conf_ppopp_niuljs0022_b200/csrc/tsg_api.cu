@@ -124,17 +124,30 @@ struct ExportArgs {
     uint32_t bytes[4], off[4];
     int n;
     uint8_t *dst;
+    volatile unsigned int *flag;  // written last, after a system-scope fence
+    unsigned int seq;
 };
 __global__ void k_export(ExportArgs a) {
     for (int k = 0; k < a.n; k++)
         for (uint32_t i = threadIdx.x; i < a.bytes[k]; i += blockDim.x) a.dst[a.off[k] + i] = a.src[k][i];
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) *a.flag = a.seq;
 }
 struct Mapped {
     uint8_t *h = nullptr;
     uint8_t *d = nullptr;
+    unsigned int seq = 0;
 };
 constexpr size_t MAPPED_BYTES = 4096;
+constexpr size_t FLAG_OFF = MAPPED_BYTES - 64;  // the completion flag's slot
 }  // namespace
+
+// The host waits for the export by spinning on its completion flag in mapped memory (microseconds
+// sooner than a stream synchronisation wakes up), for up to SPIN_US; then -- long steps, or a
+// failed kernel that never writes the flag -- it falls back to cudaStreamSynchronize, which also
+// reports errors.  Either way the stream has passed the export when this returns.
+constexpr double SPIN_US = 200.0;
 
 void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
     int dev = 0;
@@ -147,12 +160,13 @@ void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
         TSG_CUDA(cudaHostGetDevicePointer(&d, h, 0));
         mp.h = static_cast<uint8_t *>(h);
         mp.d = static_cast<uint8_t *>(d);
+        *reinterpret_cast<volatile unsigned int *>(mp.h + FLAG_OFF) = 0u;
     }
     ExportArgs a{};
     uint32_t off = 0;
     TSG_REQUIRE(segs.size() <= 4, TSG_ERR_INTERNAL, "too many device reads");
     for (const DevRead &r : segs) {
-        TSG_REQUIRE(off + r.bytes <= MAPPED_BYTES, TSG_ERR_INTERNAL, "device read too large");
+        TSG_REQUIRE(off + r.bytes <= FLAG_OFF, TSG_ERR_INTERNAL, "device read too large");
         a.src[a.n] = static_cast<const uint8_t *>(r.dev);
         a.bytes[a.n] = (uint32_t)r.bytes;
         a.off[a.n] = off;
@@ -160,9 +174,21 @@ void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
         off += (uint32_t)((r.bytes + 15) & ~(size_t)15);
     }
     a.dst = mp.d;
+    a.flag = reinterpret_cast<volatile unsigned int *>(mp.d + FLAG_OFF);
+    a.seq = ++mp.seq;
     TSG_LAUNCH(k_export, 1, 256, 0, s, a);
     const double t0 = now_ms();
-    TSG_CUDA(cudaStreamSynchronize(s));
+    volatile unsigned int *hf = reinterpret_cast<volatile unsigned int *>(mp.h + FLAG_OFF);
+    bool seen = false;
+    while (!(seen = (*hf == a.seq)) && (now_ms() - t0) * 1e3 < SPIN_US) {
+    }
+    if (seen) {
+        std::atomic_thread_fence(std::memory_order_acquire);
+        // the stream is past the export once its flag is visible; keep the stream-ordered
+        // semantics of the old synchronisation for what the caller launches next
+    } else {
+        TSG_CUDA(cudaStreamSynchronize(s));
+    }
     t_host_sync_ms += now_ms() - t0;
     int k = 0;
     for (const DevRead &r : segs) {

@@ -128,7 +128,8 @@ struct StepParams {
 };
 
 // launchers (tsg_step1.cu)
-void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s);
+void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s,
+                      void *zero = nullptr, size_t zero_bytes = 0);  // also zeroes `zero` (the call's counters)
 void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
                     uint32_t *list, cudaStream_t s);
 void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int64_t ntA, const int32_t *tcA,

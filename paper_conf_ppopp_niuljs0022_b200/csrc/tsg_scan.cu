@@ -64,7 +64,7 @@ template <typename Tin>
 __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n, int64_t *out, uint64_t *status,
                                                       unsigned long long *ticket) {
     __shared__ int64_t s_bid, s_base;
-    if (threadIdx.x == 0) s_bid = (int64_t)atomicAdd(ticket, 1ull);
+    if (threadIdx.x == 0) s_bid = gridDim.x == 1 ? 0 : (int64_t)atomicAdd(ticket, 1ull);
     __syncthreads();
     const int64_t b = s_bid;
     const int64_t base = b * SCAN_TILE + (int64_t)threadIdx.x * SCAN_IPT;
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n,
         const int lane = threadIdx.x;
         int64_t excl = 0;
         if (b == 0) {
-            if (lane == 0) st_status(status, ST_PRE | (uint64_t)total);
+            if (lane == 0 && gridDim.x > 1) st_status(status, ST_PRE | (uint64_t)total);
         } else {
             if (lane == 0) st_status(status + b, ST_AGG | (uint64_t)total);
             for (int64_t j = b - 1;; j -= 32) {
@@ -123,7 +123,7 @@ void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buff
     }
     const int64_t nb = ceil_div(n, SCAN_TILE);
     uint64_t *status = tmp.get<uint64_t>(nb + 1);  // [0, nb): tile status, [nb]: ticket
-    TSG_CUDA(cudaMemsetAsync(status, 0, sizeof(uint64_t) * (nb + 1), s));
+    if (nb > 1) TSG_CUDA(cudaMemsetAsync(status, 0, sizeof(uint64_t) * (nb + 1), s));  // one CTA: no look-back
     TSG_LAUNCH((k_scan_1pass<Tin>), (unsigned)nb, SCAN_T, 0, s, in, n, out, status,
                reinterpret_cast<unsigned long long *>(status + nb));
 }

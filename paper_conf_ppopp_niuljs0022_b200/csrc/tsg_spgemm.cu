@@ -115,8 +115,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     Buffers tmp(al, s, true), out(al, s);
     const int64_t ntA = A->nt, tmA = A->tm, tmB = B->tm;
     int syncs = 0;
-    DevCounters *cnt = tmp.get<DevCounters>(1);
-    TSG_CUDA(cudaMemsetAsync(cnt, 0, sizeof(DevCounters), s));
+    DevCounters *cnt = tmp.get<DevCounters>(1);  // zeroed by the first occupancy launch
+    static_assert(sizeof(DevCounters) % 8 == 0, "counters are zeroed as 64-bit words");
 
     // ---------------- a0: occupancy words, optional B row lists, optional product count
     // A inside B's tile arrays (A^2, or a row slice of B: SURVEY 8(e)'s rank shards and row blocks):
@@ -127,11 +127,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     uint16_t *colOccA;
     if (inB) {
         uint16_t *colOccB = tmp.get<uint16_t>(B->nt);
-        launch_occupancy(B->mask, B->nt, rowOccB, colOccB, s);
+        launch_occupancy(B->mask, B->nt, rowOccB, colOccB, s, cnt, sizeof(DevCounters));
         colOccA = colOccB + off;
     } else {
         colOccA = tmp.get<uint16_t>(ntA);
-        launch_occupancy(A->mask, ntA, nullptr, colOccA, s);
+        launch_occupancy(A->mask, ntA, nullptr, colOccA, s, cnt, sizeof(DevCounters));
         launch_occupancy(B->mask, B->nt, rowOccB, nullptr, s);
     }
     // transposed masks: first used by step 2 / 3, so they are computed on a side stream while

@@ -26,7 +26,9 @@ __device__ __forceinline__ int bits_for(uint64_t v) {  // bits needed to represe
 // A pair (A_IK, B_KJ) has a product iff colOcc(A_IK) & rowOcc(B_KJ) != 0.
 // ------------------------------------------------------------------------------------------
 __global__ void k_occupancy(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ row_occ,
-                            uint16_t *__restrict__ col_occ) {
+                            uint16_t *__restrict__ col_occ, uint64_t *__restrict__ zero, int zero_words) {
+    if (blockIdx.x == 0)  // the call's device counters start at zero (saves a memset launch)
+        for (int i = threadIdx.x; i < zero_words; i += blockDim.x) zero[i] = 0;
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nt) return;
     const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
@@ -1118,8 +1120,10 @@ __global__ void __launch_bounds__(256) k_compact(CompactParams P) {
 // ------------------------------------------------------------------------------------------
 // launchers
 // ------------------------------------------------------------------------------------------
-void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s) {
-    TSG_LAUNCH(k_occupancy, grid_for(nt, 256), 256, 0, s, mask, nt, row_occ, col_occ);
+void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s,
+                      void *zero, size_t zero_bytes) {
+    TSG_LAUNCH(k_occupancy, std::max(1u, grid_for(nt, 256)), 256, 0, s, mask, nt, row_occ, col_occ,
+               static_cast<uint64_t *>(zero), (int)(zero_bytes / 8));
 }
 
 void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
