@@ -463,3 +463,15 @@ def test_oracle_omp_equals_single_thread():
             assert np.array_equal(got.abs, ref.abs)
     full = oracle.spgemm(gen.config("C1"), gen.config("C1"), threads=4)
     assert full.nnz == 51972  # the C1 closed form
+
+
+def test_c1_golden_statistics_reproduce_with_scipy():
+    """The C1 tile statistics in tests/golden/c1_poisson2d64.txt (first measured in the survey) are
+    regenerated by a committed scipy-only script that shares nothing with oracle/ or the CUDA path."""
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "scripts", "golden_c1_stats.py"), "--check"],
+                         capture_output=True, text=True, cwd=root)
+    assert out.returncode == 0, out.stdout + out.stderr
