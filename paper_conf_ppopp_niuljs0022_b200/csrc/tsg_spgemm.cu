@@ -18,10 +18,28 @@
 #include <cstdlib>
 #include <cstring>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "tsg_kernels.cuh"
 
 namespace tsg {
 namespace {
+// NVTX ranges per step (one range per step of the method, visible in Nsight Systems /
+// ncu --nvtx; header-only NVTX3, a no-op without an attached tool)
+struct Range {
+    bool on = false;
+    void push(const char *name) {
+        pop();
+        nvtxRangePushA(name);
+        on = true;
+    }
+    void pop() {
+        if (on) nvtxRangePop();
+        on = false;
+    }
+    ~Range() { pop(); }
+};
+
 struct Timer {
     bool on = false;
     cudaStream_t s{};
@@ -112,6 +130,8 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     tm_.init((flags & TSG_STATS_TIMING) && st, s);
     tm_.mark(0);
 
+    Range nv;
+    nv.push("tsg a0 helper indices");
     Buffers tmp(al, s, true), out(al, s);
     const int64_t ntA = A->nt, tmA = A->tm, tmB = B->tm;
     int syncs = 0;
@@ -164,6 +184,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     tm_.mark(1);
 
     // ---------------- a1: plan
+    nv.push("tsg a1 plan");
     int64_t *cost = tmp.get<int64_t>(ntA);
     int64_t *startA = tmp.get<int64_t>(ntA);
     int32_t *jloA = tmp.get<int32_t>(ntA);
@@ -228,9 +249,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         P1.sRowPtrC = tmp.get<uint8_t>(TILE * Utot);
         P1.rowNnz = tmp.get<int64_t>(tmA);
         P1.dense_threshold = TH;
+        nv.push("tsg a1+a2 row path: tile layout, pairs, masks");
         launch_sym_rows(P1, tmA, s);
         tm_.mark(3);
         // ---------------- a3: tile and nonzero offsets of the rows; the one allocation of C
+        nv.push("tsg a3 scans + allocation");
         int64_t *rowOff = tmp.get<int64_t>(tmA + 1);
         exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
         exclusive_scan<int64_t>(P1.rowNnz, rowOff, tmA, s, tmp);
@@ -249,6 +272,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         tm_.mark(4);
         side.join();
         // ---------------- a4: step 3
+        nv.push("tsg a4 numeric");
         RowNumArgs R{};
         R.tm = tmA;
         R.A = A;
@@ -290,6 +314,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
             P1.bigPosB = tmp.get<uint32_t>(hc.big_u);
             P1.bigKpos = tmp.get<uint32_t>(hc.big_u);
         }
+        nv.push("tsg a1 step 1: tile layout + pairs");
         launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, (int64_t)hc.nmerge, s);
         exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
         // blocking read #2: number of C tiles
@@ -310,6 +335,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         launch_compact(PC, s);
 
         // ---------------- a2: step 2
+        nv.push("tsg a2 step 2: masks");
         side.join();
         StepParams P{};
         P.ntC = ntC;
@@ -351,6 +377,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         P.cnt = cnt;
         launch_step2(P, s);
         // ---------------- a3: offsets of C's nonzeros, allocation
+        nv.push("tsg a3 scan + allocation");
         exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp);
         DevCounters hc2{};
         read_device({{&nnzC, tile_nnz + ntC, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
@@ -359,6 +386,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
         tm_.mark(4);
         // ---------------- a4: step 3
+        nv.push("tsg a4 step 3: numeric");
         P.ixC = idx - bias;
         P.vC = static_cast<uint8_t *>(val) - bias * (int64_t)dtype_size(dtC);
         if (bias) launch_add_i64(tile_nnz, ntC + 1, bias, s);
