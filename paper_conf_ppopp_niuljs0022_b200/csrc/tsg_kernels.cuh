@@ -35,6 +35,22 @@ constexpr int SMALL_NNZ = 8;      // step-3 lane-per-entry class (k_s3_small): C
 constexpr int64_t ROWPATH_SMALL_U = 1 << 20;  // step-1 candidates below which narrow calls take the row path
 constexpr int MERGE_MAX_A = 32;   // step-1 warp-merge class: A tiles of the tile row (one lane each)
 
+// ---------------- a0 for hypersparse operands: one 16-byte record per tile.
+// A single-nonzero tile carries its entry and its value inline, so a pair of such tiles costs two
+// 16-byte loads in steps 2-3 instead of a sector each for mask, transposed mask, row offsets, value
+// offset and value (R-MAT tiles average 1.05 nonzeros).  As four 32-bit words:
+//   x, y  single: the value's bits (its dtype, low bytes first); else: the tile's nonzero offset
+//   z     tile column
+//   w     bits 0-15 row occupancy, 16-23 (r << 4) | c of the single nonzero, bit 24 single
+struct alignas(16) TileRec {
+    uint64_t v;
+    int32_t col;
+    uint32_t w;
+};
+static_assert(sizeof(TileRec) == 16, "one 16-byte load per tile");
+void launch_tile_records(int64_t nt, const int32_t *tile_col, const int64_t *tile_nnz, const uint16_t *mask,
+                         const uint8_t *idx, const void *val, int32_t dtype, TileRec *rec, cudaStream_t s);
+
 // ---------------- a1 row sort
 struct S1Params {
     const int64_t *tpA;
@@ -124,6 +140,8 @@ struct StepParams {
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     int small_stage;       // step 3: k_s3_small stages B row metadata with cp.async (hypersparse B)
+    const TileRec *recA, *recB;  // hypersparse operands: per-tile records (else nullptr)
+    int64_t recA_voff;     // added to A records' value offsets (A a row slice inside B: B's offsets)
     DevCounters *cnt;
 };
 

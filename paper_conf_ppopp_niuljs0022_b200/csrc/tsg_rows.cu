@@ -53,11 +53,11 @@ constexpr int WARP_SMEM = (OFF_WORK + WORK_BYTES + 15) & ~15;
 static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
 static_assert(OFF_WORK % 16 == 0, "work area 16-byte aligned");
 
-struct TileRec {  // a C tile left by k_num_rows to k_num_small / k_num_dense
+struct RowTileRec {  // a C tile left by k_num_rows to k_num_small / k_num_dense
     int64_t slot, off, pairs;
     uint32_t cnt, nz;
 };
-typedef TileRec DenseRec;
+typedef RowTileRec DenseRec;
 
 struct RowNumParams {
     int64_t tm;
@@ -88,7 +88,7 @@ struct RowNumParams {
     void *vC;
     int dense_threshold, small_max;
     DenseRec *dense;  // dense C tiles, for k_num_dense
-    TileRec *small;   // small C tiles, for k_num_small
+    RowTileRec *small;   // small C tiles, for k_num_small
     DevCounters *cnt;
 };
 
@@ -381,7 +381,7 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
             if (r == 0 && bS) si = (uint32_t)atomicAdd(&P.cnt->n3small, (u64c)__popc(bS));
             si = __shfl_sync(FULL, si, 16 * half);
             if (isS) {
-                TileRec &d = P.small[si + __popc(bS & lt)];
+                RowTileRec &d = P.small[si + __popc(bS & lt)];
                 d.slot = slot;
                 d.off = off;
                 d.pairs = base + st;
@@ -425,7 +425,7 @@ __global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) {
     const int64_t gw = (int64_t)blockIdx.x * (NS_T / 32) + (threadIdx.x >> 5), nw = (int64_t)gridDim.x * (NS_T / 32);
     for (int64_t g0 = gw * 32; g0 < n; g0 += nw * 32) {
         const int64_t k = g0 + lane;
-        TileRec d{};
+        RowTileRec d{};
         if (k < n) d = P.small[k];
         const uint32_t mine = k < n ? d.nz : 0u;
         uint32_t incl = mine;
@@ -557,7 +557,7 @@ void launch_num_rows(const RowNumArgs &a, cudaStream_t s) {
     P.dense_threshold = a.dense_threshold;
     P.small_max = a.small_max;
     P.dense = static_cast<DenseRec *>(a.dense);
-    P.small = static_cast<TileRec *>(a.small);
+    P.small = static_cast<RowTileRec *>(a.small);
     P.cnt = a.cnt;
     switch (a.A->dtype) {
         case TSG_F64: launch_t<double, double>(P, a.n_dense, s); break;

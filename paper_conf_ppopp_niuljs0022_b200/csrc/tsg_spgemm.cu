@@ -174,6 +174,25 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         exclusive_scan<int32_t>(lcnt, lptr, TILE * tmB, s, tmp);
         launch_rowlist(tmB, B->tile_ptr, B->mask, lptr, lcnt, list, s);
     }
+    // hypersparse operands (fewer than 4 nonzeros per B tile, no small-tile flag): 16-byte per-tile
+    // records for step 1's wide rows and steps 2-3 (inB: A's are a slice of B's)
+    TileRec *recA = nullptr, *recB = nullptr;
+    if (!(flags & (TSG_SMALL_STAGE_ON | TSG_SMALL_STAGE_OFF)) && B->nt > 0 && B->nnz < 4 * B->nt) {
+        recB = tmp.get<TileRec>(B->nt);
+        launch_tile_records(B->nt, B->tile_col, B->tile_nnz, B->mask, B->idx, B->val, B->dtype, recB, s);
+        // A's records are a slice of B's only if A's arrays are B's, shifted (a row slice of B):
+        // the records carry values, so sharing masks alone is not enough
+        const int64_t dz = (int64_t)(A->idx - B->idx);
+        const bool slice = inB && A->tile_col == B->tile_col + off && dz >= 0 &&
+                           static_cast<const uint8_t *>(A->val) ==
+                               static_cast<const uint8_t *>(B->val) + dz * (int64_t)A->vsize();
+        if (slice) {
+            recA = recB + off;
+        } else {
+            recA = tmp.get<TileRec>(std::max<int64_t>(ntA, 1));
+            launch_tile_records(ntA, A->tile_col, A->tile_nnz, A->mask, A->idx, A->val, A->dtype, recA, s);
+        }
+    }
     if (st && (flags & TSG_STATS_PRODUCTS)) {
         int32_t *rnnz = tmp.get<int32_t>(TILE * tmB);
         launch_products(tmB, B->tile_ptr, B->mask, ntA, A->tile_col, A->mask, rnnz, cnt, s);
@@ -374,6 +393,10 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         // small-tile B staging pays where B's tile metadata misses in cache: hypersparse tiles
         // (fewer than 4 nonzeros per B tile on average, e.g. R-MAT); flags force either way
         P.small_stage = (flags & TSG_SMALL_STAGE_ON) ? 1 : (flags & TSG_SMALL_STAGE_OFF) ? 0 : (B->nnz < 4 * B->nt);
+        P.recA = recA;
+        P.recB = recB;
+        // A's records are B's when A lies inside B: their value offsets count from B's values
+        P.recA_voff = (recA && recB && recA >= recB && recA < recB + B->nt) ? -(int64_t)(A->idx - B->idx) : 0;
         P.cnt = cnt;
         launch_step2(P, s);
         // ---------------- a3: offsets of C's nonzeros, allocation

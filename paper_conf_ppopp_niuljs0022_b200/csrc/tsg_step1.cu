@@ -46,6 +46,35 @@ __global__ void k_occupancy(const uint16_t *__restrict__ mask, int64_t nt, uint1
     if (col_occ) col_occ[t] = (uint16_t)co;
 }
 
+// per-tile records of a hypersparse operand (TileRec, tsg_kernels.cuh)
+template <typename TI>
+__global__ void k_tile_records(int64_t nt, const int32_t *__restrict__ tile_col, const int64_t *__restrict__ tile_nnz,
+                               const uint16_t *__restrict__ mask, const uint8_t *__restrict__ idx,
+                               const TI *__restrict__ val, TileRec *__restrict__ rec) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= nt) return;
+    const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
+    const uint4 a = __ldg(p), b = __ldg(p + 1);
+    const uint32_t w8[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    uint32_t ro = 0;
+#pragma unroll
+    for (int k = 0; k < 8; k++) ro |= ((w8[k] & 0xffffu) ? 1u : 0u) << (2 * k) | ((w8[k] >> 16) ? 1u : 0u) << (2 * k + 1);
+    const int64_t z0 = tile_nnz[t], z1 = tile_nnz[t + 1];
+    TileRec r;
+    r.col = tile_col[t];
+    if (z1 - z0 == 1) {
+        uint64_t bits = 0;
+        const TI x = val[z0];
+        memcpy(&bits, &x, sizeof(TI));
+        r.v = bits;
+        r.w = ro | (uint32_t)idx[z0] << 16 | 1u << 24;
+    } else {
+        r.v = (uint64_t)z0;
+        r.w = ro;
+    }
+    rec[t] = r;
+}
+
 // B row lists ("mode ii"): for each global row k of B, the B tiles of tile row k/16 whose row
 // k%16 is non-empty, ascending tile column.  One warp = two B tile rows, lane r = row r.
 __global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__restrict__ tpB,
@@ -1120,6 +1149,20 @@ __global__ void __launch_bounds__(256) k_compact(CompactParams P) {
 // ------------------------------------------------------------------------------------------
 // launchers
 // ------------------------------------------------------------------------------------------
+void launch_tile_records(int64_t nt, const int32_t *tile_col, const int64_t *tile_nnz, const uint16_t *mask,
+                         const uint8_t *idx, const void *val, int32_t dtype, TileRec *rec, cudaStream_t s) {
+    const unsigned g = grid_for(nt, 256);
+    if (dtype == TSG_F64)
+        TSG_LAUNCH(k_tile_records<double>, g, 256, 0, s, nt, tile_col, tile_nnz, mask, idx,
+                   static_cast<const double *>(val), rec);
+    else if (dtype == TSG_F32)
+        TSG_LAUNCH(k_tile_records<float>, g, 256, 0, s, nt, tile_col, tile_nnz, mask, idx,
+                   static_cast<const float *>(val), rec);
+    else
+        TSG_LAUNCH(k_tile_records<__half>, g, 256, 0, s, nt, tile_col, tile_nnz, mask, idx,
+                   static_cast<const __half *>(val), rec);
+}
+
 void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s,
                       void *zero, size_t zero_bytes) {
     TSG_LAUNCH(k_occupancy, std::max(1u, grid_for(nt, 256)), 256, 0, s, mask, nt, row_occ, col_occ,

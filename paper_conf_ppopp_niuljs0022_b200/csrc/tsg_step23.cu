@@ -72,30 +72,74 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
         for (int q = 0; q < 8; q++) w[q * T2L] = 0;
         const uint64_t *pp = P.pairs + P.pairBeg[t];
         const uint32_t np = P.pairCnt[t];
-        uint64_t pr = pp[0];
-        int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-        uint32_t x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
-        if (np > 1) pr = pp[1];
-        for (uint32_t p = 0; p < np; p++) {
-            const int64_t cA = pA, cB = pB;
-            uint32_t cx = x;
-            if (p + 1 < np) {
-                pA = (int64_t)(pr >> 32);
-                pB = (int64_t)(uint32_t)pr;
-                x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
-                if (p + 2 < np) pr = pp[p + 2];
+        if (P.recA) {
+            // hypersparse operands: a pair of single-nonzero tiles contributes the one bit
+            // (r_A, c_B) iff c_A == r_B, from the two records alone
+            const uint4 *RA = reinterpret_cast<const uint4 *>(P.recA), *RB = reinterpret_cast<const uint4 *>(P.recB);
+            uint64_t pr = pp[0];
+            int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+            uint4 ra = RA[pA], rb = RB[pB];
+            if (np > 1) pr = pp[1];
+            for (uint32_t p = 0; p < np; p++) {
+                const uint4 ca = ra, cb = rb;
+                const int64_t cA = pA, cB = pB;
+                if (p + 1 < np) {
+                    pA = (int64_t)(pr >> 32);
+                    pB = (int64_t)(uint32_t)pr;
+                    ra = RA[pA];
+                    rb = RB[pB];
+                    if (p + 2 < np) pr = pp[p + 2];
+                }
+                const bool sa = (ca.w >> 24) & 1u, sb = (cb.w >> 24) & 1u;
+                const uint32_t ia = (ca.w >> 16) & 0xffu, ib = (cb.w >> 16) & 0xffu;
+                if (sa && sb) {
+                    if ((ia & 15u) == (ib >> 4)) {
+                        const int r = (int)(ia >> 4);
+                        w[(r >> 1) * T2L] |= (1u << (ib & 15u)) << (16 * (r & 1));
+                    }
+                    continue;
+                }
+                uint32_t cx = (sa ? 1u << (ia & 15u) : (uint32_t)P.colOccA[cA]) & (cb.w & 0xffffu);
+                const uint16_t *mb = P.mB + cB * TILE;
+                const uint16_t *at = P.mTA + cA * TILE;
+                while (cx) {
+                    const int c = __ffs(cx) - 1;
+                    cx &= cx - 1;
+                    const uint32_t bits = sb ? 1u << (ib & 15u) : (uint32_t)mb[c];
+                    uint32_t rows = sa ? 1u << (ia >> 4) : (uint32_t)at[c];
+                    while (rows) {
+                        const int r = __ffs(rows) - 1;
+                        rows &= rows - 1;
+                        w[(r >> 1) * T2L] |= bits << (16 * (r & 1));
+                    }
+                }
             }
-            const uint16_t *mb = P.mB + cB * TILE;
-            const uint16_t *at = P.mTA + cA * TILE;
-            while (cx) {
-                const int c = __ffs(cx) - 1;
-                cx &= cx - 1;
-                const uint32_t bits = mb[c];
-                uint32_t rows = at[c];
-                while (rows) {
-                    const int r = __ffs(rows) - 1;
-                    rows &= rows - 1;
-                    w[(r >> 1) * T2L] |= bits << (16 * (r & 1));
+        } else {
+            uint64_t pr = pp[0];
+            int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
+            uint32_t x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
+            if (np > 1) pr = pp[1];
+            for (uint32_t p = 0; p < np; p++) {
+                const int64_t cA = pA, cB = pB;
+                uint32_t cx = x;
+                if (p + 1 < np) {
+                    pA = (int64_t)(pr >> 32);
+                    pB = (int64_t)(uint32_t)pr;
+                    x = (uint32_t)P.colOccA[pA] & P.rowOccB[pB];
+                    if (p + 2 < np) pr = pp[p + 2];
+                }
+                const uint16_t *mb = P.mB + cB * TILE;
+                const uint16_t *at = P.mTA + cA * TILE;
+                while (cx) {
+                    const int c = __ffs(cx) - 1;
+                    cx &= cx - 1;
+                    const uint32_t bits = mb[c];
+                    uint32_t rows = at[c];
+                    while (rows) {
+                        const int r = __ffs(rows) - 1;
+                        rows &= rows - 1;
+                        w[(r >> 1) * T2L] |= bits << (16 * (r & 1));
+                    }
                 }
             }
         }
@@ -251,8 +295,19 @@ constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <=
 #ifndef TSG_SMALL_MINB
 #define TSG_SMALL_MINB 5
 #endif
-template <typename TI, typename TO, bool STAGE>
+// REC (hypersparse operands, the default there): per pair the two tiles' 16-byte records; a
+// single-nonzero tile needs nothing else (its entry and value are inline), a multi-nonzero tile
+// its masks and row offsets as in the plain form.
+template <typename TO, typename TI>
+__device__ __forceinline__ TO rec_value(const uint4 &r) {
+    if constexpr (sizeof(TI) == 8) return vcvt<TO>(__hiloint2double((int)r.y, (int)r.x));
+    else if constexpr (sizeof(TI) == 4) return vcvt<TO>(__int_as_float((int)r.x));
+    else return vcvt<TO>(__ushort_as_half((unsigned short)(r.x & 0xffffu)));
+}
+
+template <typename TI, typename TO, int MODE>  // MODE 0: plain, 1: STAGE, 2: REC
 __global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
+    constexpr bool STAGE = MODE == 1;
     __shared__ uint8_t mapsm[TS / 32][SMAP];
     __shared__ __align__(16) uint4 stg[STAGE ? 2 : 1][3][STAGE ? TS : 1];
     const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
@@ -300,7 +355,45 @@ __global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
                 const int j = (int)__fns((uint32_t)P.mC[t * TILE + r], 0, k + 1);
                 const uint32_t lowj = (1u << j) - 1u;
                 TO acc = 0;
-                if constexpr (!STAGE) {
+                if constexpr (MODE == 2) {
+                const uint4 *RA = reinterpret_cast<const uint4 *>(P.recA), *RB = reinterpret_cast<const uint4 *>(P.recB);
+                uint64_t prn = pp[0];
+                int64_t pA = (int64_t)(prn >> 32), pB = (int64_t)(uint32_t)prn;
+                uint4 ra = RA[pA], rb = RB[pB];
+                if (np > 1) prn = pp[1];
+                for (uint32_t p = 0; p < np; p++) {
+                    const uint4 ca = ra, cb = rb;
+                    const int64_t cpA = pA, cpB = pB;
+                    if (p + 1 < np) {  // the next pair's records are loaded while this one multiplies
+                        pA = (int64_t)(prn >> 32);
+                        pB = (int64_t)(uint32_t)prn;
+                        ra = RA[pA];
+                        rb = RB[pB];
+                        if (p + 2 < np) prn = pp[p + 2];
+                    }
+                    const bool sa = (ca.w >> 24) & 1u, sb = (cb.w >> 24) & 1u;
+                    const uint32_t ia = (ca.w >> 16) & 0xffu, ib = (cb.w >> 16) & 0xffu;
+                    if (sa && sb) {
+                        if ((int)(ia >> 4) == r && (ia & 15u) == (ib >> 4) && (int)(ib & 15u) == j)
+                            acc = vfma(rec_value<TO, TI>(ca), rec_value<TO, TI>(cb), acc);
+                        continue;
+                    }
+                    const uint32_t mAr = sa ? ((int)(ia >> 4) == r ? 1u << (ia & 15u) : 0u) : (uint32_t)P.mA[cpA * TILE + r];
+                    const uint32_t mTj = sb ? ((int)(ib & 15u) == j ? 1u << (ib >> 4) : 0u) : (uint32_t)P.mTB[cpB * TILE + j];
+                    uint32_t x = mAr & mTj;
+                    if (!x) continue;
+                    const int64_t zA = sa ? 0 : (int64_t)ca.x + ((int64_t)ca.y << 32) + P.recA_voff + P.rpA[cpA * TILE + r];
+                    const int64_t zB = sb ? 0 : (int64_t)cb.x + ((int64_t)cb.y << 32);
+                    while (x) {
+                        const int c = __ffs(x) - 1;
+                        x &= x - 1;
+                        const TO a = sa ? rec_value<TO, TI>(ca) : vcvt<TO>(vA[zA + __popc(mAr & ((1u << c) - 1u))]);
+                        const TO b = sb ? rec_value<TO, TI>(cb)
+                                        : vcvt<TO>(vB[zB + P.rpB[cpB * TILE + c] + __popc((uint32_t)P.mB[cpB * TILE + c] & lowj)]);
+                        acc = vfma(a, b, acc);
+                    }
+                }
+                } else if constexpr (!STAGE) {
                 // pair p's metadata is loaded while pair p-1 is being multiplied
                 uint64_t prn = pp[0];
                 int64_t pA = (int64_t)(prn >> 32), pB = (int64_t)(uint32_t)prn;
@@ -784,14 +877,18 @@ static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s)
     const int64_t groups = (P.ntC + 31) / 32;
     StepParams Q = P;
     if (P.small_max > 0) {
-        if (P.small_stage) {
-            const Shape sp = step_shape(k_s3_small<TI, TO, true>, TS, groups, P.qoverride);
+        if (P.recA) {
+            const Shape sp = step_shape(k_s3_small<TI, TO, 2>, TS, groups, P.qoverride);
             Q.qchunk[2] = sp.chunk;
-            TSG_LAUNCH((k_s3_small<TI, TO, true>), sp.grid, TS, 0, s, Q);
+            TSG_LAUNCH((k_s3_small<TI, TO, 2>), sp.grid, TS, 0, s, Q);
+        } else if (P.small_stage) {
+            const Shape sp = step_shape(k_s3_small<TI, TO, 1>, TS, groups, P.qoverride);
+            Q.qchunk[2] = sp.chunk;
+            TSG_LAUNCH((k_s3_small<TI, TO, 1>), sp.grid, TS, 0, s, Q);
         } else {
-            const Shape sp = step_shape(k_s3_small<TI, TO, false>, TS, groups, P.qoverride);
+            const Shape sp = step_shape(k_s3_small<TI, TO, 0>, TS, groups, P.qoverride);
             Q.qchunk[2] = sp.chunk;
-            TSG_LAUNCH((k_s3_small<TI, TO, false>), sp.grid, TS, 0, s, Q);
+            TSG_LAUNCH((k_s3_small<TI, TO, 0>), sp.grid, TS, 0, s, Q);
         }
     }
     {
