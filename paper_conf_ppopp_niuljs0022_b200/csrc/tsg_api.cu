@@ -326,7 +326,15 @@ tsg_status tsg_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, co
         tsg_tiles *T = new tsg_tiles();
         T->al = al_;
         try {
-            run_spgemm(A, B, flags, al_, s, T, stats);
+            try {
+                run_spgemm(A, B, flags, al_, s, T, stats);
+            } catch (const Retry &) {
+                // step 1's scratch did not fit the cached arena (first call of a larger problem):
+                // the arena grows on entry to the second attempt
+                const int64_t syncs0 = 1;
+                run_spgemm(A, B, flags, al_, s, T, stats);
+                if (stats) stats->host_syncs += (int32_t)syncs0;
+            }
         } catch (...) {
             destroy_handle(T, s);
             throw;

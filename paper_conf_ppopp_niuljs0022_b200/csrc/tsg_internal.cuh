@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <atomic>
 #include <string>
 #include <vector>
@@ -24,6 +25,8 @@ struct Error {
     tsg_status status;
     std::string msg;
 };
+// a call whose optimistically sized scratch overflowed: redo it once (the arena has grown)
+struct Retry {};
 
 void set_last_error(const std::string &msg);
 
@@ -89,6 +92,7 @@ struct Arena {
     int dev = -1;
     char *base = nullptr;
     size_t cap = 0, off = 0, want = 0;
+    int64_t u_hint = 0;  // step-1 candidates to reserve scratch for (the largest call seen)
     cudaEvent_t done = nullptr;
     cudaStream_t last = nullptr;
     int depth = 0;
@@ -152,6 +156,14 @@ class Buffers {
     }
     // bytes handed out by get() so far (scratch is a stack within a call: this is its peak)
     size_t handed() const { return handed_; }
+    // the cached arena: whether this list draws from it, its free bytes, and a request that the
+    // next call find at least `bytes` more free than this one had (the arena grows on entry)
+    bool arena_backed() const { return arena_ != nullptr; }
+    size_t arena_free() const { return arena_ && arena_->off < arena_->cap ? arena_->cap - arena_->off : 0; }
+    void arena_need(size_t bytes) {
+        if (arena_) arena_->want = std::max(arena_->want, arena_->off + bytes);
+    }
+    int64_t *arena_hint() { return arena_ ? &arena_->u_hint : nullptr; }
 
    private:
     void enter_arena();

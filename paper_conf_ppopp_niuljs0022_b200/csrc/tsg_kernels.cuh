@@ -24,6 +24,9 @@ struct DevCounters {
     u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
     u64c n2dense;      // C tiles with nnz >= t_nnz (step 2 counts them; step 3 launches the dense kernel iff > 0)
     u64c structural;   // |C'| (TSG_STATS_STRUCTURAL)
+    u64c nsmall;       // rows sorted in shared memory (their list: smallList)
+    u64c overflow;     // step 1's candidate scratch was too small (the call is redone with a larger arena)
+    u64c next_small, next_big;  // work counters of the persistent step-1 kernels
     u64c q[5][16];     // work-queue counters of the step-2/3 kernels, one 128-byte line each
 };
 
@@ -74,6 +77,9 @@ struct S1Params {
     int64_t *nC;       // [tm]    C tiles of the row
     const int32_t *bigList;
     const int64_t *bigOff;
+    const int32_t *smallList;
+    const int64_t *utot;   // the candidate total (costOff[ntA]), read on the device
+    int64_t capU, capBig;  // capacity of the candidate-space and wide-row scratch (elements)
     uint64_t *bigKeysA, *bigKeysB;
     uint32_t *bigPosB, *bigKpos;
     DevCounters *cnt;
@@ -157,9 +163,11 @@ void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA,
                        int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s);
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
                      const int32_t *jhiA, bool merge, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass,
-                     int64_t *nC, int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s);
-void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
+                     int64_t *nC, int32_t *bigList, int64_t *bigOff, int32_t *smallList, DevCounters *cnt,
                      cudaStream_t s);
+// step 1 of the per-C-tile path; the row-class counts are read on the device (persistent grids
+// over the class lists), so no host read is needed before it
+void launch_row_sort(const S1Params &P, int64_t tm, cudaStream_t s);
 void launch_sym_rows(const S1Params &P, int64_t tm, cudaStream_t s);
 void launch_row_products(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const uint16_t *maskA, int64_t tmB,
                          const int64_t *tpB, const uint16_t *maskB, int32_t *rnnz, int64_t *w, cudaStream_t s);

@@ -297,8 +297,6 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
     unsigned char *wr = ws + OFF_WORK;
     TO *acc = reinterpret_cast<TO *>(wr) + half * 256 + r;
     MedStage &S = reinterpret_cast<MedStage *>(wr + ACC_BYTES)[half];
-    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
-    TO *vC = static_cast<TO *>(P.vC);
 
     int64_t t0 = 0, nC = 0, a0 = 0, base = 0, zrow = 0;
     int nA = 0;

@@ -218,16 +218,19 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     int64_t *nC = tmp.get<int64_t>(tmA + 1);
     int32_t *bigList = tmp.get<int32_t>(tmA);
     int64_t *bigOff = tmp.get<int64_t>(tmA);
+    int32_t *smallList = tmp.get<int32_t>(tmA);
     launch_row_plan(tmA, A->tile_ptr, costOff, jloA, jhiA, !(flags & TSG_STEP1_SORT_ONLY), rowJlo, rowJhi, rowClass,
-                    nC, bigList, bigOff, cnt, s);
-    // blocking read #1: candidate total and row classes (sizes of the step-1 scratch)
-    DevCounters hc{};
-    int64_t Utot = 0;
-    read_device({{&Utot, costOff + ntA, sizeof(int64_t)}, {&hc, cnt, sizeof(DevCounters)}}, s);
-    syncs++;
-    TSG_REQUIRE(Utot < ((int64_t)1 << 40), TSG_ERR_OVERFLOW, "too many step-1 candidates");
+                    nC, bigList, bigOff, smallList, cnt, s);
     tm_.mark(2);
 
+    // ---------------- a1: step 1 (both paths): exact C tile layout + pairs, per row class
+    // Its scratch (24 B per candidate in the candidate space, 24 B per candidate of the wide rows)
+    // is sized from the free part of the call's cached arena: the candidate total is only read
+    // with C's tile count afterwards (the paper's allocation points, are the two
+    // reads).  The kernels check the true total on the device; if it did not fit -- the first
+    // call of a larger problem -- the call is redone with the arena grown to the need.  A caller
+    // allocator (no arena) reads the total first instead (one more blocking read).
+    nv.push("tsg a1 step 1: tile layout + pairs");
     S1Params P1{};
     P1.tpA = A->tile_ptr;
     P1.tnzA = A->tile_nnz;
@@ -242,45 +245,80 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.rowClass = rowClass;
     P1.tnB = B->tn;
     P1.sort_only = (flags & TSG_STEP1_SORT_ONLY) ? 1 : 0;
-    P1.pairs = tmp.get<uint64_t>(Utot);
-    P1.tJ = tmp.get<int32_t>(Utot);
-    P1.tStart = tmp.get<uint32_t>(Utot);
-    P1.tCnt = tmp.get<uint32_t>(Utot);
-    P1.tWork = tmp.get<uint32_t>(Utot);
+    P1.utot = costOff + ntA;
+    int64_t capU;
+    if (tmp.arena_backed()) {
+        // reserve for the largest candidate total seen (not all of the free arena: the rest of
+        // the call draws from it too)
+        const size_t slack = 16 * 256;  // alignment of the nine arrays
+        const size_t freeb = tmp.arena_free();
+        const int64_t fit = freeb > slack ? (int64_t)((freeb - slack) / 48) : 0;
+        capU = std::min<int64_t>(fit, std::max<int64_t>(*tmp.arena_hint(), 1 << 16));
+    } else {
+        int64_t u = 0;
+        read_device({{&u, costOff + ntA, sizeof(int64_t)}}, s);
+        syncs++;
+        capU = u;
+    }
+    capU = std::max<int64_t>(capU, 1);
+    P1.capU = P1.capBig = capU;
+    P1.pairs = tmp.get<uint64_t>(capU);
+    P1.tJ = tmp.get<int32_t>(capU);
+    P1.tStart = tmp.get<uint32_t>(capU);
+    P1.tCnt = tmp.get<uint32_t>(capU);
+    P1.tWork = tmp.get<uint32_t>(capU);
+    P1.bigKeysA = tmp.get<uint64_t>(capU);
+    P1.bigKeysB = tmp.get<uint64_t>(capU);
+    P1.bigPosB = tmp.get<uint32_t>(capU);
+    P1.bigKpos = tmp.get<uint32_t>(capU);
     P1.nC = nC;
     P1.bigList = bigList;
     P1.bigOff = bigOff;
+    P1.smallList = smallList;
     P1.cnt = cnt;
     P1.mA = A->mask;
     P1.mB = B->mask;
+    launch_row_sort(P1, tmA, s);
+    int64_t *tile_ptr = out.get<int64_t>(tmA + 1);
+    exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
+    // blocking read #1: C's tile count, the candidate total, the row classes
+    DevCounters hc{};
+    int64_t Utot = 0, ntC = 0, nnzC = 0;
+    read_device({{&ntC, tile_ptr + tmA, sizeof(int64_t)}, {&Utot, costOff + ntA, sizeof(int64_t)},
+                 {&hc, cnt, sizeof(DevCounters)}}, s);
+    syncs++;
+    TSG_REQUIRE(Utot < ((int64_t)1 << 40), TSG_ERR_OVERFLOW, "too many step-1 candidates");
+    if (hc.overflow) {
+        const int64_t need = (int64_t)std::max<u64c>((u64c)Utot, hc.big_u);
+        *tmp.arena_hint() = std::max(*tmp.arena_hint(), need);
+        tmp.arena_need((size_t)48 * (size_t)need + ((size_t)1 << 20));
+        throw Retry{};
+    }
+    if (tmp.arena_backed()) *tmp.arena_hint() = std::max(*tmp.arena_hint(), Utot);
+    TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
+    tm_.mark(3);
 
     // the row path needs every non-empty tile row to be a merge row (<= 32 A tiles).  It wins where
-    // the call is small (fewer launches and blocking reads: C1) or A's tiles are dense enough to
-    // make dense C tiles common (C3: 0.89 vs 1.0 ms); on sparse-tile stencils (C2: 17 nnz per A
-    // tile) the per-C-tile kernels run at higher occupancy and are faster
+    // the call is small (fewer launches: C1) or A's tiles are dense enough to make dense C tiles
+    // common (C3: 0.89 vs 1.0 ms); on sparse-tile stencils (C2: 17 nnz per A tile) the per-C-tile
+    // kernels run at higher occupancy and are faster
     const bool narrow = !(flags & (TSG_PATH_GENERAL | TSG_STEP1_SORT_ONLY)) && hc.nbig == 0 && hc.max_u_small == 0 &&
                         tmA > 0;
     const bool rowpath = narrow && ((flags & TSG_PATH_ROWS_FORCE) || A->nnz >= 32 * A->nt || Utot <= ROWPATH_SMALL_U);
-    int64_t ntC = 0, nnzC = 0;
-    int64_t *tile_ptr = out.get<int64_t>(tmA + 1);
     if (rowpath) {
         P1.sMaskC = tmp.get<uint16_t>(TILE * Utot);
         P1.sRowPtrC = tmp.get<uint8_t>(TILE * Utot);
         P1.rowNnz = tmp.get<int64_t>(tmA);
         P1.dense_threshold = TH;
-        nv.push("tsg a1+a2 row path: tile layout, pairs, masks");
+        nv.push("tsg a2 row path: masks per tile row");
         launch_sym_rows(P1, tmA, s);
-        tm_.mark(3);
-        // ---------------- a3: tile and nonzero offsets of the rows; the one allocation of C
-        nv.push("tsg a3 scans + allocation");
+        // ---------------- a3: nonzero offsets of the rows; the one allocation of C
+        nv.push("tsg a3 scan + allocation");
         int64_t *rowOff = tmp.get<int64_t>(tmA + 1);
-        exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
         exclusive_scan<int64_t>(P1.rowNnz, rowOff, tmA, s, tmp);
         DevCounters hc2{};
-        read_device({{&ntC, tile_ptr + tmA, sizeof(int64_t)}, {&nnzC, rowOff + tmA, sizeof(int64_t)},
-                     {&hc2, cnt, sizeof(DevCounters)}}, s);
+        read_device({{&nnzC, rowOff + tmA, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
         syncs++;
-        TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
         C->tile_col = out.get<int32_t>(ntC);
         C->tile_nnz = out.get<int64_t>(ntC + 1);
         C->row_ptr = out.get<uint8_t>(TILE * ntC);
@@ -327,20 +365,6 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         }
         tm_.mark(5);
     } else {
-        if (hc.nbig > 0) {
-            P1.bigKeysA = tmp.get<uint64_t>(hc.big_u);
-            P1.bigKeysB = tmp.get<uint64_t>(hc.big_u);
-            P1.bigPosB = tmp.get<uint32_t>(hc.big_u);
-            P1.bigKpos = tmp.get<uint32_t>(hc.big_u);
-        }
-        nv.push("tsg a1 step 1: tile layout + pairs");
-        launch_row_sort(P1, tmA, (int64_t)hc.max_u_small, (int64_t)hc.nbig, (int64_t)hc.nmerge, s);
-        exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
-        // blocking read #2: number of C tiles
-        ntC = read_scalar(tile_ptr + tmA, s);
-        syncs++;
-        TSG_REQUIRE(ntC < ((int64_t)1 << 32), TSG_ERR_OVERFLOW, "C has >= 2^32 tiles");
-        tm_.mark(3);
         // C's tile arrays, per-tile pair ranges
         int32_t *tile_col = out.get<int32_t>(ntC);
         int64_t *tile_nnz = out.get<int64_t>(ntC + 1);
@@ -463,9 +487,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         st->ms_host_alloc = (float)t_host_alloc_ms;
         if (tm_.on) {
             st->ms_index = tm_.ms(0, 1);
-            st->ms_step1 = tm_.ms(1, 2) + (rowpath ? 0.f : tm_.ms(2, 3));
-            st->ms_step2 = rowpath ? tm_.ms(2, 3) : tm_.ms(3, 4);
-            st->ms_alloc = rowpath ? tm_.ms(3, 4) : 0.f;
+            st->ms_step1 = tm_.ms(1, 3);  // plan + step 1 (+ blocking read #1)
+            st->ms_step2 = tm_.ms(3, 4);  // step 2 (masks), the nonzero scan, read #2, allocation of C
+            st->ms_alloc = 0.f;
             st->ms_step3 = tm_.ms(4, 5);
             st->ms_total = tm_.ms(0, 5);
         }

@@ -247,7 +247,7 @@ __global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const i
                            const int32_t *__restrict__ jloA, const int32_t *__restrict__ jhiA, bool merge,
                            int32_t *__restrict__ rowJlo, int32_t *__restrict__ rowJhi, uint8_t *__restrict__ rowClass,
                            int64_t *__restrict__ nC, int32_t *__restrict__ bigList, int64_t *__restrict__ bigOff,
-                           DevCounters *cnt) {
+                           int32_t *__restrict__ smallList, DevCounters *cnt) {
     const int lane = threadIdx.x & 31;
     const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (I >= tmA) return;
@@ -281,6 +281,7 @@ __global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const i
     if (U <= ROW_CAP && wb + ub <= 32 && (a1 - a0) < 65536) {
         rowClass[I] = ROW_SMALL;
         atomicMax(&cnt->max_u_small, (u64c)U);
+        smallList[atomicAdd(&cnt->nsmall, 1ULL)] = (int32_t)I;
     } else {
         rowClass[I] = ROW_BIG;
         u64c k = atomicAdd(&cnt->nbig, 1ULL);
@@ -651,155 +652,25 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
     if (I >= tm || P.rowClass[I] != ROW_MERGE) return;  // warp-uniform
+    if (*P.utot > P.capU) {  // (scratch_fits, per warp)
+        if (lane == 0) P.cnt->overflow = 1;
+        return;
+    }
     merge_row(P, I, lane, sJ[w], sK[w]);
 }
 
 // ------------------------------------------------------------------------------------------
-// a1 + a2 fused (the row path: every tile row has <= 32 A tiles).  One warp per tile row: the
-// k-way merge above gives the row's C tiles and their contributing pairs (step 1), then, with the
-// row's A masks staged once in shared memory, each C tile's bit masks are OR-ed from its pairs
-// (step 2, Alg 2 l.19-25: mask_C[r] |= mask_B[c] for every nonzero (r,c) of A_IK) by
-// a half warp with lane r owning row r (no atomics), followed by the 16-entry row offsets and the
-// tile nnz.  Results go to the row's candidate-space slots (C is allocated once, after this
-// kernel); the row's nnz total goes to rowNnz[I] for the row-offset scan.
+// a2 on the row path (every tile row has <= 32 A tiles).  One warp per tile row: with the row's A
+// masks staged once in shared memory, each C tile's bit masks are OR-ed from its pairs (written by
+// step 1 at the row's candidate-space slots; Alg 2 l.19-25: mask_C[r] |= mask_B[c]
+// for every nonzero (r,c) of A_IK) by a half warp with lane r owning row r (no atomics), followed
+// by the 16-entry row offsets and the tile nnz.  Results stay at the row's candidate-space slots
+// (C is allocated once, after this kernel); the row's nnz total goes to rowNnz[I] for
+// the row-offset scan, the count of dense C tiles to the call's counters.
 // ------------------------------------------------------------------------------------------
-// Step 1 of one narrow tile row by bitmap ranks instead of the merge's serial steps (a warp, no
-// barriers): (1) every lane walks its A tile's candidate list and marks the tile columns J that
-// have a product (reading B3) in a bitmap over the row's J window; (2) a popcount prefix over the
-// words gives every marked J its rank = its C tile's index in the row (tile columns ascend, as
-// P:801-804 require), and the C tile records' J; (3) each candidate ORs its lane bit into its C
-// tile's lane mask -- lane order is ascending K, so a pair's slot in its tile's list is the tile's
-// start + the contributors on lower lanes (reading A8); (4) a scan of the masks' popcounts gives
-// the starts, (5) every candidate writes its pair.  Returns the row's C tile count, or ~0u when
-// the row has more than RK_MAXC C tiles (the caller falls back to the merge).  Same outputs, in
-// the same candidate-space slots, as merge_row.
-constexpr int RK_MAXU = 1024;  // candidates of the row (packed: jr or rank << 10 | k)
-constexpr int RK_WORDS = 256;  // bitmap words: a J window of <= 8192 tile columns
-constexpr int RK_MAXC = 512;   // C tiles of the row
-struct RankSmem {
-    uint32_t cand[RK_MAXU];
-    uint32_t bm[RK_WORDS];
-    uint32_t lm[RK_MAXC];
-    uint16_t pre[RK_WORDS];
-    uint16_t ps[RK_MAXC];
-};
-static_assert(sizeof(RankSmem) >= MERGE_CAP * 6, "the merge's staging fits the rank's");
-
-__device__ uint32_t rank_row(const S1Params &P, int64_t I, int lane, RankSmem &R) {
-    constexpr uint32_t BAD = 0xffffffffu;
-    const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
-    const int64_t base = P.costOff[a0];
-    const int32_t jlo = P.rowJlo[I];
-    const int words = (P.rowJhi[I] - jlo + 32) >> 5;
-    const int64_t t = a0 + lane;
-    int len = 0, off = 0;
-    int64_t st = 0;
-    bool isl = false;
-    uint32_t co = 0;
-    if (t < a1) {
-        off = (int)(P.costOff[t] - base);
-        len = (int)(P.costOff[t + 1] - base - off);
-        st = P.startA[t];
-        isl = st < 0;
-        if (isl) st = -st - 1;
-        co = P.colOccA[t];
-    }
-    const uint32_t *lst = isl ? P.list + st : nullptr;
-    const uint32_t st32 = (uint32_t)st;
-    for (int w = lane; w < words; w += 32) R.bm[w] = 0;
-    __syncwarp();
-    // (1) mark
-    uint32_t *cand = R.cand + off;
-#pragma unroll 4
-    for (int k = 0; k < len; k++) {
-        const uint32_t pos = isl ? lst[k] : st32 + (uint32_t)k;
-        const bool valid = isl || (co & (uint32_t)P.rowOccB[pos]) != 0;
-        uint32_t x = BAD;
-        if (valid) {
-            const uint32_t jr = (uint32_t)(P.tcB[pos] - jlo);
-            x = jr << 10 | (uint32_t)k;
-            atomicOr(&R.bm[jr >> 5], 1u << (jr & 31));
-        }
-        cand[k] = x;
-    }
-    __syncwarp();
-    // (2) ranks of the marked columns: word popcount prefix; the C tile records' J
-    uint32_t run = 0;
-    for (int w0 = 0; w0 < words; w0 += 32) {
-        const int w = w0 + lane;
-        const uint32_t bw = w < words ? R.bm[w] : 0u;
-        const uint32_t c = __popc(bw);
-        uint32_t incl = c;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t o = __shfl_up_sync(FULL, incl, d);
-            if (lane >= d) incl += o;
-        }
-        const uint32_t pre = run + incl - c;
-        if (w < words) R.pre[w] = (uint16_t)min(pre, 0xffffu);
-        run += __shfl_sync(FULL, incl, 31);
-        if (run <= (uint32_t)RK_MAXC) {
-            uint32_t m = bw, q = pre;
-            while (m) {
-                const int b = __ffs(m) - 1;
-                m &= m - 1;
-                P.tJ[base + q++] = jlo + 32 * w + b;
-            }
-        }
-    }
-    const uint32_t nC = run;
-    if (nC > (uint32_t)RK_MAXC) return ~0u;  // warp-uniform
-    for (uint32_t q = lane; q < nC; q += 32) R.lm[q] = 0;
-    __syncwarp();
-    // (3) contributors of every C tile, as lane masks (lane order = ascending K)
-    for (int k = 0; k < len; k++) {
-        const uint32_t x = cand[k];
-        if (x == BAD) continue;
-        const uint32_t jr = x >> 10;
-        const uint32_t rk = R.pre[jr >> 5] + __popc(R.bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
-        cand[k] = rk << 10 | (x & 1023u);
-        atomicOr(&R.lm[rk], 1u << lane);
-    }
-    __syncwarp();
-    // (4) pair starts of the C tiles (row-relative), pair counts
-    uint32_t np = 0;
-    for (uint32_t q0 = 0; q0 < nC; q0 += 32) {
-        const uint32_t q = q0 + lane;
-        const uint32_t c = q < nC ? __popc(R.lm[q]) : 0u;
-        uint32_t incl = c;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t o = __shfl_up_sync(FULL, incl, d);
-            if (lane >= d) incl += o;
-        }
-        if (q < nC) {
-            const uint32_t pst = np + incl - c;
-            R.ps[q] = (uint16_t)pst;
-            P.tStart[base + q] = pst;
-            P.tCnt[base + q] = c;
-        }
-        np += __shfl_sync(FULL, incl, 31);
-    }
-    __syncwarp();
-    // (5) the pairs, (posA << 32) | posB, in ascending K within every C tile
-    const unsigned lt = (1u << lane) - 1u;
-    const uint64_t thi = (uint64_t)t << 32;
-    for (int k = 0; k < len; k++) {
-        const uint32_t x = cand[k];
-        if (x == BAD) continue;
-        const uint32_t rk = x >> 10, kk = x & 1023u;
-        const uint32_t pos = isl ? lst[kk] : st32 + kk;
-        P.pairs[base + R.ps[rk] + __popc(R.lm[rk] & lt)] = thi | pos;
-    }
-    if (lane == 0) {
-        P.nC[I] = nC;
-        atomicAdd(&P.cnt->pairs, (u64c)np);
-    }
-    return nC;
-}
-
+constexpr int SYM_SMEM = 1024 + 2 * 576;  // per warp: A row masks [32][16], two half-warp batches
 __global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t tm) {
-    __shared__ __align__(16) RankSmem sR[MERGE_W];
+    __shared__ __align__(16) unsigned char sR[MERGE_W][SYM_SMEM];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
     if (I >= tm) return;  // warp-uniform
@@ -807,23 +678,13 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t t
         if (lane == 0) P.rowNnz[I] = 0;
         return;
     }
-    uint32_t nC = ~0u;
-    {
-        const int64_t a0 = P.tpA[I];
-        const int64_t U = P.costOff[P.tpA[I + 1]] - P.costOff[a0];
-        if (U <= RK_MAXU && P.rowJhi[I] - P.rowJlo[I] < 32 * RK_WORDS) nC = rank_row(P, I, lane, sR[w]);
-    }
-    __syncwarp();
-    if (nC == ~0u)
-        nC = merge_row(P, I, lane, reinterpret_cast<uint32_t *>(&sR[w]),
-                       reinterpret_cast<uint16_t *>(reinterpret_cast<uint32_t *>(&sR[w]) + MERGE_CAP));
-    __syncwarp();  // the row's pairs and C tile records (global) are visible to the whole warp
+    const uint32_t nC = (uint32_t)P.nC[I];  // step 1 (k_row_merge) wrote the row's C tiles and pairs
     const int64_t a0 = P.tpA[I];
     const int nA = (int)(P.tpA[I + 1] - a0);
     const int64_t base = P.costOff[a0];
     // staging area (reuses the merge's): A row masks [32][16], then per half warp the B masks,
     // B row occupancy and A slots of a batch of 16 pairs
-    unsigned char *wsm = reinterpret_cast<unsigned char *>(&sR[w]);
+    unsigned char *wsm = sR[w];
     uint16_t *sMA = reinterpret_cast<uint16_t *>(wsm);
     if (lane < nA) {
         const uint4 *g = reinterpret_cast<const uint4 *>(P.mA + (a0 + lane) * TILE);
@@ -900,28 +761,58 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t t
     }
 }
 
-__global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int64_t tm, int cap) {
+// step 1's scratch was sized from the free part of the call's arena before the candidate total
+// was known on the host: every step-1 kernel checks it on the device and, if it does not fit, flags
+// the call (read with C's tile count) and does nothing -- the host grows the arena and redoes
+__device__ __forceinline__ bool scratch_fits(const S1Params &P) {
+    const bool ok = *P.utot <= P.capU && (int64_t)P.cnt->big_u <= P.capBig;
+    if (!ok && threadIdx.x == 0) P.cnt->overflow = 1;
+    return ok;
+}
+
+__global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int cap) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t hist[256 * ROW_NW];
     __shared__ int sm[ROW_NW + 1];
-    const int64_t I = blockIdx.x;
-    if (I >= tm || P.rowClass[I] != ROW_SMALL) return;
+    if (!scratch_fits(P)) return;
     uint32_t *keysA = reinterpret_cast<uint32_t *>(smem);
     uint32_t *keysB = keysA + cap;
     uint32_t *posB = keysB + cap;
     uint16_t *kpos = reinterpret_cast<uint16_t *>(posB + cap);
-    const int64_t U = P.costOff[P.tpA[I + 1]] - P.costOff[P.tpA[I]];
-    const int ub = bits_for((uint64_t)(U > 1 ? U - 1 : 1));
-    row_sort_body<uint32_t, uint16_t>(P, I, keysA, keysB, posB, kpos, hist, sm, ub);
+    const int64_t n = (int64_t)P.cnt->nsmall;
+    __shared__ int64_t kk;
+    for (;;) {  // persistent over the small rows, one at a time from a counter
+        if (threadIdx.x == 0) kk = (int64_t)atomicAdd(&P.cnt->next_small, 1ULL);
+        __syncthreads();
+        const int64_t k = kk;
+        __syncthreads();
+        if (k >= n) break;
+        const int64_t I = P.smallList[k];
+        const int64_t U = P.costOff[P.tpA[I + 1]] - P.costOff[P.tpA[I]];
+        const int ub = bits_for((uint64_t)(U > 1 ? U - 1 : 1));
+        row_sort_body<uint32_t, uint16_t>(P, I, keysA, keysB, posB, kpos, hist, sm, ub);
+        __syncthreads();
+    }
 }
 
 __global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) {
     __shared__ uint32_t hist[256 * ROW_NW];
     __shared__ int sm[ROW_NW + 1];
-    const int64_t I = P.bigList[blockIdx.x];
-    const int64_t o = P.bigOff[I];
-    row_sort_body<uint64_t, uint32_t>(P, I, P.bigKeysA + o, P.bigKeysB + o, P.bigPosB + o, P.bigKpos + o, hist, sm,
-                                      32);
+    if (!scratch_fits(P)) return;
+    const int64_t n = (int64_t)P.cnt->nbig;
+    __shared__ int64_t kk;
+    for (;;) {
+        if (threadIdx.x == 0) kk = (int64_t)atomicAdd(&P.cnt->next_big, 1ULL);
+        __syncthreads();
+        const int64_t k = kk;
+        __syncthreads();
+        if (k >= n) break;
+        const int64_t I = P.bigList[k];
+        const int64_t o = P.bigOff[I];
+        row_sort_body<uint64_t, uint32_t>(P, I, P.bigKeysA + o, P.bigKeysB + o, P.bigPosB + o, P.bigKpos + o, hist,
+                                          sm, 32);
+        __syncthreads();
+    }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -962,11 +853,27 @@ __device__ __forceinline__ int64_t block_excl_scan64(int64_t v, int64_t *total, 
     return res;
 }
 
+__device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t *bm, int64_t *sm);
+
 __global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
     extern __shared__ uint32_t bm[];  // [wwords] bitmap, then [wwords] exclusive popcount prefix
-    uint32_t *pre = bm + wwords;
     __shared__ int64_t sm[RANK_NW + 1];
-    const int64_t I = P.bigList[blockIdx.x];
+    if (!scratch_fits(P)) return;
+    const int64_t n = (int64_t)P.cnt->nbig;
+    __shared__ int64_t kk;
+    for (;;) {  // persistent over the wide rows, one at a time from a counter (they differ widely)
+        if (threadIdx.x == 0) kk = (int64_t)atomicAdd(&P.cnt->next_big, 1ULL);
+        __syncthreads();
+        const int64_t k = kk;
+        __syncthreads();
+        if (k >= n) break;
+        rank_row_big(P, P.bigList[k], wwords, bm, sm);
+        __syncthreads();
+    }
+}
+
+__device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t *bm, int64_t *sm) {
+    uint32_t *pre = bm + wwords;
     const int64_t a0 = P.tpA[I], a1 = P.tpA[I + 1];
     const int nA = (int)(a1 - a0);
     const int64_t base = P.costOff[a0];
@@ -1199,9 +1106,10 @@ void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA,
 
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
                      const int32_t *jhiA, bool merge, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass,
-                     int64_t *nC, int32_t *bigList, int64_t *bigOff, DevCounters *cnt, cudaStream_t s) {
+                     int64_t *nC, int32_t *bigList, int64_t *bigOff, int32_t *smallList, DevCounters *cnt,
+                     cudaStream_t s) {
     TSG_LAUNCH(k_row_plan, grid_for(tmA, 8), 256, 0, s, tmA, tpA, costOff, jloA, jhiA, merge, rowJlo, rowJhi,
-               rowClass, nC, bigList, bigOff, cnt);
+               rowClass, nC, bigList, bigOff, smallList, cnt);
 }
 
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s) {
@@ -1226,25 +1134,31 @@ void launch_sym_rows(const S1Params &P, int64_t tm, cudaStream_t s) {
     TSG_LAUNCH(k_sym_rows, grid_for(tm, MERGE_W), MERGE_W * 32, 0, s, P, tm);
 }
 
-void launch_row_sort(const S1Params &P, int64_t tm, int64_t max_u_small, int64_t nbig, int64_t nmerge,
-                     cudaStream_t s) {
-    if (nmerge > 0) TSG_LAUNCH(k_row_merge, grid_for(tm, MERGE_W), MERGE_W * 32, 0, s, P, tm);
-    if (max_u_small > 0) {
-        const int cap = (int)((max_u_small + 31) & ~31LL);
+void launch_row_sort(const S1Params &P, int64_t tm, cudaStream_t s) {
+    // the row classes' sizes live on the device: the merge covers every row (others exit at once),
+    // the shared-memory sort and the wide-row kernels run persistent grids over their row lists
+    static int nsm = 0;
+    if (!nsm) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        nsm = std::max(nsm, 1);
+    }
+    if (!P.sort_only) TSG_LAUNCH(k_row_merge, grid_for(tm, MERGE_W), MERGE_W * 32, 0, s, P, tm);
+    {
+        const int cap = ROW_CAP;
         const size_t smem = (size_t)cap * (4 + 4 + 4 + 2);
         TSG_CUDA(cudaFuncSetAttribute(k_row_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        TSG_LAUNCH(k_row_small, (unsigned)tm, ROW_T, smem, s, P, tm, cap);
+        TSG_LAUNCH(k_row_small, (unsigned)std::min<int64_t>(tm, 3LL * nsm), ROW_T, smem, s, P, cap);
     }
-    if (nbig > 0) {
-        // bitmap over the J window (<= tile columns of B) in shared memory, else the global sort
-        const int64_t wwords = (P.tnB + 31) / 32;
-        const size_t smem = (size_t)wwords * 8;
-        if (!P.sort_only && smem <= 200 * 1024) {
-            TSG_CUDA(cudaFuncSetAttribute(k_row_rank, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            TSG_LAUNCH(k_row_rank, (unsigned)nbig, RANK_T, smem, s, P, (int)wwords);
-        } else {
-            TSG_LAUNCH(k_row_big, (unsigned)nbig, ROW_T, 0, s, P);
-        }
+    // bitmap over the J window (<= tile columns of B) in shared memory, else the global sort
+    const int64_t wwords = (P.tnB + 31) / 32;
+    const size_t smem = (size_t)wwords * 8;
+    if (!P.sort_only && smem <= 200 * 1024) {
+        TSG_CUDA(cudaFuncSetAttribute(k_row_rank, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        TSG_LAUNCH(k_row_rank, (unsigned)std::min<int64_t>(tm, 4LL * nsm), RANK_T, smem, s, P, (int)wwords);
+    } else {
+        TSG_LAUNCH(k_row_big, (unsigned)std::min<int64_t>(tm, 8LL * nsm), ROW_T, 0, s, P);
     }
 }
 
