@@ -193,10 +193,12 @@ TSG_API tsg_status tsg_csr_to_tiles_typed(int64_t m, int64_t n, int64_t nnz, con
  * fused multiply-add, i.e. ascending global k (reading A8/A16): deterministic run to run.
  * Value types: C's dtype follows tsg_dtype's rules (F16 inputs are widened exactly to fp32 and
  * accumulated with fp32 FMA); mixed input dtypes are INVALID_ARG.
- * Syncs: blocking scalar reads through mapped host memory -- 2 on the row path (the step-1 candidate
- * total after the plan; C's tile count and nnz(C) together after the fused steps 1-2, the paper's single
- * allocation point P:982-988), 3 on the per-C-tile path (candidate total, C tile count, nnz(C)); one more
- * at the end when `stats` is non-NULL.
+ * Syncs: 2 blocking scalar reads (through mapped host memory), the paper's allocation points
+ * (P:982-988): after step 1 (C's tile count, with the step-1 candidate total) and after step 2
+ * (nnz(C)).  Step 1's scratch is reserved from the calling thread's cached workspace before its
+ * size is known; when it does not fit (the first call of a larger problem) the call is redone
+ * once with the workspace grown (+1 read).  With a caller allocator (no workspace) the candidate
+ * total is read first (+1).  One more read at the end when `stats` is non-NULL (not counted).
  * Alignment: mask and row_ptr of A and B must be 16-byte aligned, val 8-byte aligned (tiles are
  * staged into shared memory in 16-byte chunks); handles made by this library always are.
  * Errors: INVALID_ARG (incl. alignment), SHAPE, OVERFLOW, OOM, CUDA, INTERNAL.
