@@ -290,6 +290,25 @@ def test_chained_output_as_input(tsg):
     assert_tiles_equal(host(C3), ref)
 
 
+def test_galerkin_rap_chain(tsg):
+    """The paper's AMG motivation for a tile-resident format: the Galerkin coarse
+    operator P^T (A P) with a piecewise-constant aggregation prolongator, every product fed the
+    previous one's tiles (and P^T from tsg_tiles_transpose) without conversion; equal to the
+    oracle's chain in fma mode."""
+    A = gen.poisson2d(32)
+    n, nc = A.m, A.m // 4
+    rows = np.arange(n)
+    P = gen.from_coo(n, nc, rows, rows // 4, np.full(n, 0.5), name="aggregation")
+    TA, TP = tiles_of(tsg, A), tiles_of(tsg, P)
+    AP = tsg.spgemm(TA, TP)
+    RAP = tsg.spgemm(tsg.transpose(TP), AP)
+    ap = oracle.spgemm(A, P, fma=True)
+    APc = gen.CSR(ap.m, ap.n, ap.rowptr, ap.col, ap.val)
+    ref = oracle.expected_tiles(oracle.transpose(P), APc, fma=True)
+    assert (RAP.m, RAP.n) == (nc, nc)
+    assert_tiles_equal(host(RAP), ref)
+
+
 def test_slice_rows_and_wrap(tsg):
     A = gen.rmat(11)
     T = tiles_of(tsg, A)
