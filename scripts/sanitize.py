@@ -1,6 +1,7 @@
 """Small C = A*B cases through every kernel class, for compute-sanitizer (memcheck / racecheck /
 synccheck): stencil, FEM strip (dense tiles), R-MAT (hub rows, staged small tiles), row slices,
-transpose, precision variants, tiles -> CSR."""
+transpose, precision variants, tiles -> CSR; both pipelines, the scratch retry, the tile records of
+hypersparse operands, the structural diagnostic and the device partition (round 2)."""
 import sys
 import numpy as np
 import torch
@@ -17,8 +18,13 @@ def tiles(A, dt=np.float64):
 for A in (gen.config("C1"), gen.stencil27(8), gen.strip_fem(6, 12, 6), gen.rmat(10),
           gen.hub(4096, hub_rows=(0, 3000), hub_cols=(0, 5), density=0.002)):
     T = tiles(A)
+    tsg.workspace_release()  # the first call overflows the arena and is redone (the retry path)
     C = tsg.spgemm(T, T, stats=True)
+    for opts in (dict(path_rows=True), dict(path_general=True), dict(dense_threshold=1, path_rows=True),
+                 dict(structural=True, products=True, stats=True), dict(small_stage=True), dict(sort_only=True)):
+        tsg.spgemm(T, T, **opts)
     S = tsg.spgemm(tsg.slice_rows(T, 1, max(2, T.tile_m // 2)), T)
+    tsg.partition_tile_rows(T, T, 3)
     D = tsg.spgemm(T, tsg.transpose(T))
     rp, ci, v = tsg.tiles_to_csr(C)
     C32 = tsg.spgemm(tiles(A, np.float32), tiles(A, np.float32))
