@@ -175,7 +175,7 @@ void launch_cuts(const int64_t *pre, int64_t tm, int64_t parts, int64_t *cuts, c
 bool launch_structural(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const int64_t *tpB, const int32_t *tcB,
                        int64_t tnB, DevCounters *cnt, cudaStream_t s);
 void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStream_t s);
-void launch_compact(const CompactParams &P, cudaStream_t s);
+void launch_compact(const CompactParams &P, int64_t ntC, cudaStream_t s);
 
 // ---------------- a4 on the row path (tsg_rows.cu)
 struct RowNumArgs {

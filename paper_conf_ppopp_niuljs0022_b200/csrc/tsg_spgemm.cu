@@ -375,7 +375,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         uint32_t *work = tmp.get<uint32_t>(ntC);
         CompactParams PC{tmA, A->tile_ptr, costOff, tile_ptr, P1.tJ, P1.tStart, P1.tCnt, P1.tWork,
                          tile_col, pairBeg, pairCnt, work};
-        launch_compact(PC, s);
+        launch_compact(PC, ntC, s);
 
         // ---------------- a2: step 2
         nv.push("tsg a2 step 2: masks");

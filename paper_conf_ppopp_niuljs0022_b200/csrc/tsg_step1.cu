@@ -885,34 +885,34 @@ __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t 
     uint32_t *sK = P.bigKpos + o;
     for (int w = threadIdx.x; w < wwords; w += RANK_T) bm[w] = 0;
     __syncthreads();
-    // pass 1: expand (load-balanced over the row's candidates), mark the bitmap
-    for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
-        const int64_t target = base + u;
-        int lo = 0, hi = nA - 1;
-        while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (P.costOff[a0 + mid] <= target) lo = mid;
-            else hi = mid - 1;
-        }
-        const int64_t t = a0 + lo;
-        const int64_t s = target - P.costOff[t];
+    // pass 1: expand, mark the bitmap -- a warp per A tile of the row, its lanes over that tile's
+    // candidates (no search for a candidate's owner; R-MAT A tiles hold ~40 candidates each)
+    const int wid = threadIdx.x >> 5, lid = threadIdx.x & 31;
+    for (int k = wid; k < nA; k += RANK_NW) {
+        const int64_t t = a0 + k;
+        const int64_t u0 = P.costOff[t] - base, len = P.costOff[t + 1] - base - u0;
         const int64_t st = P.startA[t];
-        uint32_t posB;
-        bool valid;
-        if (st < 0) {
-            posB = P.list[-st - 1 + s];
-            valid = true;
-        } else {
-            posB = (uint32_t)(st + s);
-            valid = (P.rowOccB[posB] & P.colOccA[t]) != 0;
+        const uint32_t co = P.colOccA[t];
+        for (int64_t s = lid; s < len; s += 32) {
+            const int64_t u = u0 + s;
+            uint32_t posB, occ = 0;
+            bool valid;
+            if (st < 0) {
+                posB = P.list[-st - 1 + s];
+                valid = true;
+            } else {
+                posB = (uint32_t)(st + s);
+                occ = P.rowOccB[posB];
+                valid = (occ & co) != 0;
+            }
+            const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : ~0u;
+            // the candidate's (pair, c) items (step 2's work estimate) ride in the top 5 bits
+            const uint32_t wk = st < 0 ? 1u : (uint32_t)__popc(occ & co);
+            sJ[u] = valid ? jr | (wk << 27) : ~0u;
+            sPos[u] = posB;
+            sK[u] = (uint32_t)k;
+            if (valid) atomicOr(&bm[jr >> 5], 1u << (jr & 31));
         }
-        const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : ~0u;
-        // the candidate's (pair, c) items (step 2's work estimate) ride in the top 5 bits
-        const uint32_t wk = st < 0 ? 1u : (uint32_t)__popc((uint32_t)(P.rowOccB[posB] & P.colOccA[t]));
-        sJ[u] = valid ? jr | (wk << 27) : ~0u;
-        sPos[u] = posB;
-        sK[u] = (uint32_t)lo;
-        if (valid) atomicOr(&bm[jr >> 5], 1u << (jr & 31));
     }
     __syncthreads();
     // ranks: exclusive popcount prefix over the bitmap words (blocked ownership)
@@ -1035,14 +1035,18 @@ __global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint1
 // compaction: per-C-tile arrays (tile column, pair range, work estimate) from the per-row step-1
 // results, one warp per tile row
 // ------------------------------------------------------------------------------------------
+// (ROWCTA: a CTA per tile row, for rows of thousands of C tiles -- R-MAT -- where a warp per row
+// serialises the long rows)
+template <bool ROWCTA>
 __global__ void __launch_bounds__(256) k_compact(CompactParams P) {
-    const int lane = threadIdx.x & 31;
-    const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int lane = ROWCTA ? (int)threadIdx.x : (int)(threadIdx.x & 31);
+    const int step = ROWCTA ? 256 : 32;
+    const int64_t I = ROWCTA ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (I >= P.tm) return;
     const int64_t base = P.costOff[P.tpA[I]];
     const int64_t t0 = P.tilePtrC[I], n = P.tilePtrC[I + 1] - t0;
 #pragma unroll 4
-    for (int64_t r = lane; r < n; r += 32) {
+    for (int64_t r = lane; r < n; r += step) {
         const int64_t slot = base + r, t = t0 + r;
         P.tile_col[t] = P.tJ[slot];
         P.pairBeg[t] = base + P.tStart[slot];
@@ -1116,8 +1120,9 @@ void launch_transpose(const uint16_t *mask, int64_t nt, uint16_t *maskT, cudaStr
     TSG_LAUNCH(k_transpose, grid_for(nt, 256), 256, 0, s, mask, nt, maskT);
 }
 
-void launch_compact(const CompactParams &P, cudaStream_t s) {
-    TSG_LAUNCH(k_compact, grid_for(P.tm, 8), 256, 0, s, P);
+void launch_compact(const CompactParams &P, int64_t ntC, cudaStream_t s) {
+    if (ntC > 512 * P.tm) TSG_LAUNCH(k_compact<true>, (unsigned)P.tm, 256, 0, s, P);
+    else TSG_LAUNCH(k_compact<false>, grid_for(P.tm, 8), 256, 0, s, P);
 }
 
 bool launch_structural(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const int64_t *tpB, const int32_t *tcB,
