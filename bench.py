@@ -206,6 +206,15 @@ def run_reference(args):
     return 0
 
 
+def _non_json(o, path="line"):
+    """Paths of values json cannot encode (a stray tensor in the bench line)."""
+    if isinstance(o, dict):
+        return [p for k, v in o.items() for p in _non_json(v, f"{path}.{k}")]
+    if isinstance(o, (list, tuple)):
+        return [p for i, v in enumerate(o) for p in _non_json(v, f"{path}[{i}]")]
+    return [] if o is None or isinstance(o, (str, int, float, bool)) else [f"{path}: {type(o).__name__}"]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -384,16 +393,16 @@ def main():
         t_r, where = None, "left distributed (each rank owns its tile rows)"
         if K == 1:
             Cl = tsg.spgemm(shards[0], Bt)
-            cb = torch.tensor([sum(v.numel() * v.element_size() for v in Cl.arrays().values())], dtype=torch.int64,
-                              device=dev)
-            dist.all_reduce(cb)
+            c_bytes = torch.tensor([sum(v.numel() * v.element_size() for v in Cl.arrays().values())],
+                                   dtype=torch.int64, device=dev)
+            dist.all_reduce(c_bytes)
             free = torch.tensor([torch.cuda.mem_get_info(dev)[0] // ranks_per_gpu], dtype=torch.int64, device=dev)
             dist.all_reduce(free, op=dist.ReduceOp.MIN)
-            if int(cb.item()) < 0.6 * int(free.item()):
+            if int(c_bytes.item()) < 0.6 * int(free.item()):
                 t_r = timed(lambda: tdist.gatherv_tiles(Cl, 0), reps=2)
-                where = f"gatherv to rank 0 ({int(cb.item()) / 1e9:.2f} GB, count-exact point-to-point)"
+                where = f"gatherv to rank 0 ({int(c_bytes.item()) / 1e9:.2f} GB, count-exact point-to-point)"
             else:
-                where = (f"left distributed: C is {int(cb.item()) / 1e9:.1f} GB, more than 60% of a rank's free "
+                where = (f"left distributed: C is {int(c_bytes.item()) / 1e9:.1f} GB, more than 60% of a rank's free "
                          "device memory")
             del Cl
         multi = {"t_bcast_ms": t_b, "bcast_bytes": int(sum(v.numel() * v.element_size() for v in Bt.arrays().values())),
@@ -600,6 +609,9 @@ def main():
         "multi_gpu": multi,
         "clocks": clocks,
     }
+    bad = _non_json(line)
+    if bad:
+        raise TypeError(f"bench line holds non-JSON values at {bad}")
     print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

@@ -84,6 +84,17 @@ def _unwire(t, k):
     return t.view(torch.uint16) if k == "mask" else t
 
 
+def _wire_dev(dev, group=None):
+    """Device the collectives move bytes on: the tensors' own device, except CUDA tensors under
+    gloo (gloo's point-to-point and all-gather take host tensors only), which stage via host."""
+    import torch
+    import torch.distributed as dist
+
+    if dev.type == "cuda" and dist.get_backend(group) == "gloo":
+        return torch.device("cpu")
+    return dev
+
+
 def _shapes(m, nt, nnz, vdt):
     import torch
 
@@ -107,19 +118,21 @@ def broadcast_tiles(arrays: dict | None, meta: tuple | None, src: int, device, g
         vals = list(meta[:4]) + [codes.index(meta[4]) if len(meta) > 4 else 0]
     else:
         vals = [0, 0, 0, 0, 0]
-    mt = torch.tensor(vals, dtype=torch.int64, device=device)
+    device = torch.device(device)
+    wdev = _wire_dev(device, group)
+    mt = torch.tensor(vals, dtype=torch.int64, device=wdev)
     dist.broadcast(mt, src, group=group)
     m, n, nt, nnz, dc = (int(x) for x in mt.tolist())
     shapes = _shapes(m, nt, nnz, codes[dc])
     out = {}
     for k in ARRAYS:
         if arrays is not None:
-            t = _wire(arrays[k].contiguous())
+            t = _wire(arrays[k].contiguous()).to(wdev)
         else:
-            t = torch.empty(shapes[k][0], dtype=shapes[k][1], device=device)
+            t = torch.empty(shapes[k][0], dtype=shapes[k][1], device=wdev)
         if t.numel():
             dist.broadcast(t, src, group=group)
-        out[k] = _unwire(t, k)
+        out[k] = _unwire(t.to(device), k)
     return (m, n, nt, nnz, codes[dc]), out
 
 
@@ -135,7 +148,7 @@ def _counts(arrays, m_local, group):
     import torch
     import torch.distributed as dist
 
-    dev = arrays["tile_ptr"].device
+    dev = _wire_dev(arrays["tile_ptr"].device, group)
     vdt = str(arrays["val"].dtype).replace("torch.", "")
     mine = torch.tensor([m_local, arrays["tile_col"].numel(), arrays["val"].numel(), _CODES.index(vdt)],
                         dtype=torch.int64, device=dev)
@@ -151,16 +164,18 @@ def allgatherv(t, group=None):
     import torch.distributed as dist
 
     world, rank = dist.get_world_size(group), dist.get_rank(group)
-    src = _wire(t.contiguous())
-    n = torch.tensor([src.numel()], dtype=torch.int64, device=t.device)
+    wdev = _wire_dev(t.device, group)
+    src = _wire(t.contiguous()).to(wdev)
+    n = torch.tensor([src.numel()], dtype=torch.int64, device=wdev)
     sizes = [torch.zeros_like(n) for _ in range(world)]
     dist.all_gather(sizes, n, group=group)
     out = []
     for g in range(world):
         sz = int(sizes[g].item())
-        buf = src if g == rank else torch.empty(sz, dtype=src.dtype, device=t.device)
+        buf = src if g == rank else torch.empty(sz, dtype=src.dtype, device=wdev)
         if sz:
             dist.broadcast(buf, dist.get_global_rank(group, g) if group is not None else g, group=group)
+        buf = buf.to(t.device)
         out.append(buf.view(t.dtype) if t.dtype != src.dtype else buf)
     return out
 
@@ -213,8 +228,9 @@ def gatherv_tiles(C, dst: int = 0, group=None, out_device=None):
     world, rank = dist.get_world_size(group), dist.get_rank(group)
     counts = _counts(arrays, m_local, group)
     glob = (lambda g: dist.get_global_rank(group, g)) if group is not None else (lambda g: g)
+    wdev = _wire_dev(arrays["tile_ptr"].device, group)
     if rank != dst:
-        ops = [dist.P2POp(dist.isend, _wire(arrays[k].contiguous()), glob(dst), group=group)
+        ops = [dist.P2POp(dist.isend, _wire(arrays[k].contiguous()).to(wdev), glob(dst), group=group)
                for k in ARRAYS if arrays[k].numel()]
         for r in dist.batch_isend_irecv(ops) if ops else []:
             r.wait()
@@ -232,19 +248,19 @@ def gatherv_tiles(C, dst: int = 0, group=None, out_device=None):
         bufs = {}
         for k in ARRAYS:
             nel, dt = shapes[k]
-            # receive into the shard's device (NCCL), staged to `dev` afterwards if that differs
-            recv_dev = arrays["tile_ptr"].device
-            bufs[k] = torch.empty(nel, dtype=dt, device=recv_dev)
+            # receive on the wire device (the shard's device under NCCL), staged to `dev`
+            # afterwards if that differs
+            bufs[k] = torch.empty(nel, dtype=dt, device=wdev)
             if nel:
                 ops.append(dist.P2POp(dist.irecv, bufs[k], glob(g), group=group))
         pieces.append(dict(m=m_g, **bufs))
     for r in dist.batch_isend_irecv(ops) if ops else []:
         r.wait()
-    if dev != arrays["tile_ptr"].device:
+    if dev != wdev or dev != arrays["tile_ptr"].device:
         for p in pieces:
             for k in ARRAYS:
                 if p[k].device != dev:
-                    h = torch.empty(p[k].shape, dtype=p[k].dtype, pin_memory=pin)
+                    h = torch.empty(p[k].shape, dtype=p[k].dtype, device=dev, pin_memory=pin)
                     h.copy_(p[k])
                     p[k] = h
     for p in pieces:
