@@ -23,6 +23,7 @@ struct DevCounters {
     u64c n3dense;
     u64c nmerge;       // tile rows of step 1 handled by the warp k-way merge
     u64c n2dense;      // C tiles with nnz >= t_nnz (step 2 counts them; step 3 launches the dense kernel iff > 0)
+    u64c max_a_dense;  // row path: most A tiles in a tile row with dense C tiles
     u64c structural;   // |C'| (TSG_STATS_STRUCTURAL)
     u64c nsmall;       // rows sorted in shared memory (their list: smallList)
     u64c overflow;     // step 1's candidate scratch was too small (the call is redone with a larger arena)
@@ -192,11 +193,12 @@ struct RowNumArgs {
     const int64_t *rowOff;        // [tm+1] exclusive scan of the rows' nnz
     int dense_threshold, small_max;
     int64_t n_dense;              // dense C tiles (counted by k_sym_rows)
-    void *dense;                  // scratch for their records (32 B each)
+    int max_a_dense;              // most A tiles in a tile row with dense C tiles (k_sym_rows)
+    const uint16_t *colOccA;      // column occupancy words of A's tiles
     void *small;                  // scratch for the small C tiles' records (32 B each, <= ntC)
     DevCounters *cnt;
 };
-constexpr int DENSE_REC_BYTES = 32;
+constexpr int ROW_REC_BYTES = 32;
 void launch_num_rows(const RowNumArgs &a, cudaStream_t s);
 
 // launchers (tsg_step23.cu)

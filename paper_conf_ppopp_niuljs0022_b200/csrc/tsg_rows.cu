@@ -57,7 +57,6 @@ struct RowTileRec {  // a C tile left by k_num_rows to k_num_small / k_num_dense
     int64_t slot, off, pairs;
     uint32_t cnt, nz;
 };
-typedef RowTileRec DenseRec;
 
 struct RowNumParams {
     int64_t tm;
@@ -87,7 +86,8 @@ struct RowNumParams {
     uint16_t *mC;
     void *vC;
     int dense_threshold, small_max;
-    DenseRec *dense;  // dense C tiles, for k_num_dense
+    int max_a_dense;     // most A tiles in a tile row that has dense C tiles (sizes k_num_dense_row's staging)
+    const uint16_t *colOccA;  // column occupancy words of A's tiles
     RowTileRec *small;   // small C tiles, for k_num_small
     DevCounters *cnt;
 };
@@ -204,80 +204,6 @@ __device__ __forceinline__ void medium_tile(const RowNumParams &P, bool hv, int6
     __syncwarp();
 }
 
-// dense tile: the whole warp; A and B of each pair staged densely, absent A entries
-// skipped, absent B entries staged as 0 (a finite a adds an exact +-0), a non-finite a falls back
-// to mask-predicated FMAs so Inf*0 never appears
-template <typename TI, typename TO>
-__device__ __forceinline__ void dense_tile(const RowNumParams &P, int64_t pairs, int64_t slot, uint32_t cnt,
-                                           int64_t off, unsigned char *wr, int lane) {
-    constexpr int AP = 17;
-    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
-    TO *Ad = reinterpret_cast<TO *>(wr);
-    TO *Bd = reinterpret_cast<TO *>(wr + 2176);
-    const int r = lane >> 1, h = lane & 1;
-    TO acc[8];
-#pragma unroll
-    for (int j = 0; j < 8; j++) acc[j] = (TO)0;
-    for (uint32_t p = 0; p < cnt; p++) {
-        const uint64_t pr = P.pairs[pairs + p];
-        const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-#pragma unroll
-        for (int e = lane; e < TILE * TILE * (int)sizeof(TO) / 16; e += 32)
-            reinterpret_cast<uint4 *>(Bd)[e] = make_uint4(0u, 0u, 0u, 0u);
-        __syncwarp();
-        bool nf = false;
-        for (int64_t e = P.tnzA[pA] + lane; e < P.tnzA[pA + 1]; e += 32) {
-            const uint32_t ix = P.ixA[e];
-            const TO v = vcvt<TO>(vA[e]);
-            nf |= !isfinite(v);
-            Ad[(ix >> 4) * AP + (ix & 15)] = v;
-        }
-        for (int64_t e = P.tnzB[pB] + lane; e < P.tnzB[pB + 1]; e += 32) {
-            const uint32_t ix = P.ixB[e];
-            Bd[(ix >> 4) * TILE + (ix & 15)] = vcvt<TO>(vB[e]);
-        }
-        const uint32_t mAr = P.mA[pA * TILE + r];
-        const bool anynf = __any_sync(FULL, nf);
-        __syncwarp();
-        if (!anynf) {
-#pragma unroll
-            for (int c = 0; c < TILE; c++) {
-                if ((mAr >> c) & 1u) {
-                    const TO a = Ad[r * AP + c];
-                    TO b[8];
-                    lds8(Bd + c * TILE + 8 * h, b);
-#pragma unroll
-                    for (int jj = 0; jj < 8; jj++) acc[jj] = vfma(a, b[jj], acc[jj]);
-                }
-            }
-        } else {
-            const uint16_t *mbt = P.mB + pB * TILE;
-            for (int c = 0; c < TILE; c++) {
-                if ((mAr >> c) & 1u) {
-                    const TO a = Ad[r * AP + c];
-                    const uint32_t mb = (uint32_t)mbt[c] >> (8 * h);
-#pragma unroll
-                    for (int jj = 0; jj < 8; jj++)
-                        if ((mb >> jj) & 1u) acc[jj] = vfma(a, Bd[c * TILE + 8 * h + jj], acc[jj]);
-                }
-            }
-        }
-        __syncwarp();
-    }
-    const uint32_t mCr = P.sMaskC[slot * TILE + r];
-    const int64_t ob = off + P.sRowPtrC[slot * TILE + r];
-#pragma unroll
-    for (int jj = 0; jj < 8; jj++) {
-        const int j = 8 * h + jj;
-        if ((mCr >> j) & 1u) {
-            const int q = __popc(mCr & ((1u << j) - 1u));
-            P.ixC[ob + q] = (uint8_t)((r << 4) | j);
-            static_cast<TO *>(P.vC)[ob + q] = acc[jj];
-        }
-    }
-    __syncwarp();
-}
-
 // One warp per two consecutive tile rows, half h owning row 2w + h, 16 lanes per row.  The loops
 // over the rows' tiles and pairs are warp-uniform (bounds = the max of the two halves) with
 // full-warp reconvergence after every pair: adjacent tile rows of a stencil have the same
@@ -355,9 +281,9 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
         const bool isD = v && (int)nz >= P.dense_threshold;
         const bool isS = v && !isD && (int)nz <= P.small_max;
         const bool isM = v && !isD && !isS;
-        const unsigned BM = __ballot_sync(FULL, isM), BS = __ballot_sync(FULL, isS), BD = __ballot_sync(FULL, isD);
+        const unsigned BM = __ballot_sync(FULL, isM), BS = __ballot_sync(FULL, isS);
         unsigned bM = (BM >> (16 * half)) & 0xffffu;
-        const unsigned bS = (BS >> (16 * half)) & 0xffffu, bD = (BD >> (16 * half)) & 0xffffu;
+        const unsigned bS = (BS >> (16 * half)) & 0xffffu;
         nmd += __popc(bM);
 
         // ---- medium tiles: each half its next one, in step
@@ -388,20 +314,7 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
             }
         }
 
-        // ---- dense tiles: recorded for k_num_dense (a warp each, after this kernel), so this
-        // kernel's registers are sized for the sparse classes
-        if (BD) {
-            uint32_t di = 0;
-            if (r == 0 && bD) di = (uint32_t)atomicAdd(&P.cnt->n3dense, (u64c)__popc(bD));
-            di = __shfl_sync(FULL, di, 16 * half);
-            if (isD) {
-                DenseRec &d = P.dense[di + __popc(bD & lt)];
-                d.slot = slot;
-                d.off = off;
-                d.pairs = base + st;
-                d.cnt = cn;
-            }
-        }
+        // ---- dense tiles: k_num_dense_row (a CTA per tile row, after this kernel) computes them
     }
     if (r == 0 && nmd) atomicAdd(&P.cnt->n3medium, nmd);
 }
@@ -489,15 +402,152 @@ __global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) {
     }
 }
 
-// dense tiles recorded by k_num_rows: one warp each
+// dense C tiles (nnz >= t_nnz): a CTA per tile row (P:1862-1870 for the accumulator).  The row's
+// A tiles are expanded once into shared memory (16 x 17 values each, absent entries 0), so every
+// dense C tile of the row reuses them -- a pair then moves only its B tile.  Warp 0 walks the
+// row's C tiles 32 at a time (their nnz and nonzero offsets, as k_num_rows computes them) and
+// lists the dense ones; the warps take them in turn.  Per pair the warp expands B_KJ into a 16 x 16
+// buffer (cleared, then scattered), and walks the columns c of colOcc(A_IK) & rowOcc(B_KJ) in
+// ascending order in warp-uniform groups of four (no divergence, immediate-offset shared
+// loads); lane (r, h) adds A(r, c) * B(c, 8h..8h+7) to its eight register accumulators.  The
+// zeros are exact: a finite a times an absent B entry, or 0 times a finite B entry, adds +-0.  A
+// pair with a non-finite value in A_IK or B_KJ instead takes mask-predicated FMAs over the true
+// nonzeros (Inf * 0 never appears).  Every C entry receives its products in ascending k.
+constexpr int DR_W = 4;  // warps per CTA
+constexpr int DR_AP = 17;  // staged A row pitch (values): conflict-free column reads
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(RN_T) k_num_dense(RowNumParams P, int64_t n) {
-    __shared__ __align__(16) unsigned char smem[RN_W][DENSE_BYTES];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t k = (int64_t)blockIdx.x * RN_W + w;
-    if (k >= n) return;
-    const DenseRec d = P.dense[k];
-    dense_tile<TI, TO>(P, d.pairs, d.slot, d.cnt, d.off, smem[w], lane);
+__global__ void __launch_bounds__(DR_W * 32) k_num_dense_row(RowNumParams P) {
+    extern __shared__ __align__(16) unsigned char dyn[];
+    __shared__ int64_t dOff[32];
+    __shared__ uint8_t dQ[32], sNF[MAX_A];
+    __shared__ int dN;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane >> 1, h = lane & 1;
+    const int64_t I = blockIdx.x;
+    const int64_t t0 = P.tpC[I], nC = P.tpC[I + 1] - t0;
+    if (nC == 0) return;  // CTA-uniform
+    const int64_t a0 = P.tpA[I];
+    const int nA = (int)(P.tpA[I + 1] - a0);
+    const int64_t base = P.costOff[a0];
+    TO *sA = reinterpret_cast<TO *>(dyn);                                 // [maxA][16 * 17]
+    TO *Bd = sA + (int64_t)P.max_a_dense * TILE * DR_AP + w * TILE * TILE;  // this warp's B tile
+    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
+    int64_t zrow = P.rowOff[I];
+    bool staged = false;
+    u64c nden = 0;
+    for (int64_t q0 = 0; q0 < nC; q0 += 32) {
+        if (w == 0) {  // this chunk's dense tiles and their nonzero offsets
+            const int64_t q = q0 + lane;
+            const uint32_t nz = q < nC ? P.tNnz[base + q] : 0u;
+            uint32_t incl = nz;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t o = __shfl_up_sync(FULL, incl, d);
+                if (lane >= d) incl += o;
+            }
+            const bool isD = q < nC && (int)nz >= P.dense_threshold;
+            const unsigned bd = __ballot_sync(FULL, isD);
+            if (isD) {
+                const int k = __popc(bd & ((1u << lane) - 1u));
+                dQ[k] = (uint8_t)lane;
+                dOff[k] = zrow + (incl - nz);
+            }
+            zrow += __shfl_sync(FULL, incl, 31);
+            if (lane == 0) dN = __popc(bd);
+        }
+        __syncthreads();
+        const int nd = dN;
+        if (nd && !staged) {  // the row's A tiles, expanded (first chunk with a dense tile)
+            for (int sI = w; sI < nA; sI += DR_W) {
+                TO *As = sA + sI * TILE * DR_AP;
+                for (int e = lane; e < TILE * DR_AP; e += 32) As[e] = (TO)0;
+                __syncwarp();
+                bool bad = false;
+                for (int64_t e = P.tnzA[a0 + sI] + lane; e < P.tnzA[a0 + sI + 1]; e += 32) {
+                    const uint32_t ix = P.ixA[e];
+                    const TO v = vcvt<TO>(vA[e]);
+                    bad |= !isfinite(v);
+                    As[(ix >> 4) * DR_AP + (ix & 15)] = v;
+                }
+                const bool any = __any_sync(FULL, bad);
+                if (lane == 0) sNF[sI] = any;
+            }
+            staged = true;
+            __syncthreads();
+        }
+        nden += nd;
+        for (int k = w; k < nd; k += DR_W) {
+            const int64_t slot = base + q0 + dQ[k];
+            const int64_t off = dOff[k];
+            const uint64_t *pp = P.pairs + base + P.tStart[slot];
+            const uint32_t cnt = P.tCnt[slot];
+            TO acc[8];
+#pragma unroll
+            for (int jj = 0; jj < 8; jj++) acc[jj] = (TO)0;
+            uint64_t prn = cnt ? pp[0] : 0;
+            for (uint32_t p = 0; p < cnt; p++) {
+                const uint64_t pr = prn;
+                if (p + 1 < cnt) prn = pp[p + 1];
+                const int sI = (int)((int64_t)(pr >> 32) - a0);
+                const int64_t pB = (int64_t)(uint32_t)pr;
+                const uint32_t u = (uint32_t)P.colOccA[a0 + sI] & (uint32_t)P.rowOccB[pB];
+#pragma unroll
+                for (int e = lane; e < TILE * TILE * (int)sizeof(TO) / 16; e += 32)
+                    reinterpret_cast<uint4 *>(Bd)[e] = make_uint4(0u, 0u, 0u, 0u);
+                __syncwarp();
+                bool bad = false;
+                for (int64_t e = P.tnzB[pB] + lane; e < P.tnzB[pB + 1]; e += 32) {
+                    const uint32_t ix = P.ixB[e];
+                    const TO v = vcvt<TO>(vB[e]);
+                    bad |= !isfinite(v);
+                    Bd[(ix >> 4) * TILE + (ix & 15)] = v;
+                }
+                const bool anybad = __any_sync(FULL, bad) || sNF[sI];
+                __syncwarp();
+                const TO *ar = sA + sI * TILE * DR_AP + r * DR_AP;
+                const TO *bs = Bd + 8 * h;
+                if (!anybad) {
+#pragma unroll
+                    for (int g = 0; g < TILE; g += 4) {
+                        if ((u >> g) & 15u) {  // warp-uniform
+#pragma unroll
+                            for (int c = g; c < g + 4; c++) {
+                                const TO a = ar[c];
+                                TO b[8];
+                                lds8(bs + c * TILE, b);
+#pragma unroll
+                                for (int jj = 0; jj < 8; jj++) acc[jj] = vfma(a, b[jj], acc[jj]);
+                            }
+                        }
+                    }
+                } else {
+                    const uint32_t mAr = P.mA[(a0 + sI) * TILE + r];
+                    for (int c = 0; c < TILE; c++) {
+                        if ((u >> c) & (mAr >> c) & 1u) {
+                            const TO a = ar[c];
+                            const uint32_t mb = (uint32_t)P.mB[pB * TILE + c] >> (8 * h);
+#pragma unroll
+                            for (int jj = 0; jj < 8; jj++)
+                                if ((mb >> jj) & 1u) acc[jj] = vfma(a, bs[c * TILE + jj], acc[jj]);
+                        }
+                    }
+                }
+                __syncwarp();  // the B buffer is rewritten by the next pair
+            }
+            const uint32_t mCr = P.sMaskC[slot * TILE + r];
+            const int64_t ob = off + P.sRowPtrC[slot * TILE + r];
+#pragma unroll
+            for (int jj = 0; jj < 8; jj++) {
+                const int j = 8 * h + jj;
+                if ((mCr >> j) & 1u) {
+                    const int q = __popc(mCr & ((1u << j) - 1u));
+                    P.ixC[ob + q] = (uint8_t)((r << 4) | j);
+                    static_cast<TO *>(P.vC)[ob + q] = acc[jj];
+                }
+            }
+        }
+        __syncthreads();  // warp 0 rewrites the list
+    }
+    if (threadIdx.x == 0 && nden) atomicAdd(&P.cnt->n3dense, nden);
 }
 
 template <typename TI, typename TO>
@@ -515,7 +565,11 @@ void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s) {
         }
         TSG_LAUNCH((k_num_small<TI, TO>), (unsigned)occ, NS_T, 0, s, P);
     }
-    if (n_dense > 0) TSG_LAUNCH((k_num_dense<TI, TO>), grid_for(n_dense, RN_W), RN_T, 0, s, P, n_dense);
+    if (n_dense > 0) {
+        const size_t smem = ((size_t)P.max_a_dense * TILE * DR_AP + (size_t)DR_W * TILE * TILE) * sizeof(TO);
+        TSG_CUDA(cudaFuncSetAttribute(k_num_dense_row<TI, TO>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        TSG_LAUNCH((k_num_dense_row<TI, TO>), (unsigned)P.tm, DR_W * 32, smem, s, P);
+    }
 }
 
 }  // namespace
@@ -554,7 +608,8 @@ void launch_num_rows(const RowNumArgs &a, cudaStream_t s) {
     P.vC = a.C->val;
     P.dense_threshold = a.dense_threshold;
     P.small_max = a.small_max;
-    P.dense = static_cast<DenseRec *>(a.dense);
+    P.max_a_dense = a.max_a_dense;
+    P.colOccA = a.colOccA;
     P.small = static_cast<RowTileRec *>(a.small);
     P.cnt = a.cnt;
     switch (a.A->dtype) {

@@ -349,8 +349,9 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         R.dense_threshold = TH;
         R.small_max = SMALL_NNZ;
         R.n_dense = (int64_t)hc2.n2dense;
-        R.dense = hc2.n2dense ? tmp.get<uint8_t>(DENSE_REC_BYTES * (int64_t)hc2.n2dense) : nullptr;
-        R.small = tmp.get<uint8_t>(DENSE_REC_BYTES * ntC);
+        R.max_a_dense = (int)hc2.max_a_dense;
+        R.colOccA = colOccA;
+        R.small = tmp.get<uint8_t>(ROW_REC_BYTES * ntC);
         R.cnt = cnt;
         if (bias) {
             launch_add_i64(rowOff, tmA + 1, bias, s);

@@ -757,7 +757,10 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t t
     ndense += __shfl_xor_sync(FULL, ndense, 16);
     if (lane == 0) {
         P.rowNnz[I] = rownnz;
-        if (ndense) atomicAdd(&P.cnt->n2dense, (u64c)ndense);
+        if (ndense) {
+            atomicAdd(&P.cnt->n2dense, (u64c)ndense);
+            atomicMax(&P.cnt->max_a_dense, (u64c)nA);
+        }
     }
 }
 
