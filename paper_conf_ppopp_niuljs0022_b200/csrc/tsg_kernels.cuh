@@ -199,7 +199,8 @@ struct RowNumArgs {
     DevCounters *cnt;
 };
 constexpr int ROW_REC_BYTES = 32;
-void launch_num_rows(const RowNumArgs &a, cudaStream_t s);
+// k_num_rows / k_num_small on `s`; the dense class (independent of them) on `sd`
+void launch_num_rows(const RowNumArgs &a, cudaStream_t s, cudaStream_t sd);
 
 // launchers (tsg_step23.cu)
 void launch_step2(const StepParams &P, cudaStream_t s);

@@ -551,7 +551,7 @@ __global__ void __launch_bounds__(DR_W * 32) k_num_dense_row(RowNumParams P) {
 }
 
 template <typename TI, typename TO>
-void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s) {
+void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s, cudaStream_t sd) {
     TSG_LAUNCH((k_num_rows<TI, TO>), grid_for(ceil_div(P.tm, 2), RN_W), RN_T, 0, s, P);
     if (P.small) {  // persistent grid: the record count is read on the device
         static int occ = 0;
@@ -568,13 +568,13 @@ void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s) {
     if (n_dense > 0) {
         const size_t smem = ((size_t)P.max_a_dense * TILE * DR_AP + (size_t)DR_W * TILE * TILE) * sizeof(TO);
         TSG_CUDA(cudaFuncSetAttribute(k_num_dense_row<TI, TO>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        TSG_LAUNCH((k_num_dense_row<TI, TO>), (unsigned)P.tm, DR_W * 32, smem, s, P);
+        TSG_LAUNCH((k_num_dense_row<TI, TO>), (unsigned)P.tm, DR_W * 32, smem, sd, P);
     }
 }
 
 }  // namespace
 
-void launch_num_rows(const RowNumArgs &a, cudaStream_t s) {
+void launch_num_rows(const RowNumArgs &a, cudaStream_t s, cudaStream_t sd) {
     RowNumParams P{};
     P.tm = a.tm;
     P.tpA = a.A->tile_ptr;
@@ -613,9 +613,9 @@ void launch_num_rows(const RowNumArgs &a, cudaStream_t s) {
     P.small = static_cast<RowTileRec *>(a.small);
     P.cnt = a.cnt;
     switch (a.A->dtype) {
-        case TSG_F64: launch_t<double, double>(P, a.n_dense, s); break;
-        case TSG_F32: launch_t<float, float>(P, a.n_dense, s); break;
-        default: launch_t<__half, float>(P, a.n_dense, s);
+        case TSG_F64: launch_t<double, double>(P, a.n_dense, s, sd); break;
+        case TSG_F32: launch_t<float, float>(P, a.n_dense, s, sd); break;
+        default: launch_t<__half, float>(P, a.n_dense, s, sd);
     }
 }
 

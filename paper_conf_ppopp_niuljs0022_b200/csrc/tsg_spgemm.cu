@@ -358,7 +358,11 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
             C->idx -= bias;
             C->val = static_cast<uint8_t *>(C->val) - bias * (int64_t)dtype_size(dtC);
         }
-        launch_num_rows(R, s);
+        {  // the dense class runs on a side stream next to k_num_rows / k_num_small (disjoint outputs)
+            SideStream sd(s);
+            launch_num_rows(R, s, sd.stream());
+            sd.join();
+        }
         if (bias) {
             launch_add_i64(C->tile_nnz, ntC + 1, -bias, s);
             C->idx += bias;
