@@ -119,21 +119,7 @@ void Allocator::free(void *p, size_t bytes, cudaStream_t s) const {
 // behind whatever the copy engine is already doing (a caller streaming the previous result to
 // the host), a kernel's posted writes do not.
 namespace {
-struct ExportArgs {
-    const uint8_t *src[4];
-    uint32_t bytes[4], off[4];
-    int n;
-    uint8_t *dst;
-    volatile unsigned int *flag;  // written last, after a system-scope fence
-    unsigned int seq;
-};
-__global__ void k_export(ExportArgs a) {
-    for (int k = 0; k < a.n; k++)
-        for (uint32_t i = threadIdx.x; i < a.bytes[k]; i += blockDim.x) a.dst[a.off[k] + i] = a.src[k][i];
-    __threadfence_system();
-    __syncthreads();
-    if (threadIdx.x == 0) *a.flag = a.seq;
-}
+__global__ void k_export(ExportArgs a) { export_segments(a); }
 struct Mapped {
     uint8_t *h = nullptr;
     uint8_t *d = nullptr;
@@ -149,7 +135,7 @@ constexpr size_t FLAG_OFF = MAPPED_BYTES - 64;  // the completion flag's slot
 // reports errors.  Either way the stream has passed the export when this returns.
 constexpr double SPIN_US = 200.0;
 
-void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
+static Mapped &mapped() {
     int dev = 0;
     TSG_CUDA(cudaGetDevice(&dev));
     static thread_local Mapped m[16];
@@ -162,6 +148,11 @@ void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
         mp.d = static_cast<uint8_t *>(d);
         *reinterpret_cast<volatile unsigned int *>(mp.h + FLAG_OFF) = 0u;
     }
+    return mp;
+}
+
+ExportArgs begin_read(std::initializer_list<DevRead> segs) {
+    Mapped &mp = mapped();
     ExportArgs a{};
     uint32_t off = 0;
     TSG_REQUIRE(segs.size() <= 4, TSG_ERR_INTERNAL, "too many device reads");
@@ -176,7 +167,11 @@ void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
     a.dst = mp.d;
     a.flag = reinterpret_cast<volatile unsigned int *>(mp.d + FLAG_OFF);
     a.seq = ++mp.seq;
-    TSG_LAUNCH(k_export, 1, 256, 0, s, a);
+    return a;
+}
+
+void finish_read(const ExportArgs &a, std::initializer_list<DevRead> segs, cudaStream_t s) {
+    Mapped &mp = mapped();
     const double t0 = now_ms();
     volatile unsigned int *hf = reinterpret_cast<volatile unsigned int *>(mp.h + FLAG_OFF);
     bool seen = false;
@@ -195,6 +190,12 @@ void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
         memcpy(r.host, mp.h + a.off[k], r.bytes);
         k++;
     }
+}
+
+void read_device(std::initializer_list<DevRead> segs, cudaStream_t s) {
+    const ExportArgs a = begin_read(segs);
+    TSG_LAUNCH(k_export, 1, 256, 0, s, a);
+    finish_read(a, segs, s);
 }
 
 int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {

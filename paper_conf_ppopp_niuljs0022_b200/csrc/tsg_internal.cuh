@@ -217,8 +217,10 @@ namespace tsg {
 // device scan: out[0] = 0, out[i+1] = out[i] + in[i]; out has n+1 entries; out may alias in
 // when Tin == int64_t.  Three-phase (reduce / scan sums / downsweep), recursive on the sums.
 // ------------------------------------------------------------------------------------------
+struct ExportArgs;
 template <typename Tin>
-void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buffers &tmp);
+void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buffers &tmp,
+                    const ExportArgs *ex = nullptr);  // ex: the CTA that writes out[n] then exports
 
 // read one int64 from device memory (blocking on stream s)
 int64_t read_scalar(const int64_t *dptr, cudaStream_t s);
@@ -230,6 +232,30 @@ struct DevRead {
     size_t bytes;
 };
 void read_device(std::initializer_list<DevRead> segs, cudaStream_t s);
+// A blocking read whose export runs at the end of a kernel the call launches anyway (the scan
+// producing the value read): begin_read() lays the segments out in the thread's mapped buffer,
+// the kernel copies them and raises the flag, finish_read() waits for it and copies them out.
+struct ExportArgs {
+    const uint8_t *src[4];
+    uint32_t bytes[4], off[4];
+    int n;  // 0: no export
+    uint8_t *dst;
+    volatile unsigned int *flag;  // written last, after a system-scope fence
+    unsigned int seq;
+};
+ExportArgs begin_read(std::initializer_list<DevRead> segs);
+void finish_read(const ExportArgs &a, std::initializer_list<DevRead> segs, cudaStream_t s);
+// inside a kernel, by one whole CTA, after everything the segments cover is written
+__device__ __forceinline__ void export_segments(const ExportArgs &a) {
+    __syncthreads();
+    __threadfence();
+    for (int k = 0; k < a.n; k++)
+        for (uint32_t i = threadIdx.x; i < a.bytes[k]; i += blockDim.x)
+            a.dst[a.off[k] + i] = *((volatile const uint8_t *)a.src[k] + i);
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) *a.flag = a.seq;
+}
 
 // per-call launch counter (thread-local)
 void reset_call_launches();

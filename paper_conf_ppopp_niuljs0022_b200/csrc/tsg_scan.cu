@@ -62,7 +62,7 @@ __device__ __forceinline__ void st_status(uint64_t *p, uint64_t v) {
 
 template <typename Tin>
 __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n, int64_t *out, uint64_t *status,
-                                                      unsigned long long *ticket) {
+                                                      unsigned long long *ticket, ExportArgs ex) {
     __shared__ int64_t s_bid, s_base;
     if (threadIdx.x == 0) s_bid = gridDim.x == 1 ? 0 : (int64_t)atomicAdd(ticket, 1ull);
     __syncthreads();
@@ -109,27 +109,30 @@ __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n,
         pre += v[i];
     }
     if (base < n && base + SCAN_IPT >= n) out[n] = pre;  // the thread holding the last element
+    if (ex.n && b == (int64_t)gridDim.x - 1) export_segments(ex);  // the CTA that wrote out[n]
 }
 
 __global__ void k_set_zero_i64(int64_t *p) { *p = 0; }
+__global__ void k_export_only(ExportArgs a) { export_segments(a); }
 
 }  // namespace
 
 template <typename Tin>
-void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buffers &tmp) {
+void exclusive_scan(const Tin *in, int64_t *out, int64_t n, cudaStream_t s, Buffers &tmp, const ExportArgs *ex) {
     if (n <= 0) {
         TSG_LAUNCH(k_set_zero_i64, 1, 1, 0, s, out);
+        if (ex) TSG_LAUNCH(k_export_only, 1, 256, 0, s, *ex);
         return;
     }
     const int64_t nb = ceil_div(n, SCAN_TILE);
     uint64_t *status = tmp.get<uint64_t>(nb + 1);  // [0, nb): tile status, [nb]: ticket
     if (nb > 1) TSG_CUDA(cudaMemsetAsync(status, 0, sizeof(uint64_t) * (nb + 1), s));  // one CTA: no look-back
     TSG_LAUNCH((k_scan_1pass<Tin>), (unsigned)nb, SCAN_T, 0, s, in, n, out, status,
-               reinterpret_cast<unsigned long long *>(status + nb));
+               reinterpret_cast<unsigned long long *>(status + nb), ex ? *ex : ExportArgs{});
 }
 
-template void exclusive_scan<int64_t>(const int64_t *, int64_t *, int64_t, cudaStream_t, Buffers &);
-template void exclusive_scan<int32_t>(const int32_t *, int64_t *, int64_t, cudaStream_t, Buffers &);
-template void exclusive_scan<uint32_t>(const uint32_t *, int64_t *, int64_t, cudaStream_t, Buffers &);
+template void exclusive_scan<int64_t>(const int64_t *, int64_t *, int64_t, cudaStream_t, Buffers &, const ExportArgs *);
+template void exclusive_scan<int32_t>(const int32_t *, int64_t *, int64_t, cudaStream_t, Buffers &, const ExportArgs *);
+template void exclusive_scan<uint32_t>(const uint32_t *, int64_t *, int64_t, cudaStream_t, Buffers &, const ExportArgs *);
 
 }  // namespace tsg

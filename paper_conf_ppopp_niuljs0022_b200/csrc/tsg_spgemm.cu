@@ -280,12 +280,17 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.mB = B->mask;
     launch_row_sort(P1, tmA, s);
     int64_t *tile_ptr = out.get<int64_t>(tmA + 1);
-    exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp);
-    // blocking read #1: C's tile count, the candidate total, the row classes
+    // blocking read #1: C's tile count, the candidate total, the row classes (exported by the scan)
     DevCounters hc{};
     int64_t Utot = 0, ntC = 0, nnzC = 0;
-    read_device({{&ntC, tile_ptr + tmA, sizeof(int64_t)}, {&Utot, costOff + ntA, sizeof(int64_t)},
-                 {&hc, cnt, sizeof(DevCounters)}}, s);
+    {
+        const std::initializer_list<DevRead> segs = {{&ntC, tile_ptr + tmA, sizeof(int64_t)},
+                                                     {&Utot, costOff + ntA, sizeof(int64_t)},
+                                                     {&hc, cnt, sizeof(DevCounters)}};
+        const ExportArgs ex = begin_read(segs);
+        exclusive_scan<int64_t>(nC, tile_ptr, tmA, s, tmp, &ex);
+        finish_read(ex, segs, s);
+    }
     syncs++;
     TSG_REQUIRE(Utot < ((int64_t)1 << 40), TSG_ERR_OVERFLOW, "too many step-1 candidates");
     if (hc.overflow) {
@@ -315,9 +320,14 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         // ---------------- a3: nonzero offsets of the rows; the one allocation of C
         nv.push("tsg a3 scan + allocation");
         int64_t *rowOff = tmp.get<int64_t>(tmA + 1);
-        exclusive_scan<int64_t>(P1.rowNnz, rowOff, tmA, s, tmp);
         DevCounters hc2{};
-        read_device({{&nnzC, rowOff + tmA, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
+        {
+            const std::initializer_list<DevRead> segs = {{&nnzC, rowOff + tmA, sizeof(int64_t)},
+                                                         {&hc2, cnt, sizeof(DevCounters)}};
+            const ExportArgs ex = begin_read(segs);
+            exclusive_scan<int64_t>(P1.rowNnz, rowOff, tmA, s, tmp, &ex);
+            finish_read(ex, segs, s);
+        }
         syncs++;
         C->tile_col = out.get<int32_t>(ntC);
         C->tile_nnz = out.get<int64_t>(ntC + 1);
@@ -430,9 +440,14 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         launch_step2(P, s);
         // ---------------- a3: offsets of C's nonzeros, allocation
         nv.push("tsg a3 scan + allocation");
-        exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp);
         DevCounters hc2{};
-        read_device({{&nnzC, tile_nnz + ntC, sizeof(int64_t)}, {&hc2, cnt, sizeof(DevCounters)}}, s);
+        {
+            const std::initializer_list<DevRead> segs = {{&nnzC, tile_nnz + ntC, sizeof(int64_t)},
+                                                         {&hc2, cnt, sizeof(DevCounters)}};
+            const ExportArgs ex = begin_read(segs);
+            exclusive_scan<int64_t>(tile_nnz, tile_nnz, ntC, s, tmp, &ex);
+            finish_read(ex, segs, s);
+        }
         syncs++;
         uint8_t *idx = out.get<uint8_t>(nnzC);
         void *val = out.get<uint8_t>((int64_t)dtype_size(dtC) * nnzC);
