@@ -180,7 +180,7 @@ void launch_compact(const CompactParams &P, int64_t ntC, cudaStream_t s);
 
 // ---------------- a4 on the row path (tsg_rows.cu)
 struct RowNumArgs {
-    int64_t tm;
+    int64_t tm, ntC;
     const tsg_tiles *A, *B;
     tsg_tiles *C;                 // tile_ptr filled; the other arrays allocated
     const uint16_t *mTB, *rowOccB;

@@ -59,7 +59,7 @@ struct RowTileRec {  // a C tile left by k_num_rows to k_num_small / k_num_dense
 };
 
 struct RowNumParams {
-    int64_t tm;
+    int64_t tm, ntC;
     // A
     const int64_t *tpA, *tnzA;
     const uint8_t *rpA, *ixA;
@@ -563,7 +563,9 @@ void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s, cudaStream
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_small<TI, TO>, NS_T, 0);
             occ = std::max(occ, 1) * nsm;
         }
-        TSG_LAUNCH((k_num_small<TI, TO>), (unsigned)occ, NS_T, 0, s, P);
+        // small C tiles <= C's tiles: no more CTAs than 32-tile groups of them
+        const int64_t need = ceil_div(ceil_div(P.ntC, 32), NS_T / 32);
+        TSG_LAUNCH((k_num_small<TI, TO>), (unsigned)std::max<int64_t>(1, std::min<int64_t>(occ, need)), NS_T, 0, s, P);
     }
     if (n_dense > 0) {
         const size_t smem = ((size_t)P.max_a_dense * TILE * DR_AP + (size_t)DR_W * TILE * TILE) * sizeof(TO);
@@ -577,6 +579,7 @@ void launch_t(const RowNumParams &P, int64_t n_dense, cudaStream_t s, cudaStream
 void launch_num_rows(const RowNumArgs &a, cudaStream_t s, cudaStream_t sd) {
     RowNumParams P{};
     P.tm = a.tm;
+    P.ntC = a.ntC;
     P.tpA = a.A->tile_ptr;
     P.tnzA = a.A->tile_nnz;
     P.rpA = a.A->row_ptr;

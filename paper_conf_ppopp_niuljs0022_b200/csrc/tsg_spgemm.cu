@@ -342,6 +342,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         nv.push("tsg a4 numeric");
         RowNumArgs R{};
         R.tm = tmA;
+        R.ntC = ntC;
         R.A = A;
         R.B = B;
         R.C = C;
