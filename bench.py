@@ -430,8 +430,8 @@ def main():
     achieved = alg[dom] / (steps_ms[dom] / 1e3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_r02_{args.config}.json")
-    if os.path.exists(tp) and world == 1 and K == 1 and args.dtype == "f64" and not args.aat:
-        traffic = json.load(open(tp)).get(dom)  # captured for the whole single-GPU fp64 call only
+    if os.path.exists(tp) and world == 1 and K == 1 and args.dtype == "f64" and not args.aat and args.path == "auto":
+        traffic = json.load(open(tp)).get(dom)  # captured for the default single-GPU fp64 call only
     bytes_alg = tile_bytes(Ashard.tile_m, Ashard.num_tiles, Ashard.nnz, vb) + \
         K * tile_bytes(Bt.tile_m, Bt.num_tiles, Bt.nnz, vb) + tile_bytes(Ashard.tile_m, ntC, nnzC, cb)
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": bw, "unit": "GB/s",

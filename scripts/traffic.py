@@ -4,8 +4,8 @@ Run under ncu with the capture limited to one warm call:
     ncu --profile-from-start off --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
         --csv --log-file gpurun_out/traffic_C2.csv python scripts/traffic.py C2
 then `python scripts/traffic.py --summarize gpurun_out/traffic_C2.csv C2` writes
-profiles/traffic_r02_C2.json: bytes per step (launches up to the first blocking-read export =
-steps 1 (a0 + a1), up to the second = step 2 (a2 + a3), after it = step 3 (a4))."""
+profiles/traffic_r02_C2.json: bytes per step (launches up to the scan that exports the first
+blocking read = step 1 (a0 + a1), up to the second = step 2 (a2 + a3), after it = step 3 (a4))."""
 import csv, json, os, sys
 
 if len(sys.argv) > 1 and sys.argv[1] == "--summarize":
@@ -21,16 +21,21 @@ if len(sys.argv) > 1 and sys.argv[1] == "--summarize":
             continue
         d = per.setdefault(int(r[ii]), {"name": r[ki]})
         d[r[mi]] = float(r[vi].replace(",", ""))
-    step, out, kern = 1, {"step1": 0.0, "step2": 0.0, "step3": 0.0}, {}
+    # a step ends with the scan that exports its blocking read: the first k_scan_1pass after the
+    # step's own kernels (step 1: the row kernels; step 2: the symbolic kernels)
+    ends = {1: ("k_row_merge", "k_row_small", "k_row_rank", "k_row_big"), 2: ("k_s2", "k_s2_light", "k_sym_rows")}
+    step, seen, out, kern = 1, False, {"step1": 0.0, "step2": 0.0, "step3": 0.0}, {}
     for i in sorted(per):
         d = per[i]
         b = d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
         out[f"step{step}"] += b
-        name = d["name"].split("(")[0].split("::")[-1]
-        kern.setdefault(f"step{step}", {}).setdefault(name, 0.0)
-        kern[f"step{step}"][name] += b
-        if "k_export" in d["name"]:
-            step = min(3, step + 1)
+        name = d["name"].split("(")[0].split("::")[-1].split("<")[0].strip()
+        kern.setdefault(f"step{step}", {}).setdefault(d["name"].split("(")[0].split("::")[-1], 0.0)
+        kern[f"step{step}"][d["name"].split("(")[0].split("::")[-1]] += b
+        if step < 3 and name in ends[step]:
+            seen = True
+        elif step < 3 and seen and name == "k_scan_1pass":
+            step, seen = step + 1, False
     out = {k: int(v) for k, v in out.items()}
     out["unit"] = "bytes (dram__bytes_read.sum + dram__bytes_write.sum) per call, one warm call, ncu"
     out["per_kernel"] = {s: {k: int(v) for k, v in m.items()} for s, m in kern.items()}
