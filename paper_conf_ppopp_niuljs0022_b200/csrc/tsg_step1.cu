@@ -929,6 +929,16 @@ __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t 
         pre[w] = (uint32_t)run;
         run += __popc(bm[w]);
     }
+    // the C tiles' tile columns, straight from the bitmap (each thread its words)
+    for (int w = w0; w < w1; w++) {
+        uint32_t m = bm[w];
+        uint32_t rk = pre[w];
+        while (m) {
+            const int b = __ffs(m) - 1;
+            m &= m - 1;
+            P.tJ[base + rk++] = jlo + (int32_t)(w * 32 + b);
+        }
+    }
     uint32_t *cursor = reinterpret_cast<uint32_t *>(P.bigKeysB + o);  // per C tile, pass 3
     for (int64_t r = threadIdx.x; r < nC; r += RANK_T) {
         P.tCnt[base + r] = 0;
@@ -936,7 +946,8 @@ __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t 
         cursor[r] = 0;
     }
     __syncthreads();
-    // pass 2: pairs and work per C tile (and its tile column)
+    // pass 2: pairs and work per C tile (global counters: shared ones for rows of up to 12 K C
+    // tiles halve the occupancy and measured slower on C4, 51 vs 39 ms)
     for (int64_t u = threadIdx.x; u < U; u += RANK_T) {
         const uint32_t jw = sJ[u];
         if (jw == ~0u) continue;
@@ -944,7 +955,6 @@ __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t 
         const uint32_t rank = pre[jr >> 5] + __popc(bm[jr >> 5] & ((1u << (jr & 31)) - 1u));
         atomicAdd(&P.tCnt[base + rank], 1u);
         atomicAdd(&P.tWork[base + rank], jw >> 27);
-        P.tJ[base + rank] = jlo + (int32_t)jr;
     }
     __syncthreads();
     // pair offsets of the C tiles (row-relative), blocked scan over the nC counts
