@@ -7,9 +7,12 @@
 //   1. tiles per tile column J of A (atomic counts) -> scan -> tile_ptr of A^T
 //   2. each tile row I drops its tiles into their column's slot range (atomic cursor per column)
 //   3. a warp per column ranks its slots by I (tile rows are unique within a column), which
-//      gives the ascending-I order of A^T's tile row J without a global sort
+//      gives the ascending-I order of A^T's tile row J without a global sort; columns wider than
+//      64 tiles (hubs) take a CTA with a tile-row bitmap and popcount ranks (linear, not k^2)
 //   4. nnz offsets of A^T (scan), then a thread per tile writes the transposed tile.
 // Exact (a permutation of A's data): compared bit for bit with the oracle's CSR transpose.
+#include <algorithm>
+
 #include "tsg_kernels.cuh"
 
 namespace tsg {
@@ -34,13 +37,40 @@ __global__ void k_tp_place(int64_t tm, const int64_t *__restrict__ tp, const int
     }
 }
 
-// warp per tile column J: rank each slot by its tile row I -> A^T's tile (J, I) in ascending I
+// warp per tile column J: rank each slot by its tile row I -> A^T's tile (J, I) in ascending I.
+// Columns of at most TP_SMALL tiles compare their slots directly (k^2 / 32 steps per lane); wider
+// ones (R-MAT hub columns) go to a list for k_tp_rank_wide.
+constexpr int TP_SMALL = 64;
 __global__ void k_tp_rank(int64_t tn, const int64_t *__restrict__ tpT, const int32_t *__restrict__ slotI,
                           const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
-                          int32_t *__restrict__ tcolT) {
+                          int32_t *__restrict__ tcolT, int32_t *__restrict__ wide, unsigned long long *nwide) {
     const int lane = threadIdx.x & 31;
     const int64_t J = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (J >= tn) return;
+    const int64_t b = tpT[J], e = tpT[J + 1];
+    if (e - b > TP_SMALL) {
+        if (lane == 0) wide[atomicAdd(nwide, 1ULL)] = (int32_t)J;
+        return;
+    }
+    for (int64_t s = b + lane; s < e; s += 32) {
+        const int32_t I = slotI[s];
+        int64_t rank = 0;
+        for (int64_t s2 = b; s2 < e; s2++) rank += slotI[s2] < I;
+        perm[b + rank] = slotSrc[s];
+        tcolT[b + rank] = I;
+    }
+}
+
+// fallback for the wide columns when the tile-row bitmap would not fit shared memory: a warp per
+// wide column, ranks by comparison
+__global__ void k_tp_rank_all(int64_t tn, const int64_t *__restrict__ tpT, const int32_t *__restrict__ slotI,
+                              const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
+                              int32_t *__restrict__ tcolT, const int32_t *__restrict__ wide,
+                              const unsigned long long *nwide) {
+    const int lane = threadIdx.x & 31;
+    const int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (k >= (int64_t)*nwide) return;
+    const int64_t J = wide[k];
     const int64_t b = tpT[J], e = tpT[J + 1];
     for (int64_t s = b + lane; s < e; s += 32) {
         const int32_t I = slotI[s];
@@ -48,6 +78,69 @@ __global__ void k_tp_rank(int64_t tn, const int64_t *__restrict__ tpT, const int
         for (int64_t s2 = b; s2 < e; s2++) rank += slotI[s2] < I;
         perm[b + rank] = slotSrc[s];
         tcolT[b + rank] = I;
+    }
+}
+
+// wide columns: a CTA each (persistent over the list), the column's tile rows marked in a
+// shared-memory bitmap over all tile rows; a slot's rank is the number of marked rows before its
+// own (per-word popcount prefix), as in step 1's rank kernel -- linear in the column's tiles
+constexpr int TPW_T = 512;
+__global__ void __launch_bounds__(TPW_T) k_tp_rank_wide(int64_t tm, const int64_t *__restrict__ tpT,
+                                                       const int32_t *__restrict__ slotI,
+                                                       const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
+                                                       int32_t *__restrict__ tcolT, const int32_t *__restrict__ wide,
+                                                       const unsigned long long *nwide) {
+    extern __shared__ uint32_t bm[];  // [words] bitmap, [words] exclusive popcount prefix
+    __shared__ uint32_t wsum[TPW_T / 32 + 1];
+    const int words = (int)((tm + 31) / 32);
+    uint32_t *pre = bm + words;
+    const int64_t n = (int64_t)*nwide;
+    for (int64_t k = blockIdx.x; k < n; k += gridDim.x) {
+        const int64_t J = wide[k];
+        const int64_t b = tpT[J], e = tpT[J + 1];
+        for (int w = threadIdx.x; w < words; w += TPW_T) bm[w] = 0;
+        __syncthreads();
+        for (int64_t s = b + threadIdx.x; s < e; s += TPW_T) {
+            const int32_t I = slotI[s];
+            atomicOr(&bm[I >> 5], 1u << (I & 31));
+        }
+        __syncthreads();
+        // exclusive prefix of the word popcounts: blocked ownership, then a CTA scan of the sums
+        const int per = (words + TPW_T - 1) / TPW_T;
+        const int w0 = min(words, (int)threadIdx.x * per), w1 = min(words, w0 + per);
+        uint32_t c = 0;
+        for (int w = w0; w < w1; w++) c += __popc(bm[w]);
+        const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
+        uint32_t incl = c;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t o = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += o;
+        }
+        if (lane == 31) wsum[wp] = incl;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t acc = 0;
+            for (int q = 0; q < TPW_T / 32; q++) {
+                const uint32_t x = wsum[q];
+                wsum[q] = acc;
+                acc += x;
+            }
+        }
+        __syncthreads();
+        uint32_t run = wsum[wp] + incl - c;
+        for (int w = w0; w < w1; w++) {
+            pre[w] = run;
+            run += __popc(bm[w]);
+        }
+        __syncthreads();
+        for (int64_t s = b + threadIdx.x; s < e; s += TPW_T) {
+            const int32_t I = slotI[s];
+            const int64_t rank = pre[I >> 5] + __popc(bm[I >> 5] & ((1u << (I & 31)) - 1u));
+            perm[b + rank] = slotSrc[s];
+            tcolT[b + rank] = I;
+        }
+        __syncthreads();
     }
 }
 
@@ -116,7 +209,22 @@ void launch_transpose_tiles(const tsg_tiles *T, const Allocator &al, cudaStream_
     TSG_LAUNCH(k_tp_place, grid_for(T->tm, 8), 256, 0, s, T->tm, T->tile_ptr, T->tile_col, cursor, slotI, slotSrc);
     int64_t *perm = tmp.get<int64_t>(nt);
     int32_t *tcolT = out.get<int32_t>(nt);
-    TSG_LAUNCH(k_tp_rank, grid_for(tmT, 8), 256, 0, s, tmT, tpT, slotI, slotSrc, perm, tcolT);
+    int32_t *wide = tmp.get<int32_t>(tmT + 1);
+    unsigned long long *nwide = reinterpret_cast<unsigned long long *>(cursor + tmT);  // zeroed below
+    TSG_CUDA(cudaMemsetAsync(nwide, 0, sizeof(unsigned long long), s));
+    TSG_LAUNCH(k_tp_rank, grid_for(tmT, 8), 256, 0, s, tmT, tpT, slotI, slotSrc, perm, tcolT, wide, nwide);
+    const int64_t words = (T->tm + 31) / 32;
+    const size_t smem = (size_t)words * 8;
+    if (smem <= 200 * 1024) {  // tile rows of A <= 819200 (else the wide columns rank by comparisons)
+        int dev = 0, nsm = 148;
+        TSG_CUDA(cudaGetDevice(&dev));
+        TSG_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+        TSG_CUDA(cudaFuncSetAttribute(k_tp_rank_wide, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        TSG_LAUNCH(k_tp_rank_wide, (unsigned)std::min<int64_t>(std::max<int64_t>(tmT, 1), 2LL * nsm), TPW_T, smem, s,
+                   T->tm, tpT, slotI, slotSrc, perm, tcolT, wide, nwide);
+    } else {
+        TSG_LAUNCH(k_tp_rank_all, grid_for(tmT, 8), 256, 0, s, tmT, tpT, slotI, slotSrc, perm, tcolT, wide, nwide);
+    }
     int64_t *tnzT = out.get<int64_t>(nt + 1);
     TSG_LAUNCH(k_tp_nnz, grid_for(nt, 256), 256, 0, s, nt, perm, T->tile_nnz, tnzT);
     exclusive_scan<int64_t>(tnzT, tnzT, nt, s, tmp);
