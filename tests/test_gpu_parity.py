@@ -120,6 +120,8 @@ def pair_cases():
     c.append(("no-products", gen.from_coo(32, 32, [0], [1], [1.0]), gen.from_coo(32, 32, [2], [3], [1.0])))
     D = gen.dense_block(64, 64)
     c.append(("dense-64", D, D))
+    # 50 dense C tiles per tile row: the row path's dense class walks a row's C tiles in chunks of 32
+    c.append(("dense-wide", D, gen.dense_block(64, 800)))
     c.append(("hub", gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004),
               gen.hub(2048, hub_rows=(0, 1000), hub_cols=(0, 7), density=0.004)))
     W = gen.hub(8192, hub_rows=(0, 5000), hub_cols=(), density=0.002)
