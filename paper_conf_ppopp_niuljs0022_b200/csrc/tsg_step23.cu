@@ -260,8 +260,8 @@ __global__ void __launch_bounds__(T2) k_s2(StepParams P) {
 // ==========================================================================================
 // step 3
 // ==========================================================================================
-// per-warp shared scratch, one union: medium = 4 KB of row accumulators + two MedStage (one per
-// half warp); dense = 4.2 KB of staged tiles; dense on the tensor cores = 5 KB
+// per-warp shared scratch of the medium class: 4 KB of row accumulators + two MedStage (one per
+// half warp)
 constexpr int WACC = 4096;
 
 struct MedStage {  // per half warp: staged metadata and tile masks / row offsets of up to 16 pairs
@@ -274,7 +274,6 @@ struct MedStage {  // per half warp: staged metadata and tile masks / row offset
 constexpr int WREG = WACC + 2 * (int)sizeof(MedStage);
 static_assert(BATCH3 == 16 && BATCH == 16, "staging lane r of a half warp stages pair r of the batch");
 static_assert(sizeof(MedStage) % 16 == 0, "MedStage keeps 16-byte alignment");
-static_assert(WREG >= 5120, "the tensor-core dense path stages 5 KB");
 
 // small tiles (nnz <= small_max): one lane per C nonzero (output-stationary; the paper's sparse
 // accumulator, with each slot owned by one lane).  Entry q of tile t is (r, j): r =
@@ -789,7 +788,7 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
 #ifndef TSG_DENSE_MINB
 #define TSG_DENSE_MINB 4
 #endif
-constexpr int DREG = 5120;  // per-warp staging of the dense paths (fp64: 16x17 + 16x16 doubles; DMMA: 2 x 16x20)
+constexpr int DREG = 2176 + 2048;  // per-warp staging of the dense path: A 16 x 17 and B 16 x 16 (fp64)
 template <typename TI, typename TO>
 __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, int split) {
     __shared__ __align__(16) unsigned char wreg[T3 / 32][DREG];
