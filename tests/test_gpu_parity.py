@@ -730,3 +730,69 @@ def test_scratch_retry_after_arena_release(tsg):
             got = host(C)
             for k in ARRAYS:
                 assert np.array_equal(got[k], ref[k]), k
+
+
+# ------------------------------------------------------------------------------------------
+# seeded random sweep: shapes, densities and tile structures mixed, every pipeline and class
+# ------------------------------------------------------------------------------------------
+def _sweep_case(rng, kind):
+    """One (A, B) pair of a given structure kind, sizes drawn so that tails are ragged."""
+    m, k, n = (int(x) for x in rng.integers(1, 200, 3))
+    dens = float(rng.choice([0.002, 0.02, 0.1, 0.45]))
+    if kind == 0:  # uniform random
+        return gen.random_sparse(m, k, dens, int(rng.integers(1 << 30))), gen.random_sparse(k, n, dens, int(rng.integers(1 << 30)))
+    if kind == 1:  # banded (stencil-like tiles), random bandwidth
+        bw = int(rng.integers(0, 20))
+        def band(r, c):
+            rows, cols = [], []
+            for i in range(r):
+                lo, hi = max(0, i - bw), min(c, i + bw + 1)
+                rows += [i] * max(0, hi - lo)
+                cols += list(range(lo, hi))
+            return gen.from_coo(r, c, rows, cols, rng.uniform(-1, 1, len(rows)))
+        return band(m, k), band(k, n)
+    if kind == 2:  # random dense 16x16 blocks on a sparse background (dense, medium and small C tiles)
+        def blocks(r, c):
+            coo_r, coo_c = [], []
+            for bi in range(-(-r // 16)):
+                for bj in range(-(-c // 16)):
+                    p = rng.random()
+                    if p < 0.25:  # full block
+                        for i in range(bi * 16, min(r, bi * 16 + 16)):
+                            for j in range(bj * 16, min(c, bj * 16 + 16)):
+                                coo_r.append(i)
+                                coo_c.append(j)
+                    elif p < 0.5:  # a few entries
+                        for _ in range(int(rng.integers(1, 6))):
+                            coo_r.append(int(rng.integers(bi * 16, min(r, bi * 16 + 16))))
+                            coo_c.append(int(rng.integers(bj * 16, min(c, bj * 16 + 16))))
+            return gen.from_coo(r, c, coo_r, coo_c, rng.uniform(-1, 1, len(coo_r)))
+        return blocks(m, k), blocks(k, n)
+    # kind 3: wide tile rows (> 32 A tiles in a tile row: the per-C-tile pipeline's hub classes)
+    kw = int(rng.integers(33 * 16, 70 * 16))
+    A = gen.random_sparse(max(m, 17), kw, dens / 4, int(rng.integers(1 << 30)))
+    rows = np.concatenate([np.repeat(np.arange(A.m), np.diff(A.rowptr)), np.zeros(kw, np.int64)])
+    cols = np.concatenate([A.col, np.arange(kw)])
+    A = gen.from_coo(A.m, kw, rows, cols, rng.uniform(-1, 1, len(rows)))  # row 0 dense: its tile row is wide
+    return A, gen.random_sparse(kw, n, dens, int(rng.integers(1 << 30)))
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_random_parity_sweep(tsg, seed):
+    """Seeded random (A, B) of four structure kinds with ragged shapes; every pipeline (default,
+    per-C-tile, per-tile-row), every tile through the dense class, and fp32: all bit for bit
+    against the oracle's fma mode."""
+    rng = np.random.default_rng(7000 + seed)
+    for kind in range(4):
+        A, B = _sweep_case(rng, kind)
+        TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
+        ref = oracle.expected_tiles(A, B, fma=True)
+        for opts in ({}, dict(path_general=True), dict(path_rows=True), dict(path_rows=True, dense_threshold=1),
+                     dict(path_general=True, dense_threshold=1), dict(path_general=True, small_stage=True),
+                     dict(list_always=True, sort_only=True)):
+            assert_tiles_equal(host(tsg.spgemm(TA, TB, **opts)), ref), (seed, kind, opts)
+        A32, B32 = _typed(A, np.float32), _typed(B, np.float32)
+        got = host(tsg.spgemm(tiles_of(tsg, A32), tiles_of(tsg, B32)))
+        ref32 = oracle.expected_tiles(A32, B32, fma=True, prec="f32")
+        assert_tiles_equal(got, ref32, values=None)
+        assert bitwise_equal_values(got["val"].astype(np.float64), ref32.val.astype(np.float64)), (seed, kind)
