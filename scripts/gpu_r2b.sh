@@ -7,7 +7,8 @@ if [ "${STAGE:-1}" = "1" ]; then
   timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -15 > gpurun_out/r2b_pytest.log
   timeout 600 python bench.py > gpurun_out/r2b_bench_default.json 2> gpurun_out/r2b_bench_default.err
   timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/r2b_bench_ref.json 2> gpurun_out/r2b_bench_ref.err
-  for c in C1 C3 C4; do
+  timeout 600 python bench.py --config C1 --steps 50 --warmup 5 --no-cpu-baseline --e2e-steps 0 > gpurun_out/r2b_bench_C1.json 2> gpurun_out/r2b_bench_C1.err
+  for c in C3 C4; do
     timeout 600 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/r2b_bench_$c.json 2> gpurun_out/r2b_bench_$c.err
   done
   timeout 900 python bench.py --config C5 --steps 2 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/r2b_bench_C5.json 2> gpurun_out/r2b_bench_C5.err
