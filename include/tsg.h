@@ -147,10 +147,6 @@ typedef struct {
                                       for small calls or dense-tile-heavy A; TSG_PATH_GENERAL wins) */
 #define TSG_SMALL_STAGE_ON 0x100u  /* step 3 small tiles: stage B row metadata by cp.async (default: iff nnz(B) < 4 tiles(B)) */
 #define TSG_SMALL_STAGE_OFF 0x200u /* step 3 small tiles: plain dependent loads (same results either way) */
-#define TSG_MED_WARP 0x1000u /* step 3 medium tiles: a warp per tile, register accumulators over B rows staged
-                                densely in shared memory */
-#define TSG_MED_HALF 0x2000u /* step 3 medium tiles: a half warp per tile, row accumulators in shared memory
-                                (same results either way; TSG_MED_HALF wins) */
 #define TSG_DEBUG_HIGH_OFFSETS 0x800u /* test aid: steps 2-3 address C's nonzeros with offsets
                                         biased by 2^32 (high words set) against base pointers shifted back by
                                         2^32 elements, rebased at the end -- any 32-bit truncation of a
@@ -158,7 +154,7 @@ typedef struct {
 #define TSG_DENSE_THRESHOLD_SHIFT 16 /* bits 16..24: override t_nnz (0 = TSG_DENSE_NNZ; 257 disables dense) */
 #define TSG_QUEUE_CHUNK_SHIFT 25     /* bits 25..28: per-C-tile pipeline work distribution, v = 0: automatic,
                                         v = 1: static grid-stride, v >= 2: work queue with v-1 groups per request */
-#define TSG_SPGEMM_FLAGS 0x1fff3f7fu /* every defined bit (anything else is INVALID_ARG) */
+#define TSG_SPGEMM_FLAGS 0x1fff0f7fu /* every defined bit (anything else is INVALID_ARG) */
 
 /*
  * tsg_csr_to_tiles -- CSR -> sparse-tile format (Section 3.2; conversion is timed

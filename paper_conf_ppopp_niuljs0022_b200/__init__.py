@@ -220,8 +220,7 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
            structural: bool = False, scan_only: bool = False, list_always: bool = False,
            dense_threshold: int | None = None, sort_only: bool = False, path_general: bool = False,
            path_rows: bool = False, debug_high_offsets: bool = False,
-           small_stage: bool | None = None, med_warp: bool | None = None, queue_chunk: int | None = None,
-           stream=None) -> Tiles:
+           small_stage: bool | None = None, queue_chunk: int | None = None, stream=None) -> Tiles:
     """C = A*B in the sparse-tile format (tsg_spgemm: steps 1-3 of Section 3.3).
 
     stats / timing / products / structural: fill ``C.stats`` (one extra blocking read), with CUDA-
@@ -229,8 +228,7 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
     options select work splits only (the result is the same bit for bit): step-1 modes, the dense
     threshold t_nnz, ``path_general`` (the per-C-tile pipeline even for narrow tile rows), ``path_rows``
     (the fused per-tile-row pipeline wherever every tile row is narrow), ``debug_high_offsets`` (C's
-    nonzero offsets carry +2^32 inside the call: a test of the 64-bit offset paths), ``med_warp``
-    (step-3 medium tiles: warp per tile with register accumulators, or the half-warp kernel),
+    nonzero offsets carry +2^32 inside the call: a test of the 64-bit offset paths),
     ``queue_chunk`` (per-C-tile work distribution: 0 static, k > 0 k groups per request)."""
     L = _lib.load()
     flags = 0
@@ -254,8 +252,6 @@ def spgemm(A: Tiles, B: Tiles, stats: bool = False, timing: bool = False, produc
         flags |= _lib.DEBUG_HIGH_OFFSETS
     if small_stage is not None:
         flags |= _lib.SMALL_STAGE_ON if small_stage else _lib.SMALL_STAGE_OFF
-    if med_warp is not None:
-        flags |= _lib.MED_WARP if med_warp else _lib.MED_HALF
     if dense_threshold is not None:
         if not 1 <= dense_threshold <= 257:
             raise ValueError("dense_threshold must be in [1, 257]")

@@ -29,8 +29,6 @@ DEBUG_HIGH_OFFSETS = 0x800
 STEP1_SORT_ONLY = 0x40
 SMALL_STAGE_ON = 0x100
 SMALL_STAGE_OFF = 0x200
-MED_WARP = 0x1000
-MED_HALF = 0x2000
 DENSE_THRESHOLD_SHIFT = 16
 QUEUE_CHUNK_SHIFT = 25
 PATH_TILES, PATH_ROWS = 0, 1  # tsg_stats.path

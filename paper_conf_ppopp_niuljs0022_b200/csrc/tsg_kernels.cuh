@@ -147,7 +147,6 @@ struct StepParams {
     int dense_threshold;
     int small_max;         // step 3: tiles with nnz <= small_max take the lane-per-entry path
     int small_stage;       // step 3: k_s3_small stages B row metadata with cp.async (hypersparse B)
-    int med_warp;          // step 3 medium tiles: k_s3w (warp per tile, register accumulators), else k_s3
     const TileRec *recA, *recB;  // hypersparse operands: per-tile records (else nullptr)
     int64_t recA_voff;     // added to A records' value offsets (A a row slice inside B: B's offsets)
     DevCounters *cnt;

@@ -433,7 +433,6 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
         // small-tile B staging pays where B's tile metadata misses in cache: hypersparse tiles
         // (fewer than 4 nonzeros per B tile on average, e.g. R-MAT); flags force either way
         P.small_stage = (flags & TSG_SMALL_STAGE_ON) ? 1 : (flags & TSG_SMALL_STAGE_OFF) ? 0 : (B->nnz < 4 * B->nt);
-        P.med_warp = (flags & TSG_MED_HALF) ? 0 : (flags & TSG_MED_WARP) ? 1 : 0;
         P.recA = recA;
         P.recB = recB;
         // A's records are B's when A lies inside B: their value offsets count from B's values

@@ -815,219 +815,6 @@ __global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, i
     }
 }
 
-// ------------------------------------------------------------------------------------------
-// medium tiles, a warp per tile with register accumulators (the default medium class).
-// Lane (r = lane & 15, h = lane >> 4) owns C(r, 8h..8h+7) in eight registers.  Per pair the warp
-// scatters A_IK into a 16 x 17 staging tile (read only at A's structural positions, so never
-// cleared) and B_KJ into a 16 x 16 staging tile that is all zero between pairs (its entries are
-// reset after use).  Lane (r, h) walks c over mask_A[r] & rowOcc(B) in ascending order and, when
-// B's row c has an entry in its half, adds a * B(c, 8h..8h+7) with eight independent FMAs -- no
-// data-dependent loop over B's row and no accumulator loads or stores.  An absent B entry is an
-// exact zero, so a finite a adds +-0 (value unchanged, reading B2); a pair whose A tile holds a
-// non-finite value takes mask-predicated FMAs instead, so Inf * 0 never appears.  Products reach
-// C(r, j) in ascending k (pairs ascending K, then c ascending): bitwise equal to the other
-// classes.  The pairs of the warp's tiles form one stream: pair p+1's metadata and its first 64
-// nonzeros of each tile are loaded into registers while pair p multiplies (across tile ends too).
-constexpr int WAP = 17;  // A staging row pitch (elements)
-template <typename TO> __host__ __device__ constexpr int wbp() { return 16 + 16 / (int)sizeof(TO); }  // B pitch
-template <typename TO> __host__ __device__ constexpr int waoff() { return (16 * WAP * (int)sizeof(TO) + 15) / 16 * 16; }
-template <typename TO> __host__ __device__ constexpr int wbytes() { return waoff<TO>() + 16 * wbp<TO>() * (int)sizeof(TO); }
-
-template <typename TI>
-struct WPair {
-    int64_t zA = 0, zB = 0, pB = 0;
-    int nA = 0, nB = 0;
-    uint32_t mAr = 0;  // mask_A[r] & rowOcc(B)
-    uint32_t ix = 0;   // bytes: ixA[lane], ixA[lane + 32], ixB[lane], ixB[lane + 32]
-    TI a0{}, a1{}, b0{}, b1{};
-};
-
-template <typename TI>
-__device__ __forceinline__ void wfetch(const StepParams &P, uint64_t pr, int lane, int r, WPair<TI> &W) {
-    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
-    const int64_t pA = (int64_t)(pr >> 32), pB = (int64_t)(uint32_t)pr;
-    W.pB = pB;
-    W.zA = P.tnzA[pA];
-    W.nA = (int)(P.tnzA[pA + 1] - W.zA);
-    W.zB = P.tnzB[pB];
-    W.nB = (int)(P.tnzB[pB + 1] - W.zB);
-    W.mAr = (uint32_t)P.mA[pA * TILE + r] & (uint32_t)P.rowOccB[pB];
-    uint32_t ix = 0;
-    if (lane < W.nA) {
-        ix = P.ixA[W.zA + lane];
-        W.a0 = vA[W.zA + lane];
-    }
-    if (lane + 32 < W.nA) {
-        ix |= (uint32_t)P.ixA[W.zA + lane + 32] << 8;
-        W.a1 = vA[W.zA + lane + 32];
-    }
-    if (lane < W.nB) {
-        ix |= (uint32_t)P.ixB[W.zB + lane] << 16;
-        W.b0 = vB[W.zB + lane];
-    }
-    if (lane + 32 < W.nB) {
-        ix |= (uint32_t)P.ixB[W.zB + lane + 32] << 24;
-        W.b1 = vB[W.zB + lane + 32];
-    }
-    W.ix = ix;
-}
-
-#ifndef TSG_MEDW_MINB
-#define TSG_MEDW_MINB 5
-#endif
-template <typename TI, typename TO>
-__global__ void __launch_bounds__(T3, TSG_MEDW_MINB) k_s3w(StepParams P) {
-    constexpr int BPE = wbp<TO>();
-    __shared__ __align__(16) unsigned char wreg[T3 / 32][wbytes<TO>()];
-    const int lane = threadIdx.x & 31, r = lane & 15, h = lane >> 4;
-    TO *Ad = reinterpret_cast<TO *>(wreg[threadIdx.x >> 5]);
-    TO *Bd = reinterpret_cast<TO *>(wreg[threadIdx.x >> 5] + waoff<TO>());
-    const TI *vA = static_cast<const TI *>(P.vA), *vB = static_cast<const TI *>(P.vB);
-    TO *vC = static_cast<TO *>(P.vC);
-    for (int e = lane; e < TILE * BPE; e += 32) Bd[e] = (TO)0;
-    __syncwarp();
-    const int64_t ngroups = (P.ntC + 31) / 32;
-    WorkQueue wq(&P.cnt->q[3][0], ngroups, P.qchunk[3], lane, T3 / 32);
-    for (int64_t g; wq.next(g, lane);) {
-        unsigned mm = P.medL[g] | P.medH[g];  // the group's medium tiles (step 2 classified them)
-        if (!mm) continue;                    // warp-uniform
-        if (lane == 0) atomicAdd(&P.cnt->n3medium, (u64c)__popc(mm));
-        int64_t t = g * 32 + (__ffs(mm) - 1);
-        mm &= mm - 1;
-        uint32_t np = P.pairCnt[t];
-        const uint64_t *pp = P.pairs + P.pairBeg[t];
-        uint64_t prl = (uint32_t)lane < np ? pp[lane] : 0;
-        WPair<TI> cur;
-        wfetch<TI>(P, __shfl_sync(FULL, prl, 0), lane, r, cur);
-        for (;;) {
-            // the next tile's pair list head, loaded while this tile multiplies
-            int64_t t2 = -1;
-            uint32_t np2 = 0;
-            const uint64_t *pp2 = nullptr;
-            uint64_t prl2 = 0;
-            if (mm) {
-                t2 = g * 32 + (__ffs(mm) - 1);
-                mm &= mm - 1;
-                np2 = P.pairCnt[t2];
-                pp2 = P.pairs + P.pairBeg[t2];
-                prl2 = (uint32_t)lane < np2 ? pp2[lane] : 0;
-            }
-            const uint32_t mCr = P.mC[t * TILE + r];
-            const int64_t ob = P.tnzC[t] + P.rpC[t * TILE + r];
-            TO acc[8];
-#pragma unroll
-            for (int jj = 0; jj < 8; jj++) acc[jj] = (TO)0;
-            for (uint32_t p = 0; p < np; p++) {
-                // ---- stage pair p: scatter A and B, B's half-row occupancy, non-finite A
-                bool nf = false;
-                uint32_t hb = 0;  // bit 2c + h: row c of B has an entry in columns 8h..8h+7
-                {
-                    const uint32_t ia0 = cur.ix & 0xffu, ia1 = (cur.ix >> 8) & 0xffu;
-                    const uint32_t ib0 = (cur.ix >> 16) & 0xffu, ib1 = cur.ix >> 24;
-                    if (lane < cur.nA) {
-                        const TO v = vcvt<TO>(cur.a0);
-                        nf |= !isfinite(v);
-                        Ad[(ia0 >> 4) * WAP + (ia0 & 15u)] = v;
-                    }
-                    if (lane + 32 < cur.nA) {
-                        const TO v = vcvt<TO>(cur.a1);
-                        nf |= !isfinite(v);
-                        Ad[(ia1 >> 4) * WAP + (ia1 & 15u)] = v;
-                    }
-                    if (lane < cur.nB) {
-                        Bd[(ib0 >> 4) * BPE + (ib0 & 15u)] = vcvt<TO>(cur.b0);
-                        hb |= 1u << (2 * (ib0 >> 4) + ((ib0 >> 3) & 1u));
-                    }
-                    if (lane + 32 < cur.nB) {
-                        Bd[(ib1 >> 4) * BPE + (ib1 & 15u)] = vcvt<TO>(cur.b1);
-                        hb |= 1u << (2 * (ib1 >> 4) + ((ib1 >> 3) & 1u));
-                    }
-                    for (int e = 64 + lane; e < cur.nA; e += 32) {  // tiles beyond 64 nonzeros
-                        const uint32_t ix = P.ixA[cur.zA + e];
-                        const TO v = vcvt<TO>(vA[cur.zA + e]);
-                        nf |= !isfinite(v);
-                        Ad[(ix >> 4) * WAP + (ix & 15u)] = v;
-                    }
-                    for (int e = 64 + lane; e < cur.nB; e += 32) {
-                        const uint32_t ix = P.ixB[cur.zB + e];
-                        Bd[(ix >> 4) * BPE + (ix & 15u)] = vcvt<TO>(vB[cur.zB + e]);
-                        hb |= 1u << (2 * (ix >> 4) + ((ix >> 3) & 1u));
-                    }
-                }
-                hb = __reduce_or_sync(FULL, hb);
-                const bool anynf = __any_sync(FULL, nf);
-                __syncwarp();
-                // ---- pair p+1 (or the next tile's first pair) into registers
-                WPair<TI> nxt;
-                if (p + 1 < np) {
-                    if (((p + 1) & 31u) == 0) prl = p + 1 + lane < np ? pp[p + 1 + lane] : 0;
-                    wfetch<TI>(P, __shfl_sync(FULL, prl, (p + 1) & 31u), lane, r, nxt);
-                } else if (t2 >= 0) {
-                    wfetch<TI>(P, __shfl_sync(FULL, prl2, 0), lane, r, nxt);
-                }
-                // ---- multiply
-                uint32_t m = cur.mAr;
-                const TO *arow = Ad + r * WAP;
-                const TO *bh = Bd + 8 * h;
-                if (!anynf) {
-                    while (m) {
-                        const int c = __ffs(m) - 1;
-                        m &= m - 1;
-                        if ((hb >> (2 * c + h)) & 1u) {
-                            const TO a = arow[c];
-                            TO b[8];
-                            lds8(bh + c * BPE, b);
-#pragma unroll
-                            for (int jj = 0; jj < 8; jj++) acc[jj] = vfma(a, b[jj], acc[jj]);
-                        }
-                    }
-                } else {
-                    const uint16_t *mbt = P.mB + cur.pB * TILE;
-                    while (m) {
-                        const int c = __ffs(m) - 1;
-                        m &= m - 1;
-                        const uint32_t mb = ((uint32_t)mbt[c] >> (8 * h)) & 0xffu;
-                        if (mb) {
-                            const TO a = arow[c];
-#pragma unroll
-                            for (int jj = 0; jj < 8; jj++)
-                                if ((mb >> jj) & 1u) acc[jj] = vfma(a, bh[c * BPE + jj], acc[jj]);
-                        }
-                    }
-                }
-                __syncwarp();
-                // ---- reset B's staged entries to zero for the next pair
-                {
-                    const uint32_t ib0 = (cur.ix >> 16) & 0xffu, ib1 = cur.ix >> 24;
-                    if (lane < cur.nB) Bd[(ib0 >> 4) * BPE + (ib0 & 15u)] = (TO)0;
-                    if (lane + 32 < cur.nB) Bd[(ib1 >> 4) * BPE + (ib1 & 15u)] = (TO)0;
-                    for (int e = 64 + lane; e < cur.nB; e += 32) {
-                        const uint32_t ix = P.ixB[cur.zB + e];
-                        Bd[(ix >> 4) * BPE + (ix & 15u)] = (TO)0;
-                    }
-                }
-                __syncwarp();
-                cur = nxt;
-            }
-            // ---- compaction through mask_C[r]
-#pragma unroll
-            for (int jj = 0; jj < 8; jj++) {
-                const int j = 8 * h + jj;
-                if ((mCr >> j) & 1u) {
-                    const int64_t o = ob + __popc(mCr & ((1u << j) - 1u));
-                    P.ixC[o] = (uint8_t)((r << 4) | j);
-                    vC[o] = acc[jj];
-                }
-            }
-            if (t2 < 0) break;
-            t = t2;
-            np = np2;
-            pp = pp2;
-            prl = prl2;
-        }
-    }
-}
-
 // Launch shape of a step-2/3 kernel over `units` work units (groups of 32 C tiles), `wpc` warps
 // per CTA.  Many units per warp: a persistent grid (the CTAs resident at once: SM count x
 // occupancy) with the work queue, so the warps running at any moment work on neighbouring C tiles
@@ -1098,11 +885,7 @@ static void launch_step3_t(const StepParams &P, int64_t n_dense, cudaStream_t s)
             TSG_LAUNCH((k_s3_small<TI, TO, 0>), sp.grid, TS, 0, s, Q);
         }
     }
-    if (P.med_warp) {
-        const Shape sp = step_shape(k_s3w<TI, TO>, T3, groups, P.qoverride);
-        Q.qchunk[3] = sp.chunk;
-        TSG_LAUNCH((k_s3w<TI, TO>), sp.grid, T3, 0, s, Q);
-    } else {
+    {
         const Shape sp = step_shape(k_s3<TI, TO>, T3, groups, P.qoverride);
         Q.qchunk[3] = sp.chunk;
         TSG_LAUNCH((k_s3<TI, TO>), sp.grid, T3, 0, s, Q);

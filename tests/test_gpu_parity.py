@@ -134,16 +134,15 @@ def pair_cases():
 PAIRS = pair_cases()
 
 
-@pytest.mark.parametrize("mode", ["default", "per-tile", "per-tile-medwarp", "per-tile-medhalf", "rows"])
+@pytest.mark.parametrize("mode", ["default", "per-tile", "rows"])
 @pytest.mark.parametrize("name,A,B", PAIRS, ids=[p[0] for p in PAIRS])
 def test_spgemm_matches_oracle(tsg, name, A, B, mode):
     """Both pipelines against the oracle: the default dispatch, the per-C-tile pipeline forced with
     path_general, and the row path forced wherever every tile row of A is narrow (path_rows)."""
     TA, TB = tiles_of(tsg, A), tiles_of(tsg, B)
-    general = mode.startswith("per-tile")
-    med = {"per-tile-medwarp": True, "per-tile-medhalf": False}.get(mode)
+    general = mode == "per-tile"
     C = tsg.spgemm(TA, TB, stats=True, products=True, structural=True, path_general=general,
-                   path_rows=mode == "rows", med_warp=med)
+                   path_rows=mode == "rows")
     ref = oracle.expected_tiles(A, B)
     ref_fma = oracle.expected_tiles(A, B, fma=True)
     got = host(C)
@@ -180,8 +179,7 @@ def _abs_csr(A, B):
                                   dict(path_rows=True, list_always=True),
                                   dict(sort_only=True), dict(sort_only=True, list_always=True),
                                   dict(sort_only=True, scan_only=True), dict(small_stage=True, path_general=True),
-                                  dict(small_stage=False, path_general=True), dict(med_warp=True, path_general=True),
-                                  dict(med_warp=False, path_general=True)])
+                                  dict(small_stage=False, path_general=True)])
 def test_modes_give_identical_results(tsg, opts):
     """Step-1 modes and the accumulator threshold change the work split, never the result."""
     for A in (gen.rmat(11), gen.strip_fem(6, 20, 6), gen.config("C1"), gen.stencil27(12),
@@ -606,7 +604,7 @@ def test_unknown_flags_rejected(tsg):
     A = gen.config("C1")
     T = tiles_of(tsg, A)
     out = C.c_void_p()
-    for bad in (0x80, 0x4000, 1 << 29):  # 0x80: the removed tensor-core flag
+    for bad in (0x80, 0x8000, 1 << 29):  # 0x80: the removed tensor-core flag
         rc = _lib.load().tsg_spgemm(T.ptr, T.ptr, bad, None, None, C.byref(out), None)
         assert rc == 1 and out.value is None
 
@@ -791,7 +789,6 @@ def test_random_parity_sweep(tsg, seed):
         ref = oracle.expected_tiles(A, B, fma=True)
         for opts in ({}, dict(path_general=True), dict(path_rows=True), dict(path_rows=True, dense_threshold=1),
                      dict(path_general=True, dense_threshold=1), dict(path_general=True, small_stage=True),
-                     dict(path_general=True, med_warp=True), dict(path_general=True, med_warp=False),
                      dict(list_always=True, sort_only=True)):
             assert_tiles_equal(host(tsg.spgemm(TA, TB, **opts)), ref), (seed, kind, opts)
         A32, B32 = _typed(A, np.float32), _typed(B, np.float32)
