@@ -475,3 +475,23 @@ def test_c1_golden_statistics_reproduce_with_scipy():
     out = subprocess.run([sys.executable, os.path.join(root, "scripts", "golden_c1_stats.py"), "--check"],
                          capture_output=True, text=True, cwd=root)
     assert out.returncode == 0, out.stdout + out.stderr
+
+
+def test_spmv_pinned_by_dense_matvec():
+    """orc_spmv (the helper of the row-sum invariant) against the dense matrix-vector product: exact
+    on small integers (no rounding), and within the recursive-summation bound on random values;
+    empty rows give 0."""
+    rng = np.random.default_rng(11)
+    for m, n, dens in ((1, 1, 1.0), (7, 5, 0.5), (40, 33, 0.1), (64, 64, 0.0)):
+        A = gen.random_sparse(m, n, dens, seed=m + n)
+        D = csr_dense(m, n, A.rowptr, A.col, A.val)
+        # integer values: every partial sum is exact in fp64
+        Ai = gen.CSR(m, n, A.rowptr, A.col, np.round(A.val * 8.0))
+        xi = rng.integers(-5, 6, n).astype(np.float64)
+        Di = csr_dense(m, n, Ai.rowptr, Ai.col, Ai.val)
+        assert np.array_equal(oracle.spmv(Ai, xi), Di @ xi)
+        x = rng.uniform(-1, 1, n)
+        y = oracle.spmv(A, x)
+        bound = np.abs(D) @ np.abs(x) * (n * np.finfo(np.float64).eps) + 1e-300
+        assert np.all(np.abs(y - D @ x) <= bound)
+        assert np.all(y[np.diff(A.rowptr) == 0] == 0.0)
