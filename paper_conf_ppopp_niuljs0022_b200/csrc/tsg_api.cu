@@ -119,7 +119,7 @@ void Allocator::free(void *p, size_t bytes, cudaStream_t s) const {
 // behind whatever the copy engine is already doing (a caller streaming the previous result to
 // the host), a kernel's posted writes do not.
 namespace {
-__global__ void k_export(ExportArgs a) { export_segments(a); }
+__global__ void k_export(ExportArgs a) { TSG_GRID_WAIT(); export_segments(a); }
 struct Mapped {
     uint8_t *h = nullptr;
     uint8_t *d = nullptr;
@@ -205,13 +205,13 @@ int64_t read_scalar(const int64_t *dptr, cudaStream_t s) {
 }
 
 namespace {
-__global__ void k_rebase(const int64_t *__restrict__ src, int64_t *__restrict__ dst, int64_t count) {
+__global__ void k_rebase(const int64_t *__restrict__ src, int64_t *__restrict__ dst, int64_t count) { TSG_GRID_WAIT();
     int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < count) dst[i] = src[i] - src[0];
 }
 }  // namespace
 
-__global__ void k_add_i64(int64_t *__restrict__ a, int64_t count, int64_t v) {
+__global__ void k_add_i64(int64_t *__restrict__ a, int64_t count, int64_t v) { TSG_GRID_WAIT();
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < count) a[i] += v;
 }

@@ -39,7 +39,7 @@ __device__ __forceinline__ int half_excl_scan(int v, int r, int *total) {
 // row_ptr[m] != nnz: the arrays are sized by nnz), else 1 for unsorted / duplicate / out-of-range
 // columns (reading A12)
 __global__ void k_validate_csr(int64_t m, int64_t n, int64_t nnz, const int64_t *__restrict__ rp,
-                               const int32_t *__restrict__ ci, int *__restrict__ bad) {
+                               const int32_t *__restrict__ ci, int *__restrict__ bad) { TSG_GRID_WAIT();
     int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     int64_t b = rp[i], e = rp[i + 1];
@@ -60,7 +60,7 @@ __global__ void k_validate_csr(int64_t m, int64_t n, int64_t nnz, const int64_t 
 
 // pass 1: number of non-empty tiles per tile row
 __global__ void __launch_bounds__(256) k_c2t_count(int64_t m, int64_t tm, const int64_t *__restrict__ rp,
-                                                   const int32_t *__restrict__ ci, int64_t *__restrict__ ntiles) {
+                                                   const int32_t *__restrict__ ci, int64_t *__restrict__ ntiles) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t I = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     const bool active = I < tm;
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(256) k_c2t_fill(int64_t m, int64_t tm, const i
                                                   const int64_t *__restrict__ tile_ptr, int32_t *__restrict__ tile_col,
                                                   int64_t *__restrict__ tile_nnz, uint8_t *__restrict__ row_ptr,
                                                   uint16_t *__restrict__ mask, uint8_t *__restrict__ idx,
-                                                  W *__restrict__ val) {
+                                                  W *__restrict__ val) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t I = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     const bool active = I < tm;
@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(256) k_c2t_fill(int64_t m, int64_t tm, const i
     }
 }
 
-__global__ void k_set_i64(int64_t *p, int64_t v) { *p = v; }
+__global__ void k_set_i64(int64_t *p, int64_t v) { TSG_GRID_WAIT(); *p = v; }
 
 // tiles -> CSR: lane r of a half owns global row 16I+r; row lengths are popcounts of the row's
 // masks across the tile row; the CSR row offsets follow from the tile row's nonzero base.
@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(256) k_t2c(int64_t m, int64_t tm, const int64_
                                              const uint8_t *__restrict__ row_ptr, const uint16_t *__restrict__ mask,
                                              const uint8_t *__restrict__ idx, const W *__restrict__ val,
                                              int64_t *__restrict__ out_rp, int32_t *__restrict__ out_ci,
-                                             W *__restrict__ out_v) {
+                                             W *__restrict__ out_v) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t I = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     const bool active = I < tm;

@@ -2,6 +2,8 @@
 // Nothing here is visible through the C ABI (include/tsg.h).
 #pragma once
 
+#include <utility>
+
 #include <initializer_list>
 
 #include <cuda_runtime.h>
@@ -49,13 +51,49 @@ void set_last_error(const std::string &msg);
 // launch bookkeeping: every kernel goes through TSG_LAUNCH so the evidence counter is exact
 extern std::atomic<int64_t> g_launches;
 
+// Programmatic dependent launch (sm_90+): every kernel is launched with programmatic stream
+// serialization, and every kernel's first statement is TSG_GRID_WAIT() (griddepcontrol.wait:
+// block until the preceding kernel of the stream has completed and its writes are visible), so
+// stream order is kept while the next launch is prepared during the previous kernel's tail --
+// chains of small kernels (C1-sized calls) lose part of the per-launch gap.  TSG_PDL=0 builds
+// plain launches.
+#ifndef TSG_PDL
+#define TSG_PDL 1
+#endif
+#if defined(__CUDA_ARCH__)
+#define TSG_GRID_WAIT() asm volatile("griddepcontrol.wait;\n" ::: "memory")
+#else
+#define TSG_GRID_WAIT()
+#endif
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
+                              Args &&...args) {
+#if TSG_PDL
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+#else
+    kernel<<<grid, block, smem, s>>>(std::forward<Args>(args)...);
+    return cudaGetLastError();
+#endif
+}
+
 #define TSG_LAUNCH(kernel, grid, block, smem, stream, ...)                                     \
     do {                                                                                        \
         if ((grid) > 0) {                                                                       \
-            kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);                         \
+            TSG_CUDA(::tsg::launch_pdl(kernel, (unsigned)(grid), (unsigned)(block), (size_t)(smem), \
+                                       (stream), ##__VA_ARGS__));                               \
             ::tsg::g_launches.fetch_add(1, std::memory_order_relaxed);                          \
             ::tsg::note_launch();                                                               \
-            TSG_CUDA(cudaGetLastError());                                                       \
         }                                                                                       \
     } while (0)
 

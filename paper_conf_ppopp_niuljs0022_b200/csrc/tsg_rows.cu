@@ -209,7 +209,7 @@ __device__ __forceinline__ void medium_tile(const RowNumParams &P, bool hv, int6
 // full-warp reconvergence after every pair: adjacent tile rows of a stencil have the same
 // structure, so both halves run the same instruction stream on all 32 lanes.
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
+__global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) { TSG_GRID_WAIT();
     __shared__ __align__(16) unsigned char smem[RN_W][WARP_SMEM];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
     const int64_t I0 = ((int64_t)blockIdx.x * RN_W + w) * 2;
@@ -326,7 +326,7 @@ __global__ void __launch_bounds__(RN_T, RN_MINB) k_num_rows(RowNumParams P) {
 // mask_A[r] & colmask_B[j] in ascending order.  Warps take 32 records at a time.
 constexpr int NS_T = 256;
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) {
+__global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) { TSG_GRID_WAIT();
     __shared__ uint8_t mapsm[NS_T / 32][32 * 16];
     const int lane = threadIdx.x & 31;
     uint8_t *map = mapsm[threadIdx.x >> 5];
@@ -416,7 +416,7 @@ __global__ void __launch_bounds__(NS_T, 5) k_num_small(RowNumParams P) {
 constexpr int DR_W = 4;  // warps per CTA
 constexpr int DR_AP = 17;  // staged A row pitch (values): conflict-free column reads
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(DR_W * 32) k_num_dense_row(RowNumParams P) {
+__global__ void __launch_bounds__(DR_W * 32) k_num_dense_row(RowNumParams P) { TSG_GRID_WAIT();
     extern __shared__ __align__(16) unsigned char dyn[];
     __shared__ int64_t dOff[32];
     __shared__ uint8_t dQ[32], sNF[MAX_A];

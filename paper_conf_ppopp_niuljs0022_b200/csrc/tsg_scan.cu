@@ -62,7 +62,7 @@ __device__ __forceinline__ void st_status(uint64_t *p, uint64_t v) {
 
 template <typename Tin>
 __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n, int64_t *out, uint64_t *status,
-                                                      unsigned long long *ticket, ExportArgs ex) {
+                                                      unsigned long long *ticket, ExportArgs ex) { TSG_GRID_WAIT();
     __shared__ int64_t s_bid, s_base;
     if (threadIdx.x == 0) s_bid = gridDim.x == 1 ? 0 : (int64_t)atomicAdd(ticket, 1ull);
     __syncthreads();
@@ -112,8 +112,8 @@ __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n,
     if (ex.n && b == (int64_t)gridDim.x - 1) export_segments(ex);  // the CTA that wrote out[n]
 }
 
-__global__ void k_set_zero_i64(int64_t *p) { *p = 0; }
-__global__ void k_export_only(ExportArgs a) { export_segments(a); }
+__global__ void k_set_zero_i64(int64_t *p) { TSG_GRID_WAIT(); *p = 0; }
+__global__ void k_export_only(ExportArgs a) { TSG_GRID_WAIT(); export_segments(a); }
 
 }  // namespace
 

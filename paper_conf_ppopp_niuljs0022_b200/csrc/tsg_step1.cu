@@ -26,7 +26,7 @@ __device__ __forceinline__ int bits_for(uint64_t v) {  // bits needed to represe
 // A pair (A_IK, B_KJ) has a product iff colOcc(A_IK) & rowOcc(B_KJ) != 0.
 // ------------------------------------------------------------------------------------------
 __global__ void k_occupancy(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ row_occ,
-                            uint16_t *__restrict__ col_occ, uint64_t *__restrict__ zero, int zero_words) {
+                            uint16_t *__restrict__ col_occ, uint64_t *__restrict__ zero, int zero_words) { TSG_GRID_WAIT();
     if (blockIdx.x == 0)  // the call's device counters start at zero (saves a memset launch)
         for (int i = threadIdx.x; i < zero_words; i += blockDim.x) zero[i] = 0;
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -50,7 +50,7 @@ __global__ void k_occupancy(const uint16_t *__restrict__ mask, int64_t nt, uint1
 template <typename TI>
 __global__ void k_tile_records(int64_t nt, const int32_t *__restrict__ tile_col, const int64_t *__restrict__ tile_nnz,
                                const uint16_t *__restrict__ mask, const uint8_t *__restrict__ idx,
-                               const TI *__restrict__ val, TileRec *__restrict__ rec) {
+                               const TI *__restrict__ val, TileRec *__restrict__ rec) { TSG_GRID_WAIT();
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nt) return;
     const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
@@ -79,7 +79,7 @@ __global__ void k_tile_records(int64_t nt, const int32_t *__restrict__ tile_col,
 // k%16 is non-empty, ascending tile column.  One warp = two B tile rows, lane r = row r.
 __global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__restrict__ tpB,
                                                  const uint16_t *__restrict__ maskB, const int64_t *__restrict__ lptr,
-                                                 int32_t *__restrict__ lcnt, uint32_t *__restrict__ list) {
+                                                 int32_t *__restrict__ lcnt, uint32_t *__restrict__ list) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t K = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     if (K >= tmB) return;
@@ -97,7 +97,7 @@ __global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__r
 
 // stats only: nnz of every global row of B, then products per A tile
 __global__ void __launch_bounds__(256) k_brow_nnz(int64_t tmB, const int64_t *__restrict__ tpB,
-                                                  const uint16_t *__restrict__ maskB, int32_t *__restrict__ rnnz) {
+                                                  const uint16_t *__restrict__ maskB, int32_t *__restrict__ rnnz) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t K = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     if (K >= tmB) return;
@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(256) k_brow_nnz(int64_t tmB, const int64_t *__
 }
 
 __global__ void k_products(int64_t ntA, const int32_t *__restrict__ tcA, const uint16_t *__restrict__ maskA,
-                           const int32_t *__restrict__ rnnz, DevCounters *cnt) {
+                           const int32_t *__restrict__ rnnz, DevCounters *cnt) { TSG_GRID_WAIT();
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     u64c p = 0;
     if (t < ntA) {
@@ -133,7 +133,7 @@ __global__ void k_products(int64_t ntA, const int32_t *__restrict__ tcA, const u
 // ------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_structural(const int64_t *__restrict__ tpA, const int32_t *__restrict__ tcA,
                                                    const int64_t *__restrict__ tpB, const int32_t *__restrict__ tcB,
-                                                   int words, DevCounters *cnt) {
+                                                   int words, DevCounters *cnt) { TSG_GRID_WAIT();
     extern __shared__ uint32_t bm[];
     const int64_t I = blockIdx.x;
     for (int w = threadIdx.x; w < words; w += blockDim.x) bm[w] = 0;
@@ -160,7 +160,7 @@ __global__ void __launch_bounds__(256) k_structural(const int64_t *__restrict__ 
 // ------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_row_products(int64_t tmA, const int64_t *__restrict__ tpA,
                                                      const int32_t *__restrict__ tcA, const uint16_t *__restrict__ maskA,
-                                                     const int32_t *__restrict__ rnnz, int64_t *__restrict__ w) {
+                                                     const int32_t *__restrict__ rnnz, int64_t *__restrict__ w) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31;
     const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (I >= tmA) return;
@@ -181,7 +181,7 @@ __global__ void __launch_bounds__(256) k_row_products(int64_t tmA, const int64_t
     if (lane == 0) w[I] = p;
 }
 
-__global__ void k_cuts(const int64_t *__restrict__ pre, int64_t tm, int64_t parts, int64_t *__restrict__ cuts) {
+__global__ void k_cuts(const int64_t *__restrict__ pre, int64_t tm, int64_t parts, int64_t *__restrict__ cuts) { TSG_GRID_WAIT();
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const int64_t total = pre[tm];
     int64_t prev = 0;
@@ -211,7 +211,7 @@ __global__ void k_atile_plan(int64_t ntA, const int32_t *__restrict__ tcA, const
                              const int64_t *__restrict__ tpB, const int32_t *__restrict__ tcB,
                              const int64_t *__restrict__ lptr, const uint32_t *__restrict__ list, bool scan_only,
                              int64_t *__restrict__ cost, int64_t *__restrict__ start, int32_t *__restrict__ jlo,
-                             int32_t *__restrict__ jhi, DevCounters *cnt) {
+                             int32_t *__restrict__ jhi, DevCounters *cnt) { TSG_GRID_WAIT();
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     bool is_list = false;
     if (t < ntA) {
@@ -247,7 +247,7 @@ __global__ void k_row_plan(int64_t tmA, const int64_t *__restrict__ tpA, const i
                            const int32_t *__restrict__ jloA, const int32_t *__restrict__ jhiA, bool merge,
                            int32_t *__restrict__ rowJlo, int32_t *__restrict__ rowJhi, uint8_t *__restrict__ rowClass,
                            int64_t *__restrict__ nC, int32_t *__restrict__ bigList, int64_t *__restrict__ bigOff,
-                           int32_t *__restrict__ smallList, DevCounters *cnt) {
+                           int32_t *__restrict__ smallList, DevCounters *cnt) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31;
     const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (I >= tmA) return;
@@ -646,7 +646,7 @@ __device__ uint32_t merge_row(const S1Params &P, int64_t I, int lane, uint32_t *
     return out.ntl;
 }
 
-__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) {
+__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) { TSG_GRID_WAIT();
     __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
     __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -669,7 +669,7 @@ __global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t 
 // the row-offset scan, the count of dense C tiles to the call's counters.
 // ------------------------------------------------------------------------------------------
 constexpr int SYM_SMEM = 1024 + 2 * 576;  // per warp: A row masks [32][16], two half-warp batches
-__global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t tm) {
+__global__ void __launch_bounds__(MERGE_W * 32) k_sym_rows(S1Params P, int64_t tm) { TSG_GRID_WAIT();
     __shared__ __align__(16) unsigned char sR[MERGE_W][SYM_SMEM];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t I = (int64_t)blockIdx.x * MERGE_W + w;
@@ -773,7 +773,7 @@ __device__ __forceinline__ bool scratch_fits(const S1Params &P) {
     return ok;
 }
 
-__global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int cap) {
+__global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int cap) { TSG_GRID_WAIT();
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t hist[256 * ROW_NW];
     __shared__ int sm[ROW_NW + 1];
@@ -798,7 +798,7 @@ __global__ void __launch_bounds__(ROW_T) k_row_small(S1Params P, int cap) {
     }
 }
 
-__global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) {
+__global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) { TSG_GRID_WAIT();
     __shared__ uint32_t hist[256 * ROW_NW];
     __shared__ int sm[ROW_NW + 1];
     if (!scratch_fits(P)) return;
@@ -858,7 +858,7 @@ __device__ __forceinline__ int64_t block_excl_scan64(int64_t v, int64_t *total, 
 
 __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t *bm, int64_t *sm);
 
-__global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) {
+__global__ void __launch_bounds__(RANK_T) k_row_rank(S1Params P, int wwords) { TSG_GRID_WAIT();
     extern __shared__ uint32_t bm[];  // [wwords] bitmap, then [wwords] exclusive popcount prefix
     __shared__ int64_t sm[RANK_NW + 1];
     if (!scratch_fits(P)) return;
@@ -1015,7 +1015,7 @@ __device__ __forceinline__ uint64_t transpose8(uint64_t x) {
 
 // transposed masks (maskT[c] bit r <=> mask[r] bit c): the 16x16 tile as four 8x8 blocks,
 // gathered with byte permutes, transposed in 64-bit words and scattered back
-__global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ maskT) {
+__global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint16_t *__restrict__ maskT) { TSG_GRID_WAIT();
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nt) return;
     const uint4 *p = reinterpret_cast<const uint4 *>(mask + t * TILE);
@@ -1051,7 +1051,7 @@ __global__ void k_transpose(const uint16_t *__restrict__ mask, int64_t nt, uint1
 // (ROWCTA: a CTA per tile row, for rows of thousands of C tiles -- R-MAT -- where a warp per row
 // serialises the long rows)
 template <bool ROWCTA>
-__global__ void __launch_bounds__(256) k_compact(CompactParams P) {
+__global__ void __launch_bounds__(256) k_compact(CompactParams P) { TSG_GRID_WAIT();
     const int lane = ROWCTA ? (int)threadIdx.x : (int)(threadIdx.x & 31);
     const int step = ROWCTA ? 256 : 32;
     const int64_t I = ROWCTA ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);

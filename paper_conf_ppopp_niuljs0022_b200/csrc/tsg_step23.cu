@@ -55,7 +55,7 @@ constexpr int BATCH3 = 16; // step 3: pairs staged per half warp at a time (also
 // loaded while the current pair is OR-ed.
 constexpr int T2L = 256;
 
-__global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
+__global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) { TSG_GRID_WAIT();
     __shared__ uint32_t wsm[8 * T2L];
     uint32_t *w = wsm + threadIdx.x;
     const int lane = threadIdx.x & 31;
@@ -174,7 +174,7 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) {
     if ((threadIdx.x & 31) == 0 && nd) atomicAdd(&P.cnt->n2dense, nd);
 }
 
-__global__ void __launch_bounds__(T2) k_s2(StepParams P) {
+__global__ void __launch_bounds__(T2) k_s2(StepParams P) { TSG_GRID_WAIT();
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
@@ -305,7 +305,7 @@ __device__ __forceinline__ TO rec_value(const uint4 &r) {
 }
 
 template <typename TI, typename TO, int MODE>  // MODE 0: plain, 1: STAGE, 2: REC
-__global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) {
+__global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) { TSG_GRID_WAIT();
     constexpr bool STAGE = MODE == 1;
     __shared__ uint8_t mapsm[TS / 32][SMAP];
     __shared__ __align__(16) uint4 stg[STAGE ? 2 : 1][3][STAGE ? TS : 1];
@@ -750,7 +750,7 @@ template <typename TI, typename TO>
 #ifndef TSG_MED_MINB
 #define TSG_MED_MINB 7
 #endif
-__global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
+__global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) { TSG_GRID_WAIT();
     __shared__ __align__(16) unsigned char wreg[T3 / 32][WREG];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, r = lane & 15, half = lane >> 4;
     unsigned char *wr = wreg[w];
@@ -790,7 +790,7 @@ __global__ void __launch_bounds__(T3, TSG_MED_MINB) k_s3(StepParams P) {
 #endif
 constexpr int DREG = 2176 + 2048;  // per-warp staging of the dense path: A 16 x 17 and B 16 x 16 (fp64)
 template <typename TI, typename TO>
-__global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, int split) {
+__global__ void __launch_bounds__(T3, TSG_DENSE_MINB) k_s3_dense(StepParams P, int split) { TSG_GRID_WAIT();
     __shared__ __align__(16) unsigned char wreg[T3 / 32][DREG];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     unsigned char *wr = wreg[w];

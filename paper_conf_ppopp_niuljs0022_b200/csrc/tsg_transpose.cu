@@ -18,7 +18,7 @@
 namespace tsg {
 namespace {
 
-__global__ void k_tp_count(int64_t nt, const int32_t *__restrict__ tcol, unsigned long long *__restrict__ cnt) {
+__global__ void k_tp_count(int64_t nt, const int32_t *__restrict__ tcol, unsigned long long *__restrict__ cnt) { TSG_GRID_WAIT();
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t < nt) atomicAdd(&cnt[tcol[t]], 1ULL);
 }
@@ -26,7 +26,7 @@ __global__ void k_tp_count(int64_t nt, const int32_t *__restrict__ tcol, unsigne
 // warp per tile row I of A: its tiles go to their column's slot range (any order)
 __global__ void k_tp_place(int64_t tm, const int64_t *__restrict__ tp, const int32_t *__restrict__ tcol,
                            unsigned long long *__restrict__ cursor, int32_t *__restrict__ slotI,
-                           int64_t *__restrict__ slotSrc) {
+                           int64_t *__restrict__ slotSrc) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31;
     const int64_t I = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (I >= tm) return;
@@ -43,7 +43,7 @@ __global__ void k_tp_place(int64_t tm, const int64_t *__restrict__ tp, const int
 constexpr int TP_SMALL = 64;
 __global__ void k_tp_rank(int64_t tn, const int64_t *__restrict__ tpT, const int32_t *__restrict__ slotI,
                           const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
-                          int32_t *__restrict__ tcolT, int32_t *__restrict__ wide, unsigned long long *nwide) {
+                          int32_t *__restrict__ tcolT, int32_t *__restrict__ wide, unsigned long long *nwide) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31;
     const int64_t J = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (J >= tn) return;
@@ -66,7 +66,7 @@ __global__ void k_tp_rank(int64_t tn, const int64_t *__restrict__ tpT, const int
 __global__ void k_tp_rank_all(int64_t tn, const int64_t *__restrict__ tpT, const int32_t *__restrict__ slotI,
                               const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
                               int32_t *__restrict__ tcolT, const int32_t *__restrict__ wide,
-                              const unsigned long long *nwide) {
+                              const unsigned long long *nwide) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31;
     const int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (k >= (int64_t)*nwide) return;
@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(TPW_T) k_tp_rank_wide(int64_t tm, const int64_
                                                        const int32_t *__restrict__ slotI,
                                                        const int64_t *__restrict__ slotSrc, int64_t *__restrict__ perm,
                                                        int32_t *__restrict__ tcolT, const int32_t *__restrict__ wide,
-                                                       const unsigned long long *nwide) {
+                                                       const unsigned long long *nwide) { TSG_GRID_WAIT();
     extern __shared__ uint32_t bm[];  // [words] bitmap, [words] exclusive popcount prefix
     __shared__ uint32_t wsum[TPW_T / 32 + 1];
     const int words = (int)((tm + 31) / 32);
@@ -145,7 +145,7 @@ __global__ void __launch_bounds__(TPW_T) k_tp_rank_wide(int64_t tm, const int64_
 }
 
 __global__ void k_tp_nnz(int64_t nt, const int64_t *__restrict__ perm, const int64_t *__restrict__ tnz,
-                         int64_t *__restrict__ tnzT) {
+                         int64_t *__restrict__ tnzT) { TSG_GRID_WAIT();
     const int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (d < nt) tnzT[d] = tnz[perm[d] + 1] - tnz[perm[d]];
 }
@@ -156,7 +156,7 @@ __global__ void k_tp_fill(int64_t nt, const int64_t *__restrict__ perm, const in
                           const uint16_t *__restrict__ mask, const uint16_t *__restrict__ maskTs,
                           const W *__restrict__ val, const int64_t *__restrict__ tnzT,
                           uint8_t *__restrict__ rpT, uint16_t *__restrict__ maskT, uint8_t *__restrict__ idxT,
-                          W *__restrict__ valT) {
+                          W *__restrict__ valT) { TSG_GRID_WAIT();
     const int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (d >= nt) return;
     const int64_t t = perm[d];
