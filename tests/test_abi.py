@@ -85,3 +85,23 @@ def test_product_package_never_imports_the_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 text = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in text and "from oracle" not in text and "tsg_oracle" not in text, f
+
+
+def test_every_kernel_waits_on_its_predecessor():
+    """Every kernel is launched with programmatic stream serialization (TSG_LAUNCH -> launch_pdl), so
+    each __global__ function must open with TSG_GRID_WAIT() (griddepcontrol.wait) before it reads
+    anything a preceding kernel wrote; and no kernel is launched outside TSG_LAUNCH."""
+    csrc = os.path.join(ROOT, "paper_conf_ppopp_niuljs0022_b200", "csrc")
+    kernels, missing = 0, []
+    for f in sorted(os.listdir(csrc)):
+        if not f.endswith(".cu"):
+            continue
+        text = open(os.path.join(csrc, f)).read()
+        assert "<<<" not in text, f"{f}: a kernel launched outside TSG_LAUNCH"
+        for m in re.finditer(r"__global__[^;{]*?\b(k_\w+)\s*\([^;{]*\)\s*\{", text, flags=re.S):
+            kernels += 1
+            if not text[m.end():m.end() + 40].lstrip().startswith("TSG_GRID_WAIT();"):
+                missing.append(f"{f}:{m.group(1)}")
+    assert kernels >= 40 and not missing, missing
+    hdr = open(os.path.join(csrc, "tsg_internal.cuh")).read()
+    assert "griddepcontrol.wait" in hdr and "cudaLaunchAttributeProgrammaticStreamSerialization" in hdr

@@ -653,6 +653,44 @@ def test_free_is_ordered_on_the_producing_stream(tsg):
             assert np.array_equal(got[k], ref[k]), k
 
 
+def test_concurrent_calls_on_two_streams(tsg):
+    """Programmatic dependent launch keeps stream order: two host threads issuing calls on their own
+    streams at the same time (every kernel launched with programmatic serialization, each waiting
+    on its predecessor in its own stream) give the sequential results bit for bit, on both
+    pipelines and on a hypersparse input."""
+    import threading
+
+    import torch
+
+    cases = [(gen.stencil27(14), {}), (gen.strip_fem(6, 20, 6), {}), (gen.rmat(11), {}),
+             (gen.stencil27(12), dict(path_general=True))]
+    tiles = [(tiles_of(tsg, A), o) for A, o in cases]
+    refs = [host(tsg.spgemm(T, T, **o)) for T, o in tiles]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    out = [[None] * len(tiles) for _ in streams]
+
+    def worker(w):
+        with torch.cuda.stream(streams[w]):
+            for rep in range(3):
+                for i in range(len(tiles)):
+                    j = (i + w) % len(tiles)  # the two threads run different cases at once
+                    T, o = tiles[j]
+                    out[w][j] = tsg.spgemm(T, T, stream=streams[w], **o)
+        streams[w].synchronize()
+
+    th = [threading.Thread(target=worker, args=(w,)) for w in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    for w in range(2):
+        for j, ref in enumerate(refs):
+            got = host(out[w][j])
+            for k in ARRAYS[:-1]:
+                assert np.array_equal(got[k], ref[k]), (w, j, k)
+            assert bitwise_equal_values(got["val"], ref["val"]), (w, j)
+
+
 def test_device_partition_matches_host_rule(tsg):
     """tsg_partition_tile_rows: per-tile-row products counted on the device and
     cut at equal shares equal the host-CSR rule, and the total equals the oracle's products."""
