@@ -1,0 +1,37 @@
+"""Warm per-kernel GPU times of tsg_spgemm on one config (torch.profiler / CUPTI, back-to-back
+production calls): where the time of a call goes, kernel by kernel.
+usage: python scripts/kernel_times.py C2 [opts-json]"""
+import json
+import sys
+
+import torch
+from torch.profiler import ProfilerActivity, profile
+
+sys.path.insert(0, ".")
+import paper_conf_ppopp_niuljs0022_b200 as tsg  # noqa: E402
+from workloads import gen  # noqa: E402
+
+cfg = sys.argv[1]
+opts = json.loads(sys.argv[2]) if len(sys.argv) > 2 else {}
+A = gen.config(cfg)
+T = tsg.csr_to_tiles(torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.col).cuda(),
+                     torch.from_numpy(A.val).cuda(), (A.m, A.n))
+for _ in range(3):
+    C = tsg.spgemm(T, T, **opts)
+    del C
+torch.cuda.synchronize()
+N = 5
+with profile(activities=[ProfilerActivity.CUDA]) as prof:
+    for _ in range(N):
+        C = tsg.spgemm(T, T, **opts)
+        del C
+    torch.cuda.synchronize()
+rows = []
+for e in prof.key_averages():
+    if e.device_type is not None and "k_" in e.key and e.self_device_time_total > 0:
+        rows.append((e.self_device_time_total / N, e.count / N, e.key.split("(")[0][-60:]))
+rows.sort(reverse=True)
+tot = sum(r[0] for r in rows)
+print(f"{cfg}: kernel time per call {tot / 1000:.3f} ms")
+for us, cnt, name in rows:
+    print(f"{us:10.1f} us  x{cnt:4.1f}  {100 * us / tot:5.1f}%  {name}")
