@@ -827,7 +827,13 @@ __global__ void __launch_bounds__(ROW_T) k_row_big(S1Params P) { TSG_GRID_WAIT()
 // insertion-sorted by A tile position, i.e. ascending K (reading A8).  Three passes over the
 // candidates (expand once into global scratch, count, scatter) instead of a multi-pass radix sort.
 // ------------------------------------------------------------------------------------------
-constexpr int RANK_T = 512;
+#ifndef TSG_RANK_T
+#define TSG_RANK_T 1024
+#endif
+#ifndef TSG_RANK_CPS
+#define TSG_RANK_CPS 2
+#endif
+constexpr int RANK_T = TSG_RANK_T;  // threads of a bitmap-rank CTA (one wide tile row at a time)
 constexpr int RANK_NW = RANK_T / 32;
 
 __device__ __forceinline__ int64_t block_excl_scan64(int64_t v, int64_t *total, int64_t *sm /* RANK_NW+1 */) {
@@ -1174,7 +1180,7 @@ void launch_row_sort(const S1Params &P, int64_t tm, cudaStream_t s) {
     const size_t smem = (size_t)wwords * 8;
     if (!P.sort_only && smem <= 200 * 1024) {
         TSG_CUDA(cudaFuncSetAttribute(k_row_rank, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        TSG_LAUNCH(k_row_rank, (unsigned)std::min<int64_t>(tm, 4LL * nsm), RANK_T, smem, s, P, (int)wwords);
+        TSG_LAUNCH(k_row_rank, (unsigned)std::min<int64_t>(tm, (int64_t)TSG_RANK_CPS * nsm), RANK_T, smem, s, P, (int)wwords);
     } else {
         TSG_LAUNCH(k_row_big, (unsigned)std::min<int64_t>(tm, 8LL * nsm), ROW_T, 0, s, P);
     }
