@@ -14,7 +14,10 @@ namespace tsg {
 namespace {
 
 constexpr int SCAN_T = 1024;
-constexpr int SCAN_IPT = 8;
+#ifndef TSG_SCAN_IPT
+#define TSG_SCAN_IPT 8
+#endif
+constexpr int SCAN_IPT = TSG_SCAN_IPT;
 constexpr int SCAN_TILE = SCAN_T * SCAN_IPT;
 
 __device__ __forceinline__ int64_t warp_incl_scan(int64_t v) {
@@ -70,10 +73,27 @@ __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n,
     const int64_t base = b * SCAN_TILE + (int64_t)threadIdx.x * SCAN_IPT;
     int64_t v[SCAN_IPT];
     int64_t sum = 0;
+    // a thread's SCAN_IPT consecutive inputs as 16-byte vector loads when the run is whole and
+    // aligned (the element-wise form touches the same lines SCAN_IPT times)
+    const bool vec = base + SCAN_IPT <= n && ((reinterpret_cast<uintptr_t>(in + base) & 15u) == 0);
+    if (vec) {
+        const uint4 *q = reinterpret_cast<const uint4 *>(in + base);
+        constexpr int PER = 16 / (int)sizeof(Tin);
 #pragma unroll
-    for (int i = 0; i < SCAN_IPT; i++) {
-        v[i] = (base + i < n) ? (int64_t)in[base + i] : 0;
-        sum += v[i];
+        for (int k = 0; k < SCAN_IPT / PER; k++) {
+            const uint4 w = q[k];
+            const Tin *e = reinterpret_cast<const Tin *>(&w);
+#pragma unroll
+            for (int i = 0; i < PER; i++) v[k * PER + i] = (int64_t)e[i];
+        }
+#pragma unroll
+        for (int i = 0; i < SCAN_IPT; i++) sum += v[i];
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_IPT; i++) {
+            v[i] = (base + i < n) ? (int64_t)in[base + i] : 0;
+            sum += v[i];
+        }
     }
     int64_t total;
     int64_t pre = block_excl_scan(sum, &total);  // all reads of `in` by this CTA happen before
@@ -103,10 +123,22 @@ __global__ void __launch_bounds__(SCAN_T) k_scan_1pass(const Tin *in, int64_t n,
     }
     __syncthreads();
     pre += s_base;
+    if (base + SCAN_IPT <= n && ((reinterpret_cast<uintptr_t>(out + base) & 15u) == 0)) {
+        uint4 *q = reinterpret_cast<uint4 *>(out + base);
 #pragma unroll
-    for (int i = 0; i < SCAN_IPT; i++) {
-        if (base + i < n) out[base + i] = pre;
-        pre += v[i];
+        for (int k = 0; k < SCAN_IPT / 2; k++) {
+            const int64_t x0 = pre;
+            pre += v[2 * k];
+            const int64_t x1 = pre;
+            pre += v[2 * k + 1];
+            q[k] = make_uint4((unsigned)x0, (unsigned)((uint64_t)x0 >> 32), (unsigned)x1, (unsigned)((uint64_t)x1 >> 32));
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_IPT; i++) {
+            if (base + i < n) out[base + i] = pre;
+            pre += v[i];
+        }
     }
     if (base < n && base + SCAN_IPT >= n) out[n] = pre;  // the thread holding the last element
     if (ex.n && b == (int64_t)gridDim.x - 1) export_segments(ex);  // the CTA that wrote out[n]
