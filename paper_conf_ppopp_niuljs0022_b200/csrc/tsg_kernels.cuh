@@ -33,7 +33,14 @@ struct DevCounters {
 
 constexpr int ROW_T = 256;        // threads of a step-1 row CTA
 constexpr int ROW_NW = ROW_T / 32;
-constexpr int ROW_CAP = 4096;     // max candidates of a row sorted in shared memory
+#ifndef TSG_ROW_CAP
+#define TSG_ROW_CAP 256
+#endif
+// max candidates of a wide row (> 32 A tiles) sorted in shared memory (k_row_small); wider rows take
+// the bitmap rank.  Measured on C4 (25 K such rows, 52 M candidates): 4096 -> 92.1 ms per call,
+// 1024 -> 91.0, 256 -> 90.8 (the rank kernel's two 1024-thread CTAs per SM beat the sort's
+// 61 ps per candidate)
+constexpr int ROW_CAP = TSG_ROW_CAP;
 constexpr int LIGHT_WORK = 16;    // step-2 thread-per-tile class: (pair, c) items of the tile
 constexpr int SMALL_NNZ = 8;      // step-3 lane-per-entry class (k_s3_small): C tile nnz (<= 16)
 constexpr int64_t ROWPATH_SMALL_U = 1 << 20;  // step-1 candidates below which narrow calls take the row path

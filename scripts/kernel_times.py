@@ -36,8 +36,9 @@ with profile(activities=[ProfilerActivity.CUDA]) as prof:
 rows = []
 for e in prof.key_averages():
     if e.device_type is not None and "k_" in e.key and e.self_device_time_total > 0:
-        name = e.key.split("(")[0].replace("void ", "").replace("tsg::(anonymous namespace)::", "")
-        rows.append((e.self_device_time_total / N, e.count / N, name[:60]))
+        import re
+        m = re.search(r"(k_\w+(<[^>]*>)?)", e.key)
+        rows.append((e.self_device_time_total / N, e.count / N, (m.group(1) if m else e.key)[:60]))
 rows.sort(reverse=True)
 tot = sum(r[0] for r in rows)
 ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
