@@ -72,6 +72,7 @@ struct S1Params {
     const int32_t *tcB;
     const uint16_t *rowOccB;
     const uint32_t *list;
+    const int32_t *listJ;     // tile column of each B row list entry (list mode)
     const int32_t *rowJlo;
     const int32_t *rowJhi;
     const uint8_t *rowClass;
@@ -163,12 +164,13 @@ struct StepParams {
 void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint16_t *col_occ, cudaStream_t s,
                       void *zero = nullptr, size_t zero_bytes = 0);  // also zeroes `zero` (the call's counters)
 void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
-                    uint32_t *list, cudaStream_t s);
+                    uint32_t *list, const int32_t *tcB, int32_t *listJ, cudaStream_t s);
 void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int64_t ntA, const int32_t *tcA,
                      const uint16_t *maskA, int32_t *rnnz, DevCounters *cnt, cudaStream_t s);
 void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA, const int64_t *tpB,
-                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, bool scan_only, int64_t *cost,
-                       int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s);
+                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, const int32_t *listJ,
+                       bool scan_only, int64_t *cost, int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt,
+                       cudaStream_t s);
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
                      const int32_t *jhiA, bool merge, int32_t *rowJlo, int32_t *rowJhi, uint8_t *rowClass,
                      int64_t *nC, int32_t *bigList, int64_t *bigOff, int32_t *smallList, DevCounters *cnt,

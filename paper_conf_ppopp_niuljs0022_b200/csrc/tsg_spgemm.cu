@@ -166,13 +166,15 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
                        ((flags & TSG_STEP1_LIST_ALWAYS) || (B->nt > 0 && B->nnz < 2 * B->nt));
     int64_t *lptr = nullptr;
     uint32_t *list = nullptr;
+    int32_t *listJ = nullptr;
     if (lists) {
         int32_t *lcnt = tmp.get<int32_t>(TILE * tmB);
         lptr = tmp.get<int64_t>(TILE * tmB + 1);
         list = tmp.get<uint32_t>(B->nnz);
-        launch_rowlist(tmB, B->tile_ptr, B->mask, nullptr, lcnt, nullptr, s);
+        listJ = tmp.get<int32_t>(B->nnz);
+        launch_rowlist(tmB, B->tile_ptr, B->mask, nullptr, lcnt, nullptr, nullptr, nullptr, s);
         exclusive_scan<int32_t>(lcnt, lptr, TILE * tmB, s, tmp);
-        launch_rowlist(tmB, B->tile_ptr, B->mask, lptr, lcnt, list, s);
+        launch_rowlist(tmB, B->tile_ptr, B->mask, lptr, lcnt, list, B->tile_col, listJ, s);
     }
     // hypersparse operands (fewer than 4 nonzeros per B tile, no small-tile flag): 16-byte per-tile
     // records for step 1's wide rows and steps 2-3 (inB: A's are a slice of B's)
@@ -208,7 +210,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     int64_t *startA = tmp.get<int64_t>(ntA);
     int32_t *jloA = tmp.get<int32_t>(ntA);
     int32_t *jhiA = tmp.get<int32_t>(ntA);
-    launch_atile_plan(ntA, A->tile_col, colOccA, B->tile_ptr, B->tile_col, lptr, list,
+    launch_atile_plan(ntA, A->tile_col, colOccA, B->tile_ptr, B->tile_col, lptr, list, listJ,
                       (bool)(flags & TSG_STEP1_SCAN_ONLY), cost, startA, jloA, jhiA, cnt, s);
     int64_t *costOff = tmp.get<int64_t>(ntA + 1);
     exclusive_scan<int64_t>(cost, costOff, ntA, s, tmp);
@@ -240,6 +242,7 @@ void run_spgemm(const tsg_tiles *A, const tsg_tiles *B, uint32_t flags, const Al
     P1.tcB = B->tile_col;
     P1.rowOccB = rowOccB;
     P1.list = list;
+    P1.listJ = listJ;
     P1.rowJlo = rowJlo;
     P1.rowJhi = rowJhi;
     P1.rowClass = rowClass;

@@ -79,7 +79,8 @@ __global__ void k_tile_records(int64_t nt, const int32_t *__restrict__ tile_col,
 // k%16 is non-empty, ascending tile column.  One warp = two B tile rows, lane r = row r.
 __global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__restrict__ tpB,
                                                  const uint16_t *__restrict__ maskB, const int64_t *__restrict__ lptr,
-                                                 int32_t *__restrict__ lcnt, uint32_t *__restrict__ list) { TSG_GRID_WAIT();
+                                                 int32_t *__restrict__ lcnt, uint32_t *__restrict__ list,
+                                                 const int32_t *__restrict__ tcB, int32_t *__restrict__ listJ) { TSG_GRID_WAIT();
     const int lane = threadIdx.x & 31, r = lane & 15;
     const int64_t K = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + (lane >> 4);
     if (K >= tmB) return;
@@ -89,9 +90,13 @@ __global__ void __launch_bounds__(256) k_rowlist(int64_t tmB, const int64_t *__r
         for (int64_t t = t0; t < t1; t++) c += maskB[t * TILE + r] != 0;
         lcnt[K * TILE + r] = c;
     } else {
+        // the entries' tile columns alongside (step 1 reads them without a dependent lookup)
         int64_t pos = lptr[K * TILE + r];
         for (int64_t t = t0; t < t1; t++)
-            if (maskB[t * TILE + r]) list[pos++] = (uint32_t)t;
+            if (maskB[t * TILE + r]) {
+                list[pos] = (uint32_t)t;
+                listJ[pos++] = tcB[t];
+            }
     }
 }
 
@@ -209,7 +214,8 @@ __global__ void k_cuts(const int64_t *__restrict__ pre, int64_t tm, int64_t part
 // ------------------------------------------------------------------------------------------
 __global__ void k_atile_plan(int64_t ntA, const int32_t *__restrict__ tcA, const uint16_t *__restrict__ colOccA,
                              const int64_t *__restrict__ tpB, const int32_t *__restrict__ tcB,
-                             const int64_t *__restrict__ lptr, const uint32_t *__restrict__ list, bool scan_only,
+                             const int64_t *__restrict__ lptr, const uint32_t *__restrict__ list,
+                             const int32_t *__restrict__ listJ, bool scan_only,
                              int64_t *__restrict__ cost, int64_t *__restrict__ start, int32_t *__restrict__ jlo,
                              int32_t *__restrict__ jhi, DevCounters *cnt) { TSG_GRID_WAIT();
     int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -230,9 +236,8 @@ __global__ void k_atile_plan(int64_t ntA, const int32_t *__restrict__ tcA, const
         cost[t] = len;
         start[t] = is_list ? -(st + 1) : st;
         if (len > 0) {
-            int64_t f = is_list ? (int64_t)list[st] : st, l = is_list ? (int64_t)list[st + len - 1] : st + len - 1;
-            jlo[t] = tcB[f];
-            jhi[t] = tcB[l];
+            jlo[t] = is_list ? listJ[st] : tcB[st];
+            jhi[t] = is_list ? listJ[st + len - 1] : tcB[st + len - 1];
         } else {
             jlo[t] = 0x7fffffff;
             jhi[t] = -1;
@@ -560,7 +565,7 @@ __device__ uint32_t merge_row(const S1Params &P, int64_t I, int lane, uint32_t *
             const uint32_t pos = isl ? lst[k] : st32 + (uint32_t)k;
             const uint32_t wk = isl ? 1u : (uint32_t)__popc(co & (uint32_t)P.rowOccB[pos]);
             if (wk) {
-                sJw[cntv] = (uint32_t)P.tcB[pos] | (wk << 27);
+                sJw[cntv] = (uint32_t)(isl ? P.listJ[st + k] : P.tcB[pos]) | (wk << 27);
                 sKw[cntv] = (uint16_t)k;
                 cntv++;
             }
@@ -914,7 +919,7 @@ __device__ void rank_row_big(const S1Params &P, int64_t I, int wwords, uint32_t 
                 occ = P.rowOccB[posB];
                 valid = (occ & co) != 0;
             }
-            const uint32_t jr = valid ? (uint32_t)(P.tcB[posB] - jlo) : ~0u;
+            const uint32_t jr = valid ? (uint32_t)((st < 0 ? P.listJ[-st - 1 + s] : P.tcB[posB]) - jlo) : ~0u;
             // the candidate's (pair, c) items (step 2's work estimate) ride in the top 5 bits
             const uint32_t wk = st < 0 ? 1u : (uint32_t)__popc(occ & co);
             sJ[u] = valid ? jr | (wk << 27) : ~0u;
@@ -1100,8 +1105,8 @@ void launch_occupancy(const uint16_t *mask, int64_t nt, uint16_t *row_occ, uint1
 }
 
 void launch_rowlist(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, const int64_t *lptr, int32_t *lcnt,
-                    uint32_t *list, cudaStream_t s) {
-    TSG_LAUNCH(k_rowlist, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, lptr, lcnt, list);
+                    uint32_t *list, const int32_t *tcB, int32_t *listJ, cudaStream_t s) {
+    TSG_LAUNCH(k_rowlist, grid_for(ceil_div(tmB, 2), 8), 256, 0, s, tmB, tpB, maskB, lptr, lcnt, list, tcB, listJ);
 }
 
 void launch_row_products(int64_t tmA, const int64_t *tpA, const int32_t *tcA, const uint16_t *maskA, int64_t tmB,
@@ -1121,10 +1126,11 @@ void launch_products(int64_t tmB, const int64_t *tpB, const uint16_t *maskB, int
 }
 
 void launch_atile_plan(int64_t ntA, const int32_t *tcA, const uint16_t *colOccA, const int64_t *tpB,
-                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, bool scan_only, int64_t *cost,
-                       int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt, cudaStream_t s) {
-    TSG_LAUNCH(k_atile_plan, grid_for(ntA, 256), 256, 0, s, ntA, tcA, colOccA, tpB, tcB, lptr, list, scan_only, cost,
-               start, jlo, jhi, cnt);
+                       const int32_t *tcB, const int64_t *lptr, const uint32_t *list, const int32_t *listJ,
+                       bool scan_only, int64_t *cost, int64_t *start, int32_t *jlo, int32_t *jhi, DevCounters *cnt,
+                       cudaStream_t s) {
+    TSG_LAUNCH(k_atile_plan, grid_for(ntA, 256), 256, 0, s, ntA, tcA, colOccA, tpB, tcB, lptr, list, listJ, scan_only,
+               cost, start, jlo, jhi, cnt);
 }
 
 void launch_row_plan(int64_t tmA, const int64_t *tpA, const int64_t *costOff, const int32_t *jloA,
