@@ -174,7 +174,10 @@ __global__ void __launch_bounds__(T2L, 8) k_s2_light(StepParams P) { TSG_GRID_WA
     if ((threadIdx.x & 31) == 0 && nd) atomicAdd(&P.cnt->n2dense, nd);
 }
 
-__global__ void __launch_bounds__(T2) k_s2(StepParams P) { TSG_GRID_WAIT();
+#ifndef TSG_S2_MINB
+#define TSG_S2_MINB 1
+#endif
+__global__ void __launch_bounds__(T2, TSG_S2_MINB) k_s2(StepParams P) { TSG_GRID_WAIT();
     __shared__ __align__(16) uint16_t sMA[T2 / 16][BATCH][TILE], sMB[T2 / 16][BATCH][TILE];
     __shared__ uint16_t sOB[T2 / 16][BATCH];
     const int lane = threadIdx.x & 31, r = lane & 15, half = lane >> 4, hw = threadIdx.x >> 4;
@@ -292,7 +295,7 @@ constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <=
 // product's B address needs a shared load instead of a dependent global one.  On cache-friendly
 // inputs (stencils: B's metadata hits L1) the staging is pure overhead and STAGE is off.
 #ifndef TSG_SMALL_MINB
-#define TSG_SMALL_MINB 5
+#define TSG_SMALL_MINB 6
 #endif
 // REC (hypersparse operands, the default there): per pair the two tiles' 16-byte records; a
 // single-nonzero tile needs nothing else (its entry and value are inline), a multi-nonzero tile
