@@ -523,7 +523,10 @@ struct MergeOut {
 #define TSG_MERGE_W 4
 #endif
 constexpr int MERGE_W = TSG_MERGE_W;  // warps (tile rows) per merge CTA
-constexpr int MERGE_CAP = 1024;  // candidates of a row staged in shared memory (6 B each)
+#ifndef TSG_MERGE_CAP
+#define TSG_MERGE_CAP 768
+#endif
+constexpr int MERGE_CAP = TSG_MERGE_CAP;  // candidates of a row staged in shared memory (6 B each)
 
 // One tile row's merge by one warp (sJw / sKw: the warp's MERGE_CAP staging slots).  Writes the
 // row's pairs and C tile records at its candidate-space slots; returns the row's C tile count
@@ -651,7 +654,10 @@ __device__ uint32_t merge_row(const S1Params &P, int64_t I, int lane, uint32_t *
     return out.ntl;
 }
 
-__global__ void __launch_bounds__(MERGE_W * 32) k_row_merge(S1Params P, int64_t tm) { TSG_GRID_WAIT();
+#ifndef TSG_MERGE_MINB
+#define TSG_MERGE_MINB 1
+#endif
+__global__ void __launch_bounds__(MERGE_W * 32, TSG_MERGE_MINB) k_row_merge(S1Params P, int64_t tm) { TSG_GRID_WAIT();
     __shared__ uint32_t sJ[MERGE_W][MERGE_CAP];
     __shared__ uint16_t sK[MERGE_W][MERGE_CAP];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
