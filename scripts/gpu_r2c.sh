@@ -6,8 +6,8 @@ if [ "${STAGE:-1}" = "1" ]; then
   nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/r2c_smi.txt 2>&1
   timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -15 > gpurun_out/r2c_pytest.log
   timeout 600 python bench.py > gpurun_out/r2c_bench_default.json 2> gpurun_out/r2c_bench_default.err
-  timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/r2c_bench_ref.json 2> gpurun_out/r2c_bench_ref.err
   timeout 600 python bench.py --config C1 --steps 50 --warmup 5 --no-cpu-baseline --e2e-steps 0 > gpurun_out/r2c_bench_C1.json 2> gpurun_out/r2c_bench_C1.err
+  timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/r2c_bench_ref.json 2> gpurun_out/r2c_bench_ref.err
   for c in C3 C4; do
     timeout 600 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/r2c_bench_$c.json 2> gpurun_out/r2c_bench_$c.err
   done
@@ -26,8 +26,10 @@ elif [ "${STAGE}" = "2" ]; then
   timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off \
     -k "regex:k_num_dense_row|k_sym_rows|k_num_rows|k_row_merge" -o /tmp/prof_r2c_C3 python scripts/traffic.py C3 > /dev/null 2>&1
   timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off \
-    -k "regex:k_s3<|k_s3_small|k_s2\\b|k_s2\\(|k_row_merge|k_s2_light" -o /tmp/prof_r2c_C2 python scripts/traffic.py C2 > /dev/null 2>&1
-  for c in C2 C3; do
+    -k "regex:^k_s3$|k_s3_small|k_s2$|k_row_merge|k_s2_light" -o /tmp/prof_r2c_C2 python scripts/traffic.py C2 > /dev/null 2>&1
+  timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off \
+    -k "regex:k_row_rank|k_s3_small|k_s2_light" -o /tmp/prof_r2c_C4 python scripts/traffic.py C4 > /dev/null 2>&1
+  for c in C2 C3 C4; do
     python profiles/summarize.py full /tmp/prof_r2c_$c.ncu-rep > gpurun_out/r2c_full_$c.md 2>&1
     sz=$(stat -c %s /tmp/prof_r2c_$c.ncu-rep)
     if [ "$sz" -lt 18000000 ]; then cp /tmp/prof_r2c_$c.ncu-rep gpurun_out/; fi
