@@ -294,8 +294,13 @@ constexpr int SMAP = 32 * 16;  // entry -> tile map bytes per warp (small_max <=
 // 0-7, mask rows 8-15][thread], 16 bytes each) is filled by cp.async one pair ahead, so a
 // product's B address needs a shared load instead of a dependent global one.  On cache-friendly
 // inputs (stencils: B's metadata hits L1) the staging is pure overhead and STAGE is off.
+// CTAs per SM of k_s3_small: 6 for the plain form (C2: 1.26 -> 1.21 ms against 5), 5 for the
+// staged and record forms (C5's record form: step 3 170 ms at 5, 179 at 6; 7+ spills heavily)
 #ifndef TSG_SMALL_MINB
-#define TSG_SMALL_MINB 6
+#define TSG_SMALL_MINB 5
+#endif
+#ifndef TSG_SMALL_MINB_PLAIN
+#define TSG_SMALL_MINB_PLAIN 6
 #endif
 // REC (hypersparse operands, the default there): per pair the two tiles' 16-byte records; a
 // single-nonzero tile needs nothing else (its entry and value are inline), a multi-nonzero tile
@@ -308,7 +313,7 @@ __device__ __forceinline__ TO rec_value(const uint4 &r) {
 }
 
 template <typename TI, typename TO, int MODE>  // MODE 0: plain, 1: STAGE, 2: REC
-__global__ void __launch_bounds__(TS, TSG_SMALL_MINB) k_s3_small(StepParams P) { TSG_GRID_WAIT();
+__global__ void __launch_bounds__(TS, MODE == 0 ? TSG_SMALL_MINB_PLAIN : TSG_SMALL_MINB) k_s3_small(StepParams P) { TSG_GRID_WAIT();
     constexpr bool STAGE = MODE == 1;
     __shared__ uint8_t mapsm[TS / 32][SMAP];
     __shared__ __align__(16) uint4 stg[STAGE ? 2 : 1][3][STAGE ? TS : 1];
